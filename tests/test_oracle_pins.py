@@ -1,0 +1,294 @@
+"""Pins of the CPU oracle against what the paper and the mathematics fix (no GPU).
+
+Each test names the plausible oracle mistake it would catch.
+"""
+import json
+import os
+from collections import OrderedDict
+
+import numpy as np
+import pytest
+
+from oracle import oracle as O
+from tests import che
+from workload import configs, gen
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def _tiny_tables(cards, dims, mode=0):
+    return [np.ascontiguousarray(t) for t in gen.make_tables(cards, dims, mode)[1]]
+
+
+# ---------------------------------------------------------------- encoder
+def test_size_aware_coding_worked_example():
+    g = json.load(open(os.path.join(GOLD, "size_aware_coding.json")))
+    bmin, base, fb = O.encode(g["cards"], g["key_bits"])
+    assert bmin == g["bmin"]
+    assert fb.tolist() == g["fbits"]
+    assert base.tolist() == g["base"]
+    B = g["key_bits"]
+    prefixes = [format(int(b) >> int(f), "0%db" % (B - int(f))) for b, f in zip(base, fb)]
+    assert prefixes == g["prefix"]
+    # prefix-free: no table-ID code is a prefix of another
+    for i, a in enumerate(prefixes):
+        for j, b in enumerate(prefixes):
+            assert i == j or not b.startswith(a)
+    # brute-force injectivity + decode by prefix match over every (table, id)
+    keys = {}
+    for t, c in enumerate(g["cards"]):
+        for i in range(c):
+            k = int(base[t]) + i
+            assert k < (1 << B) - 1  # all-ones stays free (EMPTY)
+            assert format(k, "0%db" % B).startswith(prefixes[t])
+            assert k not in keys
+            keys[k] = (t, i)
+    assert len(keys) == g["total_keys"] and max(keys) == g["max_key"]
+
+
+def test_size_aware_coding_configs_and_kraft():
+    g = json.load(open(os.path.join(GOLD, "size_aware_coding.json")))
+    for name, bmin_expected in g["config_bmin"].items():
+        w = configs.get(name)
+        bmin, base, fb = O.encode(w.cards)
+        assert bmin == bmin_expected, name
+        # Kraft: sum 2^-L_t <= 1 with the all-ones code reserved
+        assert sum(2 ** int(f) for f in fb) + 1 <= 2 ** 32
+        # each table's key range is disjoint and aligned on 2^f
+        spans = sorted((int(b), int(b) + 2 ** int(f)) for b, f in zip(base, fb))
+        for (a0, a1), (b0, _) in zip(spans, spans[1:]):
+            assert a1 <= b0
+        assert all(int(b) % (2 ** int(f)) == 0 for b, f in zip(base, fb))
+    # too many bits -> rejected (lossy fallback is out of scope)
+    assert O.encode([1 << 20] * 8, 22) is None
+
+
+# --------------------------------------------------------- self-identification (Fig 6)
+def test_fig6_self_identification():
+    g = json.load(open(os.path.join(GOLD, "fig6_self_identification.json")))
+    assert sum(g["threads"]) == g["fused_threads"] == g["scan"][-1]
+    assert g["scan"] == [0] + list(np.cumsum(g["threads"]))
+    for tid, phi, loc in g["cases"]:
+        assert O.self_identify(g["scan"], tid) == (phi, loc)
+    # every tid maps to exactly one (kernel, local) and back
+    seen = set()
+    for tid in range(g["fused_threads"]):
+        phi, loc = O.self_identify(g["scan"], tid)
+        assert 0 <= loc < g["threads"][phi]
+        seen.add((phi, loc))
+    assert len(seen) == g["fused_threads"]
+
+
+def test_self_identification_skips_empty_kernels():
+    scan = [0, 0, 5, 5, 5, 7]
+    assert [O.self_identify(scan, t) for t in range(7)] == [(1, 0), (1, 1), (1, 2), (1, 3), (1, 4), (4, 0), (4, 1)]
+
+
+# --------------------------------------------------------------- values (definition)
+@pytest.mark.parametrize("mode", [0, 1])
+def test_one_hot_values_are_direct_lookups(mode):
+    w = configs.get("cfg0").with_(invalid_ppm=20000, value_mode=mode)
+    tabs = _tiny_tables(w.cards, w.dims, mode)
+    o = O.Oracle(w.cards, w.dims, tabs, w.cache_bytes)
+    for b in range(3):
+        bt = w.batch(b)
+        out = o.query(bt.ids)
+        off = 0
+        for t, ids in enumerate(bt.ids):
+            d = w.dims[t]
+            ref = np.zeros((ids.size, d), np.float32)
+            ok = (ids >= 0) & (ids < w.cards[t])
+            ref[ok] = tabs[t][ids[ok]]
+            got = out[off: off + ids.size * d].reshape(ids.size, d)
+            assert np.array_equal(got.view(np.uint32), ref.view(np.uint32))
+            off += ids.size * d
+    s = o.stats()
+    assert s["invalid"] > 0 and s["hits"] + s["misses"] + s["invalid"] == s["lookups"]
+
+
+def test_pooled_sum_exact_on_grid():
+    # grid values: every fp32 partial sum is exact, so the sequential fp32 bag sum
+    # must equal the fp64 sum exactly (catches dropped / repeated terms, wrong rows)
+    cards, dims = [1000, 50, 7], [8, 16, 4]
+    tabs = _tiny_tables(cards, dims, 0)
+    o = O.Oracle(cards, dims, tabs, 4096)
+    rng = np.random.default_rng(1)
+    offs, ids = [], []
+    for t in range(3):
+        L = rng.integers(0, 9, size=40)
+        off = np.concatenate([[0], np.cumsum(L)]).astype(np.int64)
+        x = rng.integers(-2, cards[t] + 2, size=off[-1]).astype(np.int64)
+        offs.append(off)
+        ids.append(x)
+    out = o.query_pooled(ids, offs)
+    p = 0
+    for t in range(3):
+        d = dims[t]
+        for b in range(40):
+            ref = np.zeros(d, np.float64)
+            for i in ids[t][offs[t][b]:offs[t][b + 1]]:
+                if 0 <= i < cards[t]:
+                    ref += tabs[t][i].astype(np.float64)
+            assert np.array_equal(out[p: p + d].astype(np.float64), ref)
+            p += d
+
+
+# ------------------------------------------------------------- policy: worked example
+@pytest.mark.parametrize("mode", [O.MODE_GLOBAL])
+def test_hand_worked_example(mode):
+    g = json.load(open(os.path.join(GOLD, "hand_example.json")))
+    tabs = _tiny_tables(g["cards"], g["dims"])
+    o = O.Oracle(g["cards"], g["dims"], tabs, g["cache_bytes"], mode)
+    prev = set()
+    tot_hits = 0
+    for bt in g["batches"]:
+        before = o.stats()
+        o.query([np.array(x, np.int64) for x in bt["ids"]])
+        s = o.stats()
+        hits = s["hits"] - before["hits"]
+        assert hits == bt["hits"]
+        assert (s["hits"] + s["misses"]) - (before["hits"] + before["misses"]) == bt["valid"]
+        assert s["invalid"] - before["invalid"] == bt.get("invalid", 0)
+        assert s["occupancy_bytes"] == bt["occupancy"] <= g["cache_bytes"]
+        now = set(map(tuple, o.cached_keys()))
+        evicted = prev - now
+        assert evicted == set(map(tuple, bt["evicted"]))
+        prev = now
+        tot_hits += hits
+    assert tot_hits == g["total_hits"]
+    assert prev == set(map(tuple, g["final_cached"]))
+
+
+# ------------------------------------------------------- policy: textbook reductions
+def _textbook_lru(stream, cap):
+    lru, hits = OrderedDict(), []
+    for k in stream:
+        h = k in lru
+        hits.append(h)
+        if h:
+            lru.move_to_end(k)
+        else:
+            if len(lru) >= cap:
+                lru.popitem(last=False)
+            lru[k] = True
+    return hits
+
+
+@pytest.mark.parametrize("mode,cap", [(O.MODE_GLOBAL, 10), (O.MODE_GLOBAL, 37), (O.MODE_SETASSOC, 32),
+                                      (O.MODE_SETASSOC, 10)])
+def test_one_lookup_per_batch_is_textbook_lru(mode, cap):
+    # one lookup per batch, uniform dim: every ts is distinct, epoch protection never
+    # binds, so the policy must be exactly LRU (with S = 1 set in set-assoc mode)
+    c, d = 200, 4
+    tabs = _tiny_tables([c], [d])
+    o = O.Oracle([c], [d], tabs, cap * 4 * d, mode, hash_seed=7)
+    rng = np.random.default_rng(5)
+    hot = rng.integers(0, 15, size=3000)
+    cold = rng.integers(0, c, size=3000)
+    stream = np.where(rng.random(3000) < 0.7, hot, cold).astype(np.int64)
+    got = []
+    for k in stream:
+        h0 = o.stats()["hits"]
+        o.query([np.array([k], np.int64)])
+        got.append(o.stats()["hits"] - h0 == 1)
+    assert got == _textbook_lru(stream.tolist(), cap)
+
+
+@pytest.mark.parametrize("mode", [O.MODE_GLOBAL, O.MODE_SETASSOC])
+def test_full_capacity_hits_are_repeat_keys(mode):
+    # capacity >= all rows: nothing is ever evicted, so a lookup hits iff its key was
+    # seen in an EARLIER batch (pre-batch state) -- a set-membership closed form
+    w = configs.get("cfg0").with_(dims=[32] * 7)
+    tabs = _tiny_tables(w.cards, w.dims)
+    o = O.Oracle(w.cards, w.dims, tabs, w.table_bytes + 4096 * 32 * 4, mode)
+    seen = set()
+    for b in range(6):
+        bt = w.batch(b)
+        h0 = o.stats()["hits"]
+        o.query(bt.ids)
+        exp = sum(1 for t, x in enumerate(bt.ids) for i in x.tolist() if (t, i) in seen)
+        assert o.stats()["hits"] - h0 == exp
+        seen |= {(t, i) for t, x in enumerate(bt.ids) for i in x.tolist()}
+        assert o.stats()["evicted"] == 0
+
+
+def test_zero_capacity_never_hits():
+    w = configs.get("cfg0")
+    tabs = _tiny_tables(w.cards, w.dims)
+    o = O.Oracle(w.cards, w.dims, tabs, 0)
+    for b in range(3):
+        o.query(w.batch(b).ids)
+    s = o.stats()
+    assert s["hits"] == 0 and s["inserted"] == 0 and s["bypassed"] == s["unique_misses"] > 0
+
+
+def test_admission_probability():
+    # probability-p filter: the inserted fraction of unique misses ~ p
+    w = configs.get("cfg0")
+    tabs = _tiny_tables(w.cards, w.dims)
+    o = O.Oracle(w.cards, w.dims, tabs, w.table_bytes, admit_p=0.25, admit_seed=gen.seeds()["admit"])
+    for b in range(4):
+        o.query(w.batch(b).ids)
+    s = o.stats()
+    n = s["unique_misses"]
+    frac = s["inserted"] / n
+    assert abs(frac - 0.25) < 4 * np.sqrt(0.25 * 0.75 / n)
+    assert s["inserted"] + s["bypassed"] == n
+
+
+# -------------------------------------------------- policy: invariants under churn
+@pytest.mark.parametrize("mode", [O.MODE_GLOBAL, O.MODE_SETASSOC])
+def test_occupancy_invariant_and_no_duplicates(mode):
+    w = configs.get("cfg0").with_(skews=[0.5] * 7, dims=[16] * 7, cache_frac=0.01, invalid_ppm=3000)
+    tabs = _tiny_tables(w.cards, w.dims)
+    o = O.Oracle(w.cards, w.dims, tabs, w.cache_bytes, mode, hash_seed=3)
+    for b in range(40):
+        o.query(w.batch(b).ids)
+        s = o.stats()
+        keys = o.cached_keys()
+        assert len(keys) == len(set(keys))
+        assert s["occupancy_bytes"] == sum(4 * w.dims[t] for t, _ in keys) <= s["capacity_bytes"]
+        assert all(0 <= i < w.cards[t] for t, i in keys)
+        assert s["inserted"] - s["evicted"] == len(keys)
+
+
+# ----------------------------------------------------- policy: steady state vs Che
+def _window_hit(w, mode, warm, measure, hash_seed=0):
+    tabs = w.make_tables()[1]
+    o = O.Oracle(w.cards, w.dims, tabs, w.cache_bytes, mode, hash_seed=hash_seed)
+    for b in range(warm):
+        o.query(w.batch(b).ids)
+    s0 = o.stats()
+    for b in range(warm, warm + measure):
+        o.query(w.batch(b).ids)
+    s1 = o.stats()
+    d = {k: s1[k] - s0[k] for k in s1}
+    return d["hits"] / (d["hits"] + d["misses"]), d
+
+
+@pytest.mark.slow
+def test_cfg1_steady_state_matches_che():
+    # Che closed form for cfg1 (SURVEY c-6): 0.795; IRM optimum 0.853 bounds it.
+    w = configs.get("cfg1")
+    rows = w.cache_bytes // 128
+    ref = che.che_hit(w.cards, w.skews, rows)
+    assert abs(ref - 0.795) < 1e-3
+    hg, dg = _window_hit(w, O.MODE_GLOBAL, 80, 60)
+    assert abs(hg - ref) < 0.01, (hg, ref)
+    assert hg < che.irm_optimum(w.cards, w.skews, rows)
+    # unique keys per batch ~ sum(1 - exp(-p N))
+    assert abs(dg["unique_keys"] / 60 - che.expected_unique(w.cards, w.skews, 1024)) < 0.01 * 14587
+    # the set-associative mode stays within 0.3 pp of the global policy (32 ways)
+    hs, ds = _window_hit(w, O.MODE_SETASSOC, 80, 60, hash_seed=0x9E3779B9)
+    assert abs(hs - hg) < 0.003, (hs, hg)
+    assert ds["bypassed"] == 0
+
+
+def test_small_cache_steady_state_matches_che():
+    # a quick Che pin at a different skew / capacity (a = 0.8, 2 %): catches a wrong
+    # victim choice (e.g. MRU or random) or a missing ts refresh on hit
+    w = configs.get("cfg0").with_(cards=[20000] * 4, dims=[8] * 4, skews=[0.8] * 4, batch_size=256,
+                                  cache_frac=0.02)
+    ref = che.che_hit(w.cards, w.skews, w.cache_bytes // 32)
+    h, _ = _window_hit(w, O.MODE_GLOBAL, 150, 150)
+    assert abs(h - ref) < 0.01, (h, ref)
