@@ -5,7 +5,7 @@ PKG     := paper_conf_eurosys_xiellwgrs22_b200
 CFLAGS  := -O2 -fPIC -shared -fopenmp -Wall -Wextra
 NVFLAGS := $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC,-Wall -shared -cudart static -Iinclude
 
-all: workload/libflgen.so oracle/libfleche_oracle.so
+all: workload/libflgen.so oracle/libfleche_oracle.so $(PKG)/libfleche.so
 
 workload/libflgen.so: workload/gen.c
 	gcc $(CFLAGS) -o $@ $< -lm

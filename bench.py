@@ -1,0 +1,406 @@
+#!/usr/bin/env python
+"""bench.py — keys/s of the flat-cache lookup path on BASELINE configs[1] (cfg2).
+
+One step = one batch of the whole hot path: KQ (fused
+self-identified probe + hit gather + miss dedup + zero-copy host fetch) and KI
+(dup fill + admission + per-set LRU insert), through the C ABI (libfleche.so).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config cfg2] [--impl fleche|reference]
+
+N > 1 runs under torchrun: every rank serves its own shard of each global batch
+with its own replicated cache (no data-path collective; "scaling": "weak").
+`--impl reference` times the CPU oracle (oracle/) on the same workload, rank 0 only.
+"""
+from __future__ import annotations
+
+import argparse
+import faulthandler
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+from workload import configs  # noqa: E402
+
+PREFILL = {"cfg0": 20, "cfg1": 150, "cfg2": 300, "cfg5": 60}
+HASH_SEED = 0x9E3779B9
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=1000)
+    p.add_argument("--warmup", type=int, default=20)
+    p.add_argument("--config", default="cfg2")
+    p.add_argument("--impl", default="fleche", choices=["fleche", "reference"])
+    p.add_argument("--prefill", type=int, default=None, help="untimed batches to reach steady state")
+    p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--cpu-seconds", type=float, default=15.0, help="oracle sample budget")
+    return p.parse_args()
+
+
+def peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        return {"hbm_gbs": 6650.0, "_fallback": True}
+
+
+class ClockSampler:
+    """Samples SM clock and throttle reasons via NVML during the timed region."""
+
+    def __init__(self, device_index: int):
+        self.samples, self.ok = [], False
+        try:
+            import pynvml
+            import torch
+            pynvml.nvmlInit()
+            uuid = "GPU-" + str(torch.cuda.get_device_properties(device_index).uuid)
+            self.h = pynvml.nvmlDeviceGetHandleByUUID(uuid.encode())
+            self.nv = pynvml
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception as e:  # pragma: no cover
+            self.err = repr(e)
+        self._stop = threading.Event()
+        self.window = None
+
+    def _run(self):
+        nv = self.nv
+        while not self._stop.is_set():
+            try:
+                mhz = nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM)
+                r = nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                self.samples.append((time.perf_counter(), mhz, r))
+            except Exception:
+                pass
+            time.sleep(0.01)
+
+    def start(self):
+        if self.ok:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+
+    def mark(self, t0, t1):
+        self.window = (t0, t1)
+
+    def stop(self):
+        if not self.ok:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvml unavailable"]}
+        self._stop.set()
+        self.t.join()
+        nv = self.nv
+        t0, t1 = self.window or (0, 1e30)
+        pad = max(0.05, 0.0)
+        sel = [s for s in self.samples if t0 - pad <= s[0] <= t1 + pad] or self.samples
+        names = {
+            "gpu_idle": getattr(nv, "nvmlClocksEventReasonGpuIdle", 0x1),
+            "sw_power_cap": getattr(nv, "nvmlClocksEventReasonSwPowerCap", 0x4),
+            "hw_slowdown": getattr(nv, "nvmlClocksEventReasonHwSlowdown", 0x8),
+            "sw_thermal_slowdown": getattr(nv, "nvmlClocksEventReasonSwThermalSlowdown", 0x20),
+            "hw_thermal_slowdown": getattr(nv, "nvmlClocksEventReasonHwThermalSlowdown", 0x40),
+            "hw_power_brake_slowdown": getattr(nv, "nvmlClocksEventReasonHwPowerBrakeSlowdown", 0x80),
+        }
+        seen = set()
+        for _, _, r in sel:
+            for k, bit in names.items():
+                if r & bit and k != "gpu_idle":
+                    seen.add(k)
+        return {"sm_mhz": statistics.median([s[1] for s in sel]), "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(seen), "samples": len(sel)}
+
+
+def algorithmic_bytes(st: dict, n_queries: int, d: int) -> dict:
+    """Per-launch algorithmic bytes of KQ and KI."""
+    q = max(n_queries, 1)
+    N = st["lookups"] / q
+    U = st["unique_keys"] / q
+    Uh = st["unique_hits"] / q
+    Um = st["unique_misses"] / q
+    Ui = st["inserted"] / q
+    Nd = (st["misses"] - st["unique_misses"]) / q  # duplicate misses (restored in KI)
+    Nm = st["misses"] / q  # missed lookups (owners + duplicates)
+    row = 4 * d
+    # KQ: IDs in, one 128 B set line per unique key, hit rows read + ts sector touched,
+    #     out rows written for every non-missed lookup, 8 B dedup tag + 24 B record per unique miss
+    kq_hbm = N * 8 + U * 128 + Uh * (row + 32) + (N - Nm) * row + Um * (8 + 24) + Nd * 24
+    # KM: miss record in, host row in (host link), owner + duplicate out rows written,
+    #     per insert: the set's key+ts lines (256 B) read, the row and key/ts written
+    km_host = Um * row
+    km_hbm = Um * 24 + Nd * 16 + (Um + Nd) * row + Ui * (256 + row + 8)
+    return {"N": N, "U": U, "U_hit": Uh, "U_miss": Um, "U_ins": Ui, "kq_hbm": kq_hbm, "km_host": km_host,
+            "km_hbm": km_hbm}
+
+
+def run_reference(args, w, P, W, K):
+    """CPU oracle on the same workload (the reference arm for this tier), rank 0 only."""
+    from oracle import oracle as O
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    t_gen = time.time()
+    _, tabs = w.make_tables()
+    t_gen = time.time() - t_gen
+    orc = O.Oracle(w.cards, w.dims, tabs, w.cache_bytes, O.MODE_GLOBAL)
+    for b in range(P + W):
+        orc.query(w.batch(b).ids)
+    batches = [w.batch(P + W + k).ids for k in range(K)]
+    s0 = orc.stats()
+    t0 = time.perf_counter()
+    for ids in batches:
+        orc.query(ids)
+    dt = time.perf_counter() - t0
+    s1 = orc.stats()
+    lk = s1["lookups"] - s0["lookups"]
+    v = lk / dt / 1e6
+    hits = s1["hits"] - s0["hits"]
+    print(json.dumps({
+        "impl": "reference", "metric": "embedding lookups/s", "value": v, "unit": "Mkeys/s", "n_gpus": args.gpus,
+        "steps": K, "warmup": W, "ms_per_step": dt / K * 1e3, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+        "config": {"workload": w.name, "tables": w.n, "dim": w.dims[0], "batch": w.batch_size,
+                   "lookups_per_step": w.batch_size * w.n, "cache_frac": w.cache_frac, "prefill_batches": P},
+        "hit_ratio": hits / max(1, hits + s1["misses"] - s0["misses"]),
+        "cpu_baseline": {"value": v, "unit": "Mkeys/s", "cores": 1, "kind": "oracle",
+                         "sample": f"{K} full batches of {w.name} after {P + W} untimed batches; single-threaded "
+                                   f"C++ oracle (global byte-LRU policy); host tables generated in {t_gen:.0f}s"},
+        "e2e": {"value": v, "unit": "Mkeys/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }), flush=True)
+
+
+def cpu_baseline(w, tabs, budget_s):
+    """Oracle timed on a bounded sample of the same workload (cold start, batches 0..B-1)."""
+    from oracle import oracle as O
+    orc = O.Oracle(w.cards, w.dims, tabs, w.cache_bytes, O.MODE_GLOBAL)
+    t0 = time.perf_counter()
+    nb, lk = 0, 0
+    gen_t = 0.0
+    while time.perf_counter() - t0 - gen_t < budget_s:
+        tg = time.perf_counter()
+        ids = w.batch(nb).ids
+        gen_t += time.perf_counter() - tg
+        orc.query(ids)
+        nb += 1
+        lk += sum(x.size for x in ids)
+    dt = time.perf_counter() - t0 - gen_t
+    return {"value": lk / dt / 1e6, "unit": "Mkeys/s", "cores": 1, "kind": "oracle",
+            "sample": f"batches 0..{nb - 1} of {w.name} from a cold cache ({lk} lookups, {dt:.1f}s CPU), "
+                      f"single-threaded C++ oracle, 1 of {os.cpu_count()} host cores"}
+
+
+def log(*a):
+    print(f"[bench {time.strftime('%H:%M:%S')}]", *a, file=sys.stderr, flush=True)
+
+
+def main():
+    faulthandler.enable()
+    args = parse()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    w = configs.get(args.config)
+    P = PREFILL.get(args.config, 300) if args.prefill is None else args.prefill
+    W, K = max(args.warmup, 0), max(args.steps, 1)
+    if args.impl == "reference":
+        return run_reference(args, w, P, W, K)
+
+    import torch
+    import paper_conf_eurosys_xiellwgrs22_b200 as fl
+    torch.cuda.set_device(local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
+    N = w.batch_size * w.n
+    d = w.dims[0]
+
+    # host tier: every table in one buffer, page-locked + mapped by fleche_create
+    log("host tier")
+    t_gen = time.time()
+    hostbuf, tabs = w.make_tables()
+    t_gen = time.time() - t_gen
+    log("create")
+    cache = fl.FlatCache(w.cards, w.dims, tabs, w.cache_bytes, N, local, 1.0, 0, HASH_SEED)
+    stream = torch.cuda.current_stream()
+
+    def gen_batch(b):
+        return np.concatenate(w.batch(b, rank=rank).ids)
+
+    lens = [w.batch_size] * w.n
+
+    def views(t):
+        return [t[i * w.batch_size:(i + 1) * w.batch_size] for i in range(w.n)]
+
+    # steady state: untimed prefill batches
+    stage = torch.empty(N, dtype=torch.int64, device=dev)
+    outs = [torch.empty(N * d, dtype=torch.float32, device=dev) for _ in range(4)]  # 4 x out > L2 when N*d*4 large
+    log("prefill")
+    for b in range(P):
+        stage.copy_(torch.from_numpy(gen_batch(b)))
+        cache.query(views(stage), outs[b % 4])
+    torch.cuda.synchronize()
+
+    # pre-generated device-resident batches for warm-up, timed and profiled passes
+    log("pregen")
+    KP = min(K, 300)
+    ids_dev = torch.empty((W + K + KP, N), dtype=torch.int64, device=dev)
+    for i in range(W + K + KP):
+        ids_dev[i].copy_(torch.from_numpy(gen_batch(P + i)))
+    torch.cuda.synchronize()
+
+    log("timed")
+    clock = ClockSampler(local)
+    clock.start()
+    for i in range(W):
+        cache.query(views(ids_dev[i]), outs[i % 4])
+    torch.cuda.synchronize()
+    if dist:
+        dist.barrier()
+    s0 = cache.stats()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    tw0 = time.perf_counter()
+    e0.record(stream)
+    for k in range(K):
+        cache.query(views(ids_dev[W + k]), outs[k % 4])
+    e1.record(stream)
+    torch.cuda.synchronize()
+    tw1 = time.perf_counter()
+    clock.mark(tw0, tw1)
+    if dist:
+        dist.barrier()
+    ms = e0.elapsed_time(e1)
+    s1 = cache.stats()
+    clk = clock.stop()
+    ms_max = ms
+    if dist:
+        t = torch.tensor([ms], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms_max = float(t.item())
+    dst = {k: s1[k] - s0[k] for k in fl.STAT_FIELDS}
+    keys_total = dst["lookups"] * world
+    value = keys_total / (ms_max * 1e-3) / 1e6
+    hit = dst["hits"] / max(1, dst["hits"] + dst["misses"])
+    uhit = dst["unique_hits"] / max(1, dst["unique_keys"])
+
+    # per-kernel device time (profiled pass: CUDA events on the launching stream)
+    log("profiled pass")
+    cache.set_profiling(True)
+    sp0 = cache.stats()
+    for k in range(KP):
+        cache.query(views(ids_dev[W + K + k]), outs[k % 4])
+    torch.cuda.synchronize()
+    kq_ms, ki_ms, nq = cache.kernel_times()
+    sp1 = cache.stats()
+    cache.set_profiling(False)
+    dsp = {k: sp1[k] - sp0[k] for k in fl.STAT_FIELDS}
+    kq_avg, ki_avg = kq_ms / nq, ki_ms / nq
+    ab = algorithmic_bytes(dsp, nq, d)
+
+    # host-link peaks, both measured in-run with KM's access pattern (16 B vector loads,
+    # one row per lane) over rows of 4d bytes: (a) uniformly random rows over the WHOLE host
+    # tier = the ceiling for this workload's misses (large spans are limited by address
+    # translation, ~80-90 M rows/s on this platform: profiles/hostlink_r01.json);
+    # (b) random rows inside a 1 GiB window = the link's bandwidth
+    log("host probe")
+    hp = int(hostbuf.ctypes.data)
+    host_rand = fl.binding.probe_host_read(hp, int(hostbuf.nbytes), 4 * d, 1 << 21, 7)
+    host_link = fl.binding.probe_host_read(hp, min(1 << 30, int(hostbuf.nbytes)), 4 * d, 1 << 21, 9)
+    hbm_peak = float(peaks().get("hbm_gbs", 6650.0))
+    kern = {
+        "kq_kernel": {"ms": kq_avg, "bound": "hbm", "bytes": ab["kq_hbm"], "peak": hbm_peak,
+                      "peak_source": "MEASURED_PEAKS.json hbm_gbs (of measured)"},
+        "km_kernel": {"ms": ki_avg, "bound": "host_link", "bytes": ab["km_host"], "peak": host_rand,
+                      "peak_source": "measured in-run: random-row zero-copy read over the whole host tier",
+                      "hbm_bytes": ab["km_hbm"]},
+    }
+    for kd in kern.values():
+        kd["achieved"] = kd["bytes"] / (kd["ms"] * 1e-3) / 1e9
+        kd["frac"] = kd["achieved"] / kd["peak"]
+    dom = max(kern, key=lambda k: kern[k]["ms"])
+    kd = kern[dom]
+    roof = {"bound": kd["bound"], "achieved": kd["achieved"], "peak": kd["peak"], "unit": "GB/s", "frac": kd["frac"],
+            "traffic": None, "kernel": dom, "kernel_ms": kd["ms"], "share_of_step": kd["ms"] / (kq_avg + ki_avg),
+            "peak_source": kd["peak_source"], "host_link_1GiB_gbs": host_link,
+            "frac_of_link_bw": kern["km_kernel"]["achieved"] / host_link, "kernels": kern,
+            "algorithmic_bytes_per_step": {"hbm": ab["kq_hbm"] + ab["km_hbm"], "host": ab["km_host"]}}
+    t_roof_step = max((ab["kq_hbm"] + ab["km_hbm"]) / (hbm_peak * 1e9), ab["km_host"] / (host_rand * 1e9))
+    roof["step_roofline_us"] = t_roof_step * 1e6
+    roof["step_frac"] = t_roof_step / (ms / K * 1e-3)
+
+    # latency mode: host clock around query + stream sync (includes launch overhead)
+    log("latency")
+    lat = []
+    for k in range(min(200, K)):
+        t0 = time.perf_counter()
+        cache.query(views(ids_dev[W + k]), outs[k % 4])
+        stream.synchronize()
+        lat.append((time.perf_counter() - t0) * 1e6)
+    lat.sort()
+
+    # end to end through the host-buffer entry point: H2D ids + query + D2H out per step
+    log("e2e")
+    e2e = None
+    if not args.no_e2e:
+        KE = min(K, 100)
+        hids = [torch.from_numpy(gen_batch(P + W + K + KP + i)).pin_memory() for i in range(KE)]
+        hout = torch.empty(N * d, dtype=torch.float32).pin_memory()
+        hv = [[h.numpy()[i * w.batch_size:(i + 1) * w.batch_size] for i in range(w.n)] for h in hids]
+        torch.cuda.synchronize()
+        if dist:
+            dist.barrier()
+        f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        f0.record(stream)
+        for i in range(KE):
+            cache.query_host(hv[i], hout, lengths=lens)
+        f1.record(stream)
+        torch.cuda.synchronize()
+        ems = f0.elapsed_time(f1)
+        if dist:
+            t = torch.tensor([ems], device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ems = float(t.item())
+        e2e = {"value": KE * N * world / (ems * 1e-3) / 1e6, "unit": "Mkeys/s", "h2d_bytes_per_step": N * 8,
+               "d2h_bytes_per_step": N * d * 4, "steps": KE,
+               "note": "fleche_query_host: pinned host IDs -> HBM, query, full output -> pinned host"}
+
+    log("cpu baseline")
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cpu = cpu_baseline(w, tabs, args.cpu_seconds)
+
+    if rank == 0:
+        print(json.dumps({
+            "metric": "embedding lookups/s", "value": value, "unit": "Mkeys/s", "n_gpus": world, "steps": K,
+            "warmup": W, "ms_per_step": ms_max / K, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "dtype": "f32", "data": "synthetic",
+            "config": {"workload": f"{w.name}: {w.n} tables, dim {d}, batch {w.batch_size} per GPU, cache "
+                                   f"{w.cache_frac:.0%} of table bytes, Zipf a={w.skews[0]}",
+                       "tables": w.n, "dim": d, "batch": w.batch_size, "lookups_per_step": N,
+                       "cache_bytes": w.cache_bytes, "host_table_bytes": w.table_bytes,
+                       "parallelism": f"replicated x{world}" if world > 1 else "single GPU",
+                       "prefill_batches": P,
+                       "l2": "inputs larger than L2: fresh ID batch per step, 4 rotating output buffers "
+                             f"({4 * N * d * 4 / 1e6:.0f} MB), {w.cache_bytes / 1e6:.0f} MB slab"},
+            "hit_ratio": hit, "hit_ratio_unique": uhit,
+            "unique_misses_per_step": dst["unique_misses"] / K,
+            "p50_batch_latency_us": lat[len(lat) // 2], "p99_batch_latency_us": lat[int(len(lat) * 0.99) - 1],
+            "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
+            "gpu_launches": int(dst["kernels_launched"]), "clocks": clk,
+            "host_tier_gen_s": t_gen,
+        }), flush=True)
+    if dist:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,171 @@
+/*
+ * include/fleche.h — C ABI of libfleche.so, the B200 (sm_100a) flat embedding cache.
+ *
+ * What it computes (paper: /root/reference/PAPER.md, cited P:L<a>-<b>):
+ *   A DLRM has embedding tables E_0..E_{n-1}; E_t has capacity (corpus size) c_t and
+ *   value dimension d_t.  A query for table t carries an ID list
+ *   ID_List_t and fills the output matrix O_t of shape len(ID_List_t) x d_t with the
+ *   rows E_t[id].  Fleche answers the queries of ALL tables through one
+ *   flat GPU-resident cache shared by every table (flat cache, P:L503-507,
+ *   P:L513-528) with one fused, self-identified launch and
+ *   "still supports the original interface of multi-cache queries":
+ *   that interface is fleche_query below.  Rows that miss in HBM are read straight
+ *   from the CPU-DRAM layer by the GPU (unified index); missed rows are
+ *   inserted with approximate-LRU replacement.
+ *
+ * The result (`out`) is the plain definition: out row = E_t[id], bit for bit; the
+ * cache only changes how fast it is produced.
+ *
+ * Threading / ordering: a ctx is not thread-safe.  Calls on one ctx execute on the
+ * device in call order, even when they are issued on different streams (the
+ * library chains them with an internal event).  Every call except fleche_stats,
+ * fleche_debug_snapshot and fleche_destroy is asynchronous with respect to the host.
+ *
+ * Errors: status codes only; nothing is thrown across the ABI.  Host-side argument
+ * validation returns FLECHE_EINVAL with nothing enqueued.  A CUDA error poisons the
+ * ctx: that call returns FLECHE_ECUDA and every later call FLECHE_ESTATE.
+ */
+#ifndef FLECHE_H_
+#define FLECHE_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct fleche_ctx fleche_ctx; /* opaque; one per (process, GPU) */
+typedef void* fleche_stream;           /* a cudaStream_t; NULL = legacy default stream */
+
+typedef enum {
+  FLECHE_OK = 0,
+  FLECHE_EINVAL = -1, /* bad argument; nothing was enqueued                                    */
+  FLECHE_ENOMEM = -2, /* device or pinned-host allocation failed                               */
+  FLECHE_ECUDA = -3,  /* a CUDA call failed; the ctx is now poisoned                          */
+  FLECHE_ENCCL = -4,  /* reserved for the key-sharded multi-GPU mode                          */
+  FLECHE_ERANGE = -5, /* fleche_stats: some query since the last reset carried an ID outside
+                         [0, c_t); the stats are still valid (see fleche_query)               */
+  FLECHE_ESTATE = -6  /* ctx poisoned by an earlier CUDA error                                */
+} fleche_status;
+
+#define FLECHE_MAX_TABLES 1024
+
+typedef struct {
+  int32_t num_tables;            /* n, 1 <= n <= FLECHE_MAX_TABLES                               */
+  const int64_t* cardinalities;  /* [n] host array: c_t >= 1 rows of table t                    */
+  const int32_t* dims;           /* [n] host array: d_t in {8, 16, 32, 64, 128, 256} (rows are moved
+                                    as 16-byte vectors by warp-shaped kernels specialised per
+                                    width).  Round 1: all d_t must be equal (one slab class);
+                                    mixed dims return FLECHE_EINVAL.                              */
+  uint64_t cache_bytes;          /* HBM budget for cached embedding ROWS (the paper expresses the
+                                    cache size as a fraction of all table bytes);
+                                    capacity = floor(cache_bytes / (4 d)) rows.  The index
+                                    (8 B per row) and scratch are reported in index_bytes.       */
+  const float* const* host_tables;/* [n] host array of host pointers: E_t row-major c_t x d_t fp32,
+                                    16-byte aligned, caller-owned, must outlive the ctx.  The ctx
+                                    page-locks and maps them (cudaHostRegister Mapped|Portable)
+                                    unless they are already registered/pinned; the GPU then reads
+                                    missed rows with zero-copy loads over the host link.          */
+  int64_t max_lookups;           /* upper bound on sum_t lengths[t] per fleche_query call; sizes
+                                    every per-batch scratch buffer once at create (no allocation
+                                    on the query path)                                */
+  int32_t device;                /* CUDA device ordinal                                           */
+  double admit_prob;             /* admission probability p; <= 0 or >= 1 => admit
+                                    every miss.  Coin: splitmix64(admit_seed ^ fk ^ (batch << 32))
+                                    < p * 2^64, batch = 0-based query count (R8)        */
+  uint64_t admit_seed;
+  uint32_t hash_seed;            /* set index = (fmix32(fk ^ hash_seed) * S) >> 32 (R12)  */
+  uint32_t flags;                /* reserved, must be 0                                            */
+} fleche_config;
+
+typedef struct {
+  uint64_t batches;            /* query calls                                                       */
+  uint64_t lookups;            /* IDs looked up (valid + invalid)                                   */
+  uint64_t hits;               /* lookups whose key was cached before the batch started             */
+  uint64_t misses;             /* valid lookups that were not cached (duplicates included)          */
+  uint64_t invalid;            /* IDs outside [0, c_t): zero row, never cached                      */
+  uint64_t unique_keys;        /* unique valid keys per batch, summed                               */
+  uint64_t unique_hits;
+  uint64_t unique_misses;      /* = rows read from the host tier                                    */
+  uint64_t inserted;           /* rows admitted into the cache                                      */
+  uint64_t evicted;            /* cached rows replaced                                              */
+  uint64_t bypassed;           /* unique misses not inserted (admission coin, or every way of the
+                                  set was read/written in the same batch)                          */
+  uint64_t occupancy_bytes;    /* rows currently cached x row bytes (<= capacity_bytes)             */
+  uint64_t capacity_bytes;     /* capacity rows x row bytes                                         */
+  uint64_t index_bytes;        /* HBM used by index + scratch (not counted in cache_bytes)          */
+  uint64_t host_bytes_fetched; /* bytes read from the host tier over the host link                  */
+  uint64_t kernels_launched;   /* kernels this ctx launched                                         */
+} fleche_stats_t;
+
+/* Create a cache for the tables in *cfg on cfg->device.  Allocates every device
+ * buffer once.  Returns FLECHE_EINVAL for an invalid configuration,
+ * including tables whose size-aware flat keys do not fit in 32 bits. */
+fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out);
+
+/* One batch of one-hot lookups for every table.
+ *   ids[t]     : DEVICE pointer to lengths[t] int64 IDs of table t (may be NULL if
+ *                lengths[t] == 0); ids itself is a HOST array of n pointers.
+ *   lengths[t] : HOST array, len(ID_List_t) >= 0; sum <= max_lookups.
+ *   out        : DEVICE fp32 buffer, table-major concatenation of O_t: table t starts
+ *                at float offset sum_{u<t} lengths[u] * d_u; row j of O_t = E_t[ids[t][j]].
+ *                16-byte aligned.
+ *   stream     : cudaStream_t the work is enqueued on.
+ * IDs outside [0, c_t) (reading R15) yield a zero row, count as `invalid`, are never
+ * cached, and make the next fleche_stats return FLECHE_ERANGE.  Caller owns ids and
+ * out; they must stay valid until the stream has passed this call.  Enqueues 2
+ * kernels and never blocks the host. */
+fleche_status fleche_query(fleche_ctx* ctx, const int64_t* const* ids, const int64_t* lengths, float* out,
+                           fleche_stream stream);
+
+/* Same lookups with HOST buffers: ids[t] are host pointers (ideally pinned), out is a
+ * host buffer.  Enqueues host->device copies of the IDs, the query, and the
+ * device->host copy of out on `stream` (ctx-owned device staging, allocated at the
+ * first call).  Asynchronous: out is complete once the stream is synchronised. */
+fleche_status fleche_query_host(fleche_ctx* ctx, const int64_t* const* ids, const int64_t* lengths, float* out,
+                                fleche_stream stream);
+
+/* Counters accumulated since create / the last reset.  Blocks until the ctx's
+ * work has finished.  Returns FLECHE_ERANGE (with *out filled) if an invalid ID
+ * was seen since the last reset. */
+fleche_status fleche_stats(fleche_ctx* ctx, fleche_stats_t* out);
+fleche_status fleche_reset_stats(fleche_ctx* ctx);
+
+/* Release every device buffer and host registration the ctx made. */
+fleche_status fleche_destroy(fleche_ctx* ctx);
+
+const char* fleche_strerror(fleche_status status);
+
+/* Introspection for tests.
+ * fleche_get_encoding: base[t] (first flat key of table t), fbits[t] (feature bits),
+ *   *key_bits = minimal key width B_min of the size-aware code.
+ * fleche_get_geometry: number of index sets S, capacity rows, row floats d.
+ * fleche_debug_snapshot: blocking copy of the index (keys[S*32], ts[S*32]; uint32,
+ *   EMPTY key = 0xFFFFFFFF) and of the slab (S*32 rows x d floats; row of way w of set
+ *   s at (s*32 + w) * d) into host buffers of at least the given element counts. */
+fleche_status fleche_get_encoding(fleche_ctx* ctx, uint64_t* base, int32_t* fbits, int32_t* key_bits);
+fleche_status fleche_get_geometry(fleche_ctx* ctx, int64_t* sets, int64_t* rows, int32_t* row_floats);
+fleche_status fleche_debug_snapshot(fleche_ctx* ctx, uint32_t* keys, uint32_t* ts, size_t ways_cap, float* slab,
+                                    size_t slab_floats_cap);
+
+/* Diagnostics for measurement (bench.py).
+ * fleche_set_profiling: when enabled, every later query records CUDA events on its
+ *   stream around each of its kernels (adds ~3 event records per call).
+ * fleche_kernel_times: blocking; summed device time (ms) of the query kernel (KQ) and
+ *   the insert kernel (KI) over the profiled queries since the last call, and their
+ *   count; resets the accumulation.
+ * fleche_probe_host_read: measures random-row zero-copy read bandwidth of the host
+ *   link: a kernel with the KQ miss-fetch access pattern reads `rows` rows of
+ *   `row_bytes` (multiple of 16, <= 4096) at seeded random row indices of the mapped
+ *   host buffer [host, host + bytes) (already registered, e.g. a ctx's table), timed
+ *   with CUDA events on `stream`; *gbps = rows * row_bytes / time.  Blocking. */
+fleche_status fleche_set_profiling(fleche_ctx* ctx, int enable);
+fleche_status fleche_kernel_times(fleche_ctx* ctx, double* kq_ms, double* ki_ms, uint64_t* queries);
+fleche_status fleche_probe_host_read(const void* host, uint64_t bytes, int32_t row_bytes, int64_t rows, uint64_t seed,
+                                     fleche_stream stream, double* gbps);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* FLECHE_H_ */

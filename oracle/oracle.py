@@ -21,7 +21,7 @@ MODE_GLOBAL = 0
 MODE_SETASSOC = 1
 
 STAT_FIELDS = ["batches", "lookups", "hits", "misses", "invalid", "unique_keys", "unique_hits", "unique_misses",
-               "inserted", "evicted", "bypassed", "occupancy_bytes", "capacity_bytes"]
+               "inserted", "evicted", "bypassed", "occupancy_bytes", "capacity_bytes", "bypass_full"]
 
 
 class _Stats(ctypes.Structure):

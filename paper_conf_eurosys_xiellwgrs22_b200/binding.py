@@ -1,0 +1,204 @@
+"""Thin ctypes binding of libfleche.so (include/fleche.h).  Argument marshalling only:
+every step of the lookup path runs in the library's CUDA kernels.  There is no CPU
+fallback: if the shared library is missing this module raises at import time.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libfleche.so")
+
+if not os.path.exists(LIB_PATH):
+    raise ImportError(f"libfleche.so not built at {LIB_PATH}: run `make` (or __graft_entry__.build()) first; "
+                      "the flat cache has no CPU fallback")
+
+_lib = ctypes.CDLL(LIB_PATH)
+
+OK, EINVAL, ENOMEM, ECUDA, ENCCL, ERANGE, ESTATE = 0, -1, -2, -3, -4, -5, -6
+MAX_TABLES = 1024
+
+_vp, _i64, _i32, _u64, _u32 = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32, ctypes.c_uint64, ctypes.c_uint32
+
+
+class fleche_config(ctypes.Structure):
+    _fields_ = [("num_tables", _i32), ("cardinalities", _vp), ("dims", _vp), ("cache_bytes", _u64),
+                ("host_tables", _vp), ("max_lookups", _i64), ("device", _i32), ("admit_prob", ctypes.c_double),
+                ("admit_seed", _u64), ("hash_seed", _u32), ("flags", _u32)]
+
+
+STAT_FIELDS = ["batches", "lookups", "hits", "misses", "invalid", "unique_keys", "unique_hits", "unique_misses",
+               "inserted", "evicted", "bypassed", "occupancy_bytes", "capacity_bytes", "index_bytes",
+               "host_bytes_fetched", "kernels_launched"]
+
+
+class fleche_stats_t(ctypes.Structure):
+    _fields_ = [(f, _u64) for f in STAT_FIELDS]
+
+
+def _sig(name, res, args):
+    f = getattr(_lib, name)
+    f.restype = res
+    f.argtypes = args
+    return f
+
+
+fleche_create = _sig("fleche_create", ctypes.c_int, [ctypes.POINTER(fleche_config), ctypes.POINTER(_vp)])
+fleche_query = _sig("fleche_query", ctypes.c_int, [_vp, _vp, _vp, _vp, _vp])
+fleche_query_host = _sig("fleche_query_host", ctypes.c_int, [_vp, _vp, _vp, _vp, _vp])
+fleche_stats = _sig("fleche_stats", ctypes.c_int, [_vp, ctypes.POINTER(fleche_stats_t)])
+fleche_reset_stats = _sig("fleche_reset_stats", ctypes.c_int, [_vp])
+fleche_destroy = _sig("fleche_destroy", ctypes.c_int, [_vp])
+fleche_strerror = _sig("fleche_strerror", ctypes.c_char_p, [ctypes.c_int])
+fleche_get_encoding = _sig("fleche_get_encoding", ctypes.c_int, [_vp, _vp, _vp, ctypes.POINTER(_i32)])
+fleche_get_geometry = _sig("fleche_get_geometry", ctypes.c_int,
+                           [_vp, ctypes.POINTER(_i64), ctypes.POINTER(_i64), ctypes.POINTER(_i32)])
+fleche_debug_snapshot = _sig("fleche_debug_snapshot", ctypes.c_int, [_vp, _vp, _vp, ctypes.c_size_t, _vp,
+                                                                     ctypes.c_size_t])
+
+fleche_set_profiling = _sig("fleche_set_profiling", ctypes.c_int, [_vp, ctypes.c_int])
+fleche_kernel_times = _sig("fleche_kernel_times", ctypes.c_int, [_vp, ctypes.POINTER(ctypes.c_double),
+                                                                 ctypes.POINTER(ctypes.c_double),
+                                                                 ctypes.POINTER(_u64)])
+fleche_probe_host_read = _sig("fleche_probe_host_read", ctypes.c_int, [_vp, _u64, _i32, _i64, _u64, _vp,
+                                                                       ctypes.POINTER(ctypes.c_double)])
+
+EXPORTED = ["fleche_create", "fleche_query", "fleche_query_host", "fleche_stats", "fleche_reset_stats",
+            "fleche_destroy", "fleche_strerror", "fleche_get_encoding", "fleche_get_geometry",
+            "fleche_debug_snapshot", "fleche_set_profiling", "fleche_kernel_times", "fleche_probe_host_read"]
+
+
+def probe_host_read(host_ptr: int, nbytes: int, row_bytes: int, rows: int, seed: int = 1, stream=None) -> float:
+    """Random-row zero-copy read bandwidth (GB/s) of an already-registered host buffer."""
+    g = ctypes.c_double()
+    _check(fleche_probe_host_read(host_ptr, nbytes, row_bytes, rows, seed, _stream_handle(stream), ctypes.byref(g)),
+           "fleche_probe_host_read")
+    return float(g.value)
+
+
+class FlecheError(RuntimeError):
+    def __init__(self, status: int, what: str):
+        super().__init__(f"{what}: {fleche_strerror(status).decode()} ({status})")
+        self.status = status
+
+
+def _check(status: int, what: str, allow=(OK,)):
+    if status not in allow:
+        raise FlecheError(status, what)
+    return status
+
+
+def _ptr(x) -> int:
+    """Raw address of a torch tensor / numpy array / int."""
+    if x is None:
+        return 0
+    if isinstance(x, int):
+        return x
+    if hasattr(x, "data_ptr"):
+        return int(x.data_ptr())
+    if isinstance(x, np.ndarray):
+        return int(x.ctypes.data)
+    raise TypeError(type(x))
+
+
+def _stream_handle(stream) -> int:
+    if stream is None:
+        import torch
+        return int(torch.cuda.current_stream().cuda_stream)
+    if isinstance(stream, int):
+        return stream
+    return int(stream.cuda_stream)
+
+
+class FlatCache:
+    """One flat GPU cache over the given host tables (fleche_create / fleche_query / fleche_stats)."""
+
+    def __init__(self, cards, dims, host_tables, cache_bytes: int, max_lookups: int, device: int = 0,
+                 admit_prob: float = 1.0, admit_seed: int = 0, hash_seed: int = 0):
+        self.n = len(cards)
+        self.cards = np.ascontiguousarray(cards, dtype=np.int64)
+        self.dims = np.ascontiguousarray(dims, dtype=np.int32)
+        self._tables = list(host_tables)  # keep the host tier alive for the ctx's lifetime
+        self._tp = (_vp * self.n)(*[_ptr(t) for t in self._tables])
+        cfg = fleche_config(self.n, self.cards.ctypes.data, self.dims.ctypes.data, int(cache_bytes),
+                            ctypes.cast(self._tp, _vp), int(max_lookups), int(device), float(admit_prob),
+                            int(admit_seed), int(hash_seed), 0)
+        h = _vp()
+        _check(fleche_create(ctypes.byref(cfg), ctypes.byref(h)), "fleche_create")
+        self.h = h.value
+        self.device = device
+        self.max_lookups = int(max_lookups)
+
+    def close(self):
+        if getattr(self, "h", None):
+            fleche_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def out_floats(self, lengths) -> int:
+        return int(sum(int(l) * int(d) for l, d in zip(lengths, self.dims)))
+
+    def query(self, ids, out, stream=None, lengths=None):
+        """ids: list of n device int64 tensors (or pointers with `lengths`); out: device fp32 buffer."""
+        if lengths is None:
+            lengths = [int(x.numel()) for x in ids]
+        lp = (_i64 * self.n)(*lengths)
+        ip = (_vp * self.n)(*[_ptr(x) for x in ids])
+        _check(fleche_query(self.h, ip, lp, _ptr(out), _stream_handle(stream)), "fleche_query")
+
+    def query_host(self, ids, out, stream=None, lengths=None):
+        """ids: list of n host int64 arrays (ideally pinned); out: host fp32 buffer."""
+        if lengths is None:
+            lengths = [int(x.size if isinstance(x, np.ndarray) else x.numel()) for x in ids]
+        lp = (_i64 * self.n)(*lengths)
+        ip = (_vp * self.n)(*[_ptr(x) for x in ids])
+        _check(fleche_query_host(self.h, ip, lp, _ptr(out), _stream_handle(stream)), "fleche_query_host")
+
+    def stats(self, allow_invalid: bool = True) -> dict:
+        s = fleche_stats_t()
+        st = fleche_stats(self.h, ctypes.byref(s))
+        _check(st, "fleche_stats", (OK, ERANGE) if allow_invalid else (OK,))
+        d = {f: int(getattr(s, f)) for f in STAT_FIELDS}
+        d["invalid_seen"] = st == ERANGE
+        return d
+
+    def reset_stats(self):
+        _check(fleche_reset_stats(self.h), "fleche_reset_stats")
+
+    def set_profiling(self, on: bool):
+        _check(fleche_set_profiling(self.h, 1 if on else 0), "fleche_set_profiling")
+
+    def kernel_times(self):
+        """(KQ ms total, KI ms total, profiled queries) since the last call."""
+        a, b, q = ctypes.c_double(), ctypes.c_double(), _u64()
+        _check(fleche_kernel_times(self.h, ctypes.byref(a), ctypes.byref(b), ctypes.byref(q)), "fleche_kernel_times")
+        return float(a.value), float(b.value), int(q.value)
+
+    def encoding(self):
+        base = np.zeros(self.n, dtype=np.uint64)
+        fb = np.zeros(self.n, dtype=np.int32)
+        kb = _i32()
+        _check(fleche_get_encoding(self.h, base.ctypes.data, fb.ctypes.data, ctypes.byref(kb)), "fleche_get_encoding")
+        return int(kb.value), base, fb
+
+    def geometry(self):
+        s, r, d = _i64(), _i64(), _i32()
+        _check(fleche_get_geometry(self.h, ctypes.byref(s), ctypes.byref(r), ctypes.byref(d)), "fleche_get_geometry")
+        return int(s.value), int(r.value), int(d.value)
+
+    def snapshot(self):
+        sets, rows, d = self.geometry()
+        keys = np.empty(sets * 32, np.uint32)
+        ts = np.empty(sets * 32, np.uint32)
+        slab = np.empty(sets * 32 * d, np.float32)
+        _check(fleche_debug_snapshot(self.h, keys.ctypes.data, ts.ctypes.data, keys.size, slab.ctypes.data, slab.size),
+               "fleche_debug_snapshot")
+        return keys, ts, slab.reshape(sets * 32, d)

@@ -1,0 +1,548 @@
+// fleche.cu — host side of libfleche.so: the C ABI declared in include/fleche.h.
+//
+// Owns every device allocation (made once in fleche_create), the
+// host-tier registration (pinned + mapped tables read by zero-copy loads,
+// P:L855-860), per-call argument packing into kernel parameters (the Args Array and
+// scan of P:L713-737 travel as __grid_constant__ parameters: no metadata copy on the
+// query path), cross-stream ordering, and the stats read-back.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <vector>
+
+#include "fleche.h"
+#include "kernels.cuh"
+
+using namespace fl;
+
+struct fleche_ctx {
+  int device = 0;
+  int n = 0;
+  int dim = 0;
+  int sm_count = 148;
+  bool poisoned = false;
+  int64_t max_lookups = 0;
+  std::vector<int64_t> card;
+  std::vector<int32_t> dims;
+  std::vector<uint64_t> base;
+  std::vector<int32_t> fbits;
+  int key_bits = 0;
+  std::vector<std::pair<void*, size_t>> registered;  // host ranges we registered
+  Dev dv{};
+  TableInfo* d_tables = nullptr;
+  int ki_blocks = 0;
+  // host-side counters
+  uint64_t batches = 0, lookups = 0, kernels = 0;
+  // ordering across streams
+  cudaStream_t last_stream = nullptr;
+  bool have_last = false;
+  cudaEvent_t chain_ev = nullptr;
+  // fleche_query_host staging (lazy)
+  int64_t* d_ids_stage = nullptr;
+  float* d_out_stage = nullptr;
+  uint64_t index_bytes = 0;
+  // profiling (fleche_set_profiling)
+  bool profiling = false;
+  std::vector<cudaEvent_t> ev_pool;  // 3 per profiled query
+  size_t ev_used = 0;
+};
+
+namespace {
+
+fleche_status poison(fleche_ctx* c, cudaError_t e, const char* what) {
+  if (c) c->poisoned = true;
+  fprintf(stderr, "[fleche] CUDA error in %s: %s\n", what, cudaGetErrorString(e));
+  return FLECHE_ECUDA;
+}
+
+#define FL_CUDA(ctx, call)                                   \
+  do {                                                       \
+    cudaError_t e_ = (call);                                 \
+    if (e_ != cudaSuccess) return poison((ctx), e_, #call);  \
+  } while (0)
+
+int ceil_log2_u64(int64_t c) {
+  int f = 0;
+  while (f < 63 && (int64_t(1) << f) < c) ++f;
+  return f;
+}
+
+// Size-aware coding (R3): larger tables get shorter table IDs.
+// feature bits f_t = max(1, ceil(log2 c_t)); table IDs assigned as a canonical prefix
+// code in order of increasing length; fk = base_t + id.  Returns B_min or -1 if the
+// code plus the reserved all-ones key does not fit in 32 bits.
+int size_aware_code(const std::vector<int64_t>& card, std::vector<uint64_t>& base, std::vector<int32_t>& fb) {
+  const int n = (int)card.size();
+  fb.resize(n);
+  base.resize(n);
+  unsigned __int128 span = 1;  // the EMPTY key
+  for (int t = 0; t < n; ++t) {
+    fb[t] = std::max(1, ceil_log2_u64(card[t]));
+    span += (unsigned __int128)1 << fb[t];
+  }
+  int bmin = 0;
+  while (((unsigned __int128)1 << bmin) < span) ++bmin;
+  if (bmin > 32) return -1;
+  std::vector<int> idx(n);
+  for (int t = 0; t < n; ++t) idx[t] = t;
+  std::sort(idx.begin(), idx.end(), [&](int a, int b) { return fb[a] != fb[b] ? fb[a] > fb[b] : a < b; });
+  uint64_t at = 0;
+  for (int t : idx) {
+    base[t] = at;
+    at += uint64_t(1) << fb[t];
+  }
+  return bmin;
+}
+
+uint32_t next_pow2(uint64_t x) {
+  uint64_t p = 1;
+  while (p < x) p <<= 1;
+  return (uint32_t)p;
+}
+
+// Page-lock and map the caller's tables.  Ranges are merged on page boundaries
+// (tables usually share one allocation, and a page may only be registered once).
+fleche_status register_host(fleche_ctx* c, const float* const* host, std::vector<const float*>& dev_ptrs) {
+  const uintptr_t pg = 4096;
+  std::vector<std::pair<uintptr_t, uintptr_t>> r;
+  for (int t = 0; t < c->n; ++t) {
+    uintptr_t a = (uintptr_t)host[t], b = a + (size_t)c->card[t] * (size_t)c->dims[t] * 4u;
+    r.push_back({a, b});
+  }
+  std::sort(r.begin(), r.end());
+  std::vector<std::pair<uintptr_t, uintptr_t>> m;
+  for (auto& x : r) {  // ranges that touch a common page are registered together
+    if (!m.empty() && (x.first & ~(pg - 1)) <= ((m.back().second - 1) & ~(pg - 1)))
+      m.back().second = std::max(m.back().second, x.second);
+    else
+      m.push_back(x);
+  }
+  for (auto& x : m) {
+    void* p = (void*)x.first;
+    cudaPointerAttributes at{};
+    if (cudaPointerGetAttributes(&at, p) == cudaSuccess && at.type == cudaMemoryTypeHost) continue;  // pinned already
+    cudaGetLastError();
+    cudaError_t e = cudaHostRegister(p, x.second - x.first, cudaHostRegisterMapped | cudaHostRegisterPortable);
+    if (e == cudaErrorHostMemoryAlreadyRegistered) {
+      cudaGetLastError();  // caller pinned it already (cudaHostAlloc / earlier ctx)
+      continue;
+    }
+    if (e != cudaSuccess) return poison(c, e, "cudaHostRegister");
+    c->registered.push_back({p, x.second - x.first});
+  }
+  dev_ptrs.resize(c->n);
+  for (int t = 0; t < c->n; ++t) {
+    void* dp = nullptr;
+    FL_CUDA(c, cudaHostGetDevicePointer(&dp, (void*)host[t], 0));
+    dev_ptrs[t] = (const float*)dp;
+  }
+  return FLECHE_OK;
+}
+
+void free_all(fleche_ctx* c) {
+  void* ptrs[] = {c->dv.keys, c->dv.ts, c->dv.slab, c->dv.scratch, c->dv.dup_head, c->dv.miss, c->dv.dup,
+                  c->dv.ctl, c->dv.stats, c->d_tables, c->d_ids_stage, c->d_out_stage};
+  for (void* p : ptrs)
+    if (p) cudaFree(p);
+  for (auto& r : c->registered) cudaHostUnregister(r.first);
+  c->registered.clear();
+  if (c->chain_ev) cudaEventDestroy(c->chain_ev);
+  for (cudaEvent_t e : c->ev_pool) cudaEventDestroy(e);
+  c->ev_pool.clear();
+}
+
+fleche_status ensure_device(fleche_ctx* c) {
+  int cur = -1;
+  if (cudaGetDevice(&cur) != cudaSuccess || cur != c->device) FL_CUDA(c, cudaSetDevice(c->device));
+  return FLECHE_OK;
+}
+
+// Calls on one ctx run in call order even across streams.
+fleche_status order_on(fleche_ctx* c, cudaStream_t s) {
+  if (c->have_last && s != c->last_stream) {
+    FL_CUDA(c, cudaEventRecord(c->chain_ev, c->last_stream));
+    FL_CUDA(c, cudaStreamWaitEvent(s, c->chain_ev, 0));
+  }
+  c->last_stream = s;
+  c->have_last = true;
+  return FLECHE_OK;
+}
+
+template <int MAXT>
+fleche_status launch_query(fleche_ctx* c, const int64_t* const* ids, const int64_t* lengths, float* out,
+                           cudaStream_t s, int64_t total) {
+  QArgs<MAXT> qa;
+  memset(&qa, 0, sizeof(qa));
+  qa.n = c->n;
+  qa.out = out;
+  int64_t acc = 0, oacc = 0;
+  for (int t = 0; t < c->n; ++t) {
+    qa.ids[t] = ids[t];
+    qa.scan[t] = acc;
+    qa.out_off[t] = oacc;
+    acc += lengths[t];
+    oacc += lengths[t] * (int64_t)c->dims[t];
+  }
+  qa.scan[c->n] = acc;
+  cudaEvent_t ev[3] = {nullptr, nullptr, nullptr};
+  if (c->profiling) {
+    while (c->ev_pool.size() < c->ev_used + 3) {
+      cudaEvent_t e;
+      FL_CUDA(c, cudaEventCreate(&e));
+      c->ev_pool.push_back(e);
+    }
+    for (int i = 0; i < 3; ++i) ev[i] = c->ev_pool[c->ev_used + i];
+    c->ev_used += 3;
+    FL_CUDA(c, cudaEventRecord(ev[0], s));
+  }
+  if (total > 0) {
+    const int64_t blocks = (total + 127) / 128;
+    kq_kernel<MAXT><<<(unsigned)blocks, 128, 0, s>>>(qa, c->dv);
+    c->kernels++;
+  }
+  if (ev[1]) FL_CUDA(c, cudaEventRecord(ev[1], s));
+  km_kernel<<<c->ki_blocks, 128, 0, s>>>(c->dv, out);
+  c->kernels++;
+  if (ev[2]) FL_CUDA(c, cudaEventRecord(ev[2], s));
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return poison(c, e, "kernel launch");
+  return FLECHE_OK;
+}
+
+fleche_status query_impl(fleche_ctx* c, const int64_t* const* ids, const int64_t* lengths, float* out,
+                         cudaStream_t s) {
+  int64_t total = 0;
+  for (int t = 0; t < c->n; ++t) {
+    if (lengths[t] < 0) return FLECHE_EINVAL;
+    if (lengths[t] > 0 && !ids[t]) return FLECHE_EINVAL;
+    total += lengths[t];
+  }
+  if (total > c->max_lookups) return FLECHE_EINVAL;
+  if (total > 0 && (!out || ((uintptr_t)out & 15u))) return FLECHE_EINVAL;
+  fleche_status st = ensure_device(c);
+  if (st != FLECHE_OK) return st;
+  st = order_on(c, s);
+  if (st != FLECHE_OK) return st;
+  if (c->n <= 32) st = launch_query<32>(c, ids, lengths, out, s, total);
+  else if (c->n <= 128) st = launch_query<128>(c, ids, lengths, out, s, total);
+  else st = launch_query<FLECHE_MAX_TABLES>(c, ids, lengths, out, s, total);
+  if (st == FLECHE_OK) {
+    c->batches++;
+    c->lookups += (uint64_t)total;
+  }
+  return st;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char* fleche_strerror(fleche_status s) {
+  switch (s) {
+    case FLECHE_OK: return "ok";
+    case FLECHE_EINVAL: return "invalid argument";
+    case FLECHE_ENOMEM: return "out of memory";
+    case FLECHE_ECUDA: return "CUDA error";
+    case FLECHE_ENCCL: return "NCCL error";
+    case FLECHE_ERANGE: return "an ID outside [0, c_t) was looked up";
+    case FLECHE_ESTATE: return "context poisoned by an earlier CUDA error";
+  }
+  return "unknown status";
+}
+
+fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
+  if (!cfg || !out) return FLECHE_EINVAL;
+  *out = nullptr;
+  const int n = cfg->num_tables;
+  if (n < 1 || n > FLECHE_MAX_TABLES || !cfg->cardinalities || !cfg->dims || !cfg->host_tables) return FLECHE_EINVAL;
+  if (cfg->max_lookups < 1 || cfg->max_lookups > (int64_t(1) << 31) || cfg->flags != 0) return FLECHE_EINVAL;
+  for (int t = 0; t < n; ++t) {
+    const int d = cfg->dims[t];
+    if (cfg->cardinalities[t] < 1 || d != cfg->dims[0]) return FLECHE_EINVAL;
+    if (d != 8 && d != 16 && d != 32 && d != 64 && d != 128 && d != 256) return FLECHE_EINVAL;
+    if (!cfg->host_tables[t] || ((uintptr_t)cfg->host_tables[t] & 15u)) return FLECHE_EINVAL;
+  }
+  fleche_ctx* c = new (std::nothrow) fleche_ctx();
+  if (!c) return FLECHE_ENOMEM;
+  c->device = cfg->device;
+  c->n = n;
+  c->dim = cfg->dims[0];
+  c->max_lookups = cfg->max_lookups;
+  c->card.assign(cfg->cardinalities, cfg->cardinalities + n);
+  c->dims.assign(cfg->dims, cfg->dims + n);
+  c->key_bits = size_aware_code(c->card, c->base, c->fbits);
+  const uint64_t rows = cfg->cache_bytes / (4ull * (uint64_t)c->dim);
+  if (c->key_bits < 0 || rows > 0xFFFFFFE0ull) {
+    delete c;
+    return FLECHE_EINVAL;
+  }
+  auto fail = [&](fleche_status s) {
+    free_all(c);
+    delete c;
+    return s;
+  };
+  if (cudaSetDevice(c->device) != cudaSuccess) return fail(FLECHE_EINVAL);
+  cudaDeviceGetAttribute(&c->sm_count, cudaDevAttrMultiProcessorCount, c->device);
+
+  const uint64_t sets = std::max<uint64_t>(1, (rows + 31) / 32);
+  const uint32_t scr_n = next_pow2(std::max<uint64_t>(1024, 2ull * (uint64_t)cfg->max_lookups));
+  Dev& dv = c->dv;
+  dv.sets = (uint32_t)sets;
+  dv.rows = (uint32_t)rows;
+  dv.dim = c->dim;
+  dv.hash_seed = cfg->hash_seed;
+  dv.scr_mask = scr_n - 1;
+  const double p = cfg->admit_prob;
+  dv.admit_all = (p <= 0.0 || p >= 1.0) ? 1 : 0;
+  dv.admit_thr = dv.admit_all ? ~0ull : (uint64_t)ldexp(p, 64);
+  dv.admit_seed = cfg->admit_seed;
+
+  auto alloc = [&](void** p, size_t bytes) { return cudaMalloc(p, bytes) == cudaSuccess; };
+  const size_t ways = (size_t)sets * 32u;
+  bool ok = alloc((void**)&dv.keys, ways * 4) && alloc((void**)&dv.ts, ways * 4) &&
+            alloc((void**)&dv.slab, ways * (size_t)c->dim * 4) &&
+            alloc((void**)&dv.scratch, (size_t)scr_n * 8) && alloc((void**)&dv.dup_head, (size_t)scr_n * 8) &&
+            alloc((void**)&dv.miss, (size_t)cfg->max_lookups * sizeof(MissRec)) &&
+            alloc((void**)&dv.dup, (size_t)cfg->max_lookups * sizeof(DupRec)) &&
+            alloc((void**)&dv.ctl, sizeof(Ctl)) &&
+            alloc((void**)&dv.stats, sizeof(unsigned long long) * kStripes * kNumCtr) &&
+            alloc((void**)&c->d_tables, sizeof(TableInfo) * n);
+  if (!ok) {
+    cudaGetLastError();
+    return fail(FLECHE_ENOMEM);
+  }
+  c->index_bytes = ways * 8 + (size_t)scr_n * 16 + (size_t)cfg->max_lookups * (sizeof(MissRec) + sizeof(DupRec));
+  dv.tables = c->d_tables;
+  if (cudaMemset(dv.keys, 0xFF, ways * 4) != cudaSuccess || cudaMemset(dv.ts, 0, ways * 4) != cudaSuccess ||
+      cudaMemset(dv.scratch, 0, (size_t)scr_n * 8) != cudaSuccess ||
+      cudaMemset(dv.dup_head, 0, (size_t)scr_n * 8) != cudaSuccess ||
+      cudaMemset(dv.stats, 0, sizeof(unsigned long long) * kStripes * kNumCtr) != cudaSuccess)
+    return fail(FLECHE_ECUDA);
+  Ctl ctl{};
+  ctl.epoch = 1;
+  if (cudaMemcpy(dv.ctl, &ctl, sizeof(Ctl), cudaMemcpyHostToDevice) != cudaSuccess) return fail(FLECHE_ECUDA);
+
+  std::vector<const float*> dptr;
+  if (register_host(c, cfg->host_tables, dptr) != FLECHE_OK) return fail(FLECHE_ECUDA);
+  std::vector<TableInfo> ti(n);
+  for (int t = 0; t < n; ++t) ti[t] = TableInfo{dptr[t], c->card[t], (uint32_t)c->base[t], c->dims[t]};
+  if (cudaMemcpy(c->d_tables, ti.data(), sizeof(TableInfo) * n, cudaMemcpyHostToDevice) != cudaSuccess)
+    return fail(FLECHE_ECUDA);
+  if (cudaEventCreateWithFlags(&c->chain_ev, cudaEventDisableTiming) != cudaSuccess) return fail(FLECHE_ECUDA);
+  // KI: enough warps for the expected unique misses, capped at 4 CTAs (32 warps) per SM
+  c->ki_blocks = (int)std::min<int64_t>(4 * c->sm_count, std::max<int64_t>(1, (cfg->max_lookups + 255) / 256));
+  if (cudaDeviceSynchronize() != cudaSuccess) return fail(FLECHE_ECUDA);
+  *out = c;
+  return FLECHE_OK;
+}
+
+fleche_status fleche_query(fleche_ctx* c, const int64_t* const* ids, const int64_t* lengths, float* out,
+                           fleche_stream stream) {
+  if (!c || !ids || !lengths) return FLECHE_EINVAL;
+  if (c->poisoned) return FLECHE_ESTATE;
+  return query_impl(c, ids, lengths, out, (cudaStream_t)stream);
+}
+
+fleche_status fleche_query_host(fleche_ctx* c, const int64_t* const* ids, const int64_t* lengths, float* out,
+                                fleche_stream stream) {
+  if (!c || !ids || !lengths) return FLECHE_EINVAL;
+  if (c->poisoned) return FLECHE_ESTATE;
+  int64_t total = 0;
+  for (int t = 0; t < c->n; ++t) {
+    if (lengths[t] < 0 || (lengths[t] > 0 && !ids[t])) return FLECHE_EINVAL;
+    total += lengths[t];
+  }
+  if (total > c->max_lookups || (total > 0 && !out)) return FLECHE_EINVAL;
+  fleche_status st = ensure_device(c);
+  if (st != FLECHE_OK) return st;
+  cudaStream_t s = (cudaStream_t)stream;
+  if (!c->d_ids_stage) {
+    FL_CUDA(c, cudaMalloc((void**)&c->d_ids_stage, (size_t)c->max_lookups * 8));
+    FL_CUDA(c, cudaMalloc((void**)&c->d_out_stage, (size_t)c->max_lookups * (size_t)c->dim * 4));
+  }
+  st = order_on(c, s);
+  if (st != FLECHE_OK) return st;
+  std::vector<const int64_t*> dids(c->n);
+  // one copy when the per-table host arrays are consecutive in memory, else one per table
+  bool contiguous = true;
+  for (int t = 0; t + 1 < c->n; ++t)
+    if (lengths[t] > 0 && ids[t] + lengths[t] != ids[t + 1]) contiguous = false;
+  int64_t acc = 0;
+  const int64_t* first = nullptr;
+  for (int t = 0; t < c->n; ++t) {
+    if (!first && lengths[t] > 0) first = ids[t];
+    dids[t] = c->d_ids_stage + acc;
+    if (!contiguous && lengths[t] > 0)
+      FL_CUDA(c, cudaMemcpyAsync(c->d_ids_stage + acc, ids[t], (size_t)lengths[t] * 8, cudaMemcpyHostToDevice, s));
+    acc += lengths[t];
+  }
+  if (contiguous && total > 0)
+    FL_CUDA(c, cudaMemcpyAsync(c->d_ids_stage, first, (size_t)total * 8, cudaMemcpyHostToDevice, s));
+  st = query_impl(c, dids.data(), lengths, c->d_out_stage, s);
+  if (st != FLECHE_OK) return st;
+  if (total > 0)
+    FL_CUDA(c, cudaMemcpyAsync(out, c->d_out_stage, (size_t)total * (size_t)c->dim * 4, cudaMemcpyDeviceToHost, s));
+  return FLECHE_OK;
+}
+
+fleche_status fleche_stats(fleche_ctx* c, fleche_stats_t* out) {
+  if (!c || !out) return FLECHE_EINVAL;
+  if (c->poisoned) return FLECHE_ESTATE;
+  fleche_status st = ensure_device(c);
+  if (st != FLECHE_OK) return st;
+  if (c->have_last) FL_CUDA(c, cudaStreamSynchronize(c->last_stream));
+  std::vector<unsigned long long> h(kStripes * kNumCtr);
+  Ctl ctl;
+  FL_CUDA(c, cudaMemcpy(h.data(), c->dv.stats, h.size() * 8, cudaMemcpyDeviceToHost));
+  FL_CUDA(c, cudaMemcpy(&ctl, c->dv.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost));
+  unsigned long long v[kNumCtr] = {0};
+  for (int s = 0; s < kStripes; ++s)
+    for (int k = 0; k < kNumCtr; ++k) v[k] += h[s * kNumCtr + k];
+  memset(out, 0, sizeof(*out));
+  out->batches = c->batches;
+  out->lookups = c->lookups;
+  out->hits = v[C_HITS];
+  out->misses = v[C_MISSES];
+  out->invalid = v[C_INVALID];
+  out->unique_hits = v[C_UHITS];
+  out->unique_misses = v[C_UMISS];
+  out->unique_keys = v[C_UHITS] + v[C_UMISS];
+  out->inserted = v[C_INSERTED];
+  out->evicted = v[C_EVICTED];
+  out->bypassed = v[C_BYPASSED];
+  out->occupancy_bytes = (uint64_t)ctl.occ_rows * 4ull * (uint64_t)c->dim;
+  out->capacity_bytes = (uint64_t)c->dv.rows * 4ull * (uint64_t)c->dim;
+  out->index_bytes = c->index_bytes;
+  out->host_bytes_fetched = v[C_HOSTBYTES];
+  out->kernels_launched = c->kernels;
+  return ctl.err_invalid ? FLECHE_ERANGE : FLECHE_OK;
+}
+
+fleche_status fleche_reset_stats(fleche_ctx* c) {
+  if (!c) return FLECHE_EINVAL;
+  if (c->poisoned) return FLECHE_ESTATE;
+  fleche_status st = ensure_device(c);
+  if (st != FLECHE_OK) return st;
+  if (c->have_last) FL_CUDA(c, cudaStreamSynchronize(c->last_stream));
+  FL_CUDA(c, cudaMemset(c->dv.stats, 0, sizeof(unsigned long long) * kStripes * kNumCtr));
+  FL_CUDA(c, cudaMemset(&c->dv.ctl->err_invalid, 0, sizeof(uint32_t)));
+  FL_CUDA(c, cudaDeviceSynchronize());
+  c->batches = c->lookups = c->kernels = 0;
+  return FLECHE_OK;
+}
+
+fleche_status fleche_destroy(fleche_ctx* c) {
+  if (!c) return FLECHE_EINVAL;
+  int cur = -1;
+  cudaGetDevice(&cur);
+  if (cur != c->device) cudaSetDevice(c->device);
+  if (c->have_last) cudaStreamSynchronize(c->last_stream);
+  free_all(c);
+  delete c;
+  return FLECHE_OK;
+}
+
+fleche_status fleche_get_encoding(fleche_ctx* c, uint64_t* base, int32_t* fbits, int32_t* key_bits) {
+  if (!c) return FLECHE_EINVAL;
+  for (int t = 0; t < c->n; ++t) {
+    if (base) base[t] = c->base[t];
+    if (fbits) fbits[t] = c->fbits[t];
+  }
+  if (key_bits) *key_bits = c->key_bits;
+  return FLECHE_OK;
+}
+
+fleche_status fleche_get_geometry(fleche_ctx* c, int64_t* sets, int64_t* rows, int32_t* row_floats) {
+  if (!c) return FLECHE_EINVAL;
+  if (sets) *sets = c->dv.sets;
+  if (rows) *rows = c->dv.rows;
+  if (row_floats) *row_floats = c->dim;
+  return FLECHE_OK;
+}
+
+fleche_status fleche_debug_snapshot(fleche_ctx* c, uint32_t* keys, uint32_t* ts, size_t ways_cap, float* slab,
+                                    size_t slab_floats_cap) {
+  if (!c) return FLECHE_EINVAL;
+  if (c->poisoned) return FLECHE_ESTATE;
+  const size_t ways = (size_t)c->dv.sets * 32u;
+  if ((keys || ts) && ways_cap < ways) return FLECHE_EINVAL;
+  if (slab && slab_floats_cap < ways * (size_t)c->dim) return FLECHE_EINVAL;
+  fleche_status st = ensure_device(c);
+  if (st != FLECHE_OK) return st;
+  if (c->have_last) FL_CUDA(c, cudaStreamSynchronize(c->last_stream));
+  if (keys) FL_CUDA(c, cudaMemcpy(keys, c->dv.keys, ways * 4, cudaMemcpyDeviceToHost));
+  if (ts) FL_CUDA(c, cudaMemcpy(ts, c->dv.ts, ways * 4, cudaMemcpyDeviceToHost));
+  if (slab) FL_CUDA(c, cudaMemcpy(slab, c->dv.slab, ways * (size_t)c->dim * 4, cudaMemcpyDeviceToHost));
+  return FLECHE_OK;
+}
+
+}  // extern "C"
+
+extern "C" {
+
+fleche_status fleche_set_profiling(fleche_ctx* c, int enable) {
+  if (!c) return FLECHE_EINVAL;
+  c->profiling = enable != 0;
+  return FLECHE_OK;
+}
+
+fleche_status fleche_kernel_times(fleche_ctx* c, double* kq_ms, double* ki_ms, uint64_t* queries) {
+  if (!c) return FLECHE_EINVAL;
+  if (c->poisoned) return FLECHE_ESTATE;
+  double a = 0, b = 0;
+  for (size_t i = 0; i + 3 <= c->ev_used; i += 3) {
+    float x = 0, y = 0;
+    FL_CUDA(c, cudaEventSynchronize(c->ev_pool[i + 2]));
+    FL_CUDA(c, cudaEventElapsedTime(&x, c->ev_pool[i], c->ev_pool[i + 1]));
+    FL_CUDA(c, cudaEventElapsedTime(&y, c->ev_pool[i + 1], c->ev_pool[i + 2]));
+    a += x;
+    b += y;
+  }
+  if (kq_ms) *kq_ms = a;
+  if (ki_ms) *ki_ms = b;
+  if (queries) *queries = c->ev_used / 3;
+  c->ev_used = 0;
+  return FLECHE_OK;
+}
+
+fleche_status fleche_probe_host_read(const void* host, uint64_t bytes, int32_t row_bytes, int64_t rows, uint64_t seed,
+                                     fleche_stream stream, double* gbps) {
+  if (!host || !gbps || rows < 1 || row_bytes < 16 || (row_bytes & 15) || bytes < (uint64_t)row_bytes)
+    return FLECHE_EINVAL;
+  const int D = row_bytes / 4;
+  if (D != 32 && D != 64 && D != 128 && D != 256) return FLECHE_EINVAL;
+  void* dev = nullptr;
+  if (cudaHostGetDevicePointer(&dev, (void*)host, 0) != cudaSuccess) return FLECHE_EINVAL;
+  float* sink = nullptr;
+  if (cudaMalloc((void**)&sink, 4096ull * row_bytes) != cudaSuccess) return FLECHE_ENOMEM;
+  cudaStream_t s = (cudaStream_t)stream;
+  cudaEvent_t e0, e1;
+  cudaEventCreate(&e0);
+  cudaEventCreate(&e1);
+  const uint64_t span = bytes / (uint64_t)row_bytes;
+  const unsigned blocks = (unsigned)((rows + 127) / 128);
+  auto launch = [&](uint64_t sd) {
+    if (D == 32) probe_host_kernel<32><<<blocks, 128, 0, s>>>((const float*)dev, span, rows, sd, sink);
+    else if (D == 64) probe_host_kernel<64><<<blocks, 128, 0, s>>>((const float*)dev, span, rows, sd, sink);
+    else if (D == 128) probe_host_kernel<128><<<blocks, 128, 0, s>>>((const float*)dev, span, rows, sd, sink);
+    else probe_host_kernel<256><<<blocks, 128, 0, s>>>((const float*)dev, span, rows, sd, sink);
+  };
+  launch(seed ^ 0x5555);  // warm-up (TLB, clocks)
+  cudaEventRecord(e0, s);
+  launch(seed);
+  cudaEventRecord(e1, s);
+  cudaError_t e = cudaEventSynchronize(e1);
+  float ms = 0;
+  if (e == cudaSuccess) e = cudaEventElapsedTime(&ms, e0, e1);
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  cudaFree(sink);
+  if (e != cudaSuccess) return FLECHE_ECUDA;
+  *gbps = (double)rows * (double)row_bytes / ((double)ms * 1e-3) / 1e9;
+  return FLECHE_OK;
+}
+
+}  // extern "C"
