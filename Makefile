@@ -20,3 +20,7 @@ clean:
 	rm -f workload/libflgen.so oracle/libfleche_oracle.so $(PKG)/libfleche.so
 
 .PHONY: all clean
+
+# timing-experiment build (tools only; semantics-breaking knobs behind FLECHE_EXP_MODE)
+$(PKG)/libfleche_exp.so: $(wildcard $(PKG)/csrc/*.cu $(PKG)/csrc/*.cuh) include/fleche.h
+	$(NVCC) $(NVFLAGS) -DFLECHE_EXPERIMENTS -o $@ $(PKG)/csrc/fleche.cu

@@ -44,6 +44,7 @@ def parse():
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=15.0, help="oracle sample budget")
+    p.add_argument("--flags", type=int, default=0, help="fleche_config.flags (ablations)")
     return p.parse_args()
 
 
@@ -229,7 +230,7 @@ def main():
     hostbuf, tabs = w.make_tables()
     t_gen = time.time() - t_gen
     log("create")
-    cache = fl.FlatCache(w.cards, w.dims, tabs, w.cache_bytes, N, local, 1.0, 0, HASH_SEED)
+    cache = fl.FlatCache(w.cards, w.dims, tabs, w.cache_bytes, N, local, 1.0, 0, HASH_SEED, args.flags)
     stream = torch.cuda.current_stream()
 
     def gen_batch(b):

@@ -76,8 +76,13 @@ typedef struct {
                                     < p * 2^64, batch = 0-based query count (R8)        */
   uint64_t admit_seed;
   uint32_t hash_seed;            /* set index = (fmix32(fk ^ hash_seed) * S) >> 32 (R12)  */
-  uint32_t flags;                /* reserved, must be 0                                            */
+  uint32_t flags;                /* bitwise OR of FLECHE_FLAG_*; other bits must be 0              */
 } fleche_config;
+
+/* Experimental: the query kernel starts each unique miss's host-row transfer into L2
+ * (cp.async.bulk.prefetch.L2) so the miss kernel's loads hit L2.  Off by default: it
+ * measured slower on B200 (profiles/README.md, round 1). */
+#define FLECHE_FLAG_L2_PREFETCH 0x1u
 
 typedef struct {
   uint64_t batches;            /* query calls                                                       */

@@ -10,7 +10,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libfleche.so")
+LIB_PATH = os.path.join(_HERE, os.environ.get("FLECHE_LIB", "libfleche.so"))  # FLECHE_LIB: experiment builds
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"libfleche.so not built at {LIB_PATH}: run `make` (or __graft_entry__.build()) first; "
@@ -19,6 +19,7 @@ if not os.path.exists(LIB_PATH):
 _lib = ctypes.CDLL(LIB_PATH)
 
 OK, EINVAL, ENOMEM, ECUDA, ENCCL, ERANGE, ESTATE = 0, -1, -2, -3, -4, -5, -6
+FLAG_L2_PREFETCH = 0x1
 MAX_TABLES = 1024
 
 _vp, _i64, _i32, _u64, _u32 = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32, ctypes.c_uint64, ctypes.c_uint32
@@ -117,7 +118,7 @@ class FlatCache:
     """One flat GPU cache over the given host tables (fleche_create / fleche_query / fleche_stats)."""
 
     def __init__(self, cards, dims, host_tables, cache_bytes: int, max_lookups: int, device: int = 0,
-                 admit_prob: float = 1.0, admit_seed: int = 0, hash_seed: int = 0):
+                 admit_prob: float = 1.0, admit_seed: int = 0, hash_seed: int = 0, flags: int = 0):
         self.n = len(cards)
         self.cards = np.ascontiguousarray(cards, dtype=np.int64)
         self.dims = np.ascontiguousarray(dims, dtype=np.int32)
@@ -125,7 +126,7 @@ class FlatCache:
         self._tp = (_vp * self.n)(*[_ptr(t) for t in self._tables])
         cfg = fleche_config(self.n, self.cards.ctypes.data, self.dims.ctypes.data, int(cache_bytes),
                             ctypes.cast(self._tp, _vp), int(max_lookups), int(device), float(admit_prob),
-                            int(admit_seed), int(hash_seed), 0)
+                            int(admit_seed), int(hash_seed), int(flags))
         h = _vp()
         _check(fleche_create(ctypes.byref(cfg), ctypes.byref(h)), "fleche_create")
         self.h = h.value

@@ -34,6 +34,7 @@ struct fleche_ctx {
   Dev dv{};
   TableInfo* d_tables = nullptr;
   int ki_blocks = 0;
+  int km_bps = 4;  // KM CTAs per SM
   // host-side counters
   uint64_t batches = 0, lookups = 0, kernels = 0;
   // ordering across streams
@@ -258,7 +259,7 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   *out = nullptr;
   const int n = cfg->num_tables;
   if (n < 1 || n > FLECHE_MAX_TABLES || !cfg->cardinalities || !cfg->dims || !cfg->host_tables) return FLECHE_EINVAL;
-  if (cfg->max_lookups < 1 || cfg->max_lookups > (int64_t(1) << 31) || cfg->flags != 0) return FLECHE_EINVAL;
+  if (cfg->max_lookups < 1 || cfg->max_lookups > (int64_t(1) << 31) || (cfg->flags & ~FLECHE_FLAG_L2_PREFETCH)) return FLECHE_EINVAL;
   for (int t = 0; t < n; ++t) {
     const int d = cfg->dims[t];
     if (cfg->cardinalities[t] < 1 || d != cfg->dims[0]) return FLECHE_EINVAL;
@@ -299,6 +300,13 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   dv.admit_all = (p <= 0.0 || p >= 1.0) ? 1 : 0;
   dv.admit_thr = dv.admit_all ? ~0ull : (uint64_t)ldexp(p, 64);
   dv.admit_seed = cfg->admit_seed;
+  dv.prefetch = (cfg->flags & FLECHE_FLAG_L2_PREFETCH) ? 1 : 0;
+  dv.km_m = c->dim <= 32 ? 16 : 8;
+  if (const char* e = getenv("FLECHE_KM_M")) dv.km_m = atoi(e);  // tuning knob (bench sweeps)
+  if (const char* e = getenv("FLECHE_KM_BLOCKS_PER_SM")) c->km_bps = atoi(e);
+#ifdef FLECHE_EXPERIMENTS
+  if (const char* e = getenv("FLECHE_EXP_MODE")) dv.exp_mode = atoi(e);
+#endif
 
   auto alloc = [&](void** p, size_t bytes) { return cudaMalloc(p, bytes) == cudaSuccess; };
   const size_t ways = (size_t)sets * 32u;
@@ -333,7 +341,8 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
     return fail(FLECHE_ECUDA);
   if (cudaEventCreateWithFlags(&c->chain_ev, cudaEventDisableTiming) != cudaSuccess) return fail(FLECHE_ECUDA);
   // KI: enough warps for the expected unique misses, capped at 4 CTAs (32 warps) per SM
-  c->ki_blocks = (int)std::min<int64_t>(4 * c->sm_count, std::max<int64_t>(1, (cfg->max_lookups + 255) / 256));
+  c->ki_blocks = (int)std::min<int64_t>((int64_t)c->km_bps * c->sm_count,
+                                         std::max<int64_t>(1, (cfg->max_lookups + 255) / 256));
   if (cudaDeviceSynchronize() != cudaSuccess) return fail(FLECHE_ECUDA);
   *out = c;
   return FLECHE_OK;

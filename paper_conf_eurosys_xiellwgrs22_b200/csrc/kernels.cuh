@@ -90,6 +90,12 @@ struct Dev {
   uint32_t sets, rows, scr_mask, hash_seed;
   int32_t dim, admit_all;
   uint64_t admit_thr, admit_seed;
+  int32_t prefetch;  // KQ starts each unique miss's host-row transfer into L2
+  int32_t km_m;      // unique misses per KM warp iteration (4, 8, 16, 32)
+#ifdef FLECHE_EXPERIMENTS
+  int32_t exp_mode;  // timing experiments only (libfleche_exp.so); breaks semantics
+  int32_t exp_pad;
+#endif
 };
 
 template <int MAXT>
@@ -342,7 +348,14 @@ __global__ void __launch_bounds__(128) kq_kernel(const __grid_constant__ QArgs<M
       uint32_t b = 0;
       if (lane == __ffs(own_m) - 1) b = atomicAdd(&dv.ctl->counts[par][0], (uint32_t)__popc(own_m));
       b = __shfl_sync(kFull, b, __ffs(own_m) - 1);
-      if (kind == 1) dv.miss[b + __popc(own_m & lt)] = MissRec{off, fk, scr, t, 0};
+      if (kind == 1) {
+        dv.miss[b + __popc(own_m & lt)] = MissRec{off, fk, scr, t, 0};
+        // start the host-link transfer now: KM's loads of this row then hit L2
+        if (dv.prefetch) {
+          const float* hrow = ti->host + (size_t)id * (size_t)d;
+          asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(hrow), "r"(4u * (unsigned)d) : "memory");
+        }
+      }
     }
     if (dup_m) {
       uint32_t b = 0;
@@ -415,14 +428,13 @@ __device__ __forceinline__ int64_t claim_victim(const Dev& dv, uint32_t fk, uint
 }
 
 // KM for row width D: each warp iteration handles M unique misses.
-template <int D>
+template <int D, int M>
 __device__ __forceinline__ void km_rows(const Dev& dv, float* __restrict__ out, uint32_t epoch, uint32_t nmiss,
                                         int lane, uint32_t gw, uint32_t nw, unsigned& ins, unsigned& ev,
                                         unsigned& byp, unsigned long long& hostb) {
-  constexpr int M = D <= 32 ? 16 : (D <= 128 ? 8 : 4);  // misses per warp iteration
   for (uint32_t base = gw * M; base < nmiss; base += nw * M) {
     const uint32_t k = base + lane;
-    const bool has = lane < M && k < nmiss;
+    bool has = lane < M && k < nmiss;
     MissRec m{};
     const float* src = nullptr;
     if (has) {
@@ -430,6 +442,10 @@ __device__ __forceinline__ void km_rows(const Dev& dv, float* __restrict__ out, 
       const TableInfo* ti = dv.tables + m.t;
       src = ti->host + (size_t)(m.fk - ti->base) * D;  // unified index: computed host address
     }
+#ifdef FLECHE_EXPERIMENTS
+    if (dv.exp_mode == 2) src = nullptr;  // timing experiment: no host loads
+    if (dv.exp_mode == 1) has = false;    // timing experiment: loads only, no claim/store
+#endif
     // A6: all of this warp's host-row loads go out now (zero-copy over the host link)
     RowBuf<D, M> rb;
     rb.load(src, lane);
@@ -489,15 +505,25 @@ __global__ void __launch_bounds__(128) km_kernel(const __grid_constant__ Dev dv,
   const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
   unsigned ins = 0, ev = 0, byp = 0;
   unsigned long long hostb = 0;
-  switch (dv.dim) {
-    case 8: km_rows<8>(dv, out, epoch, nmiss, lane, gw, nw, ins, ev, byp, hostb); break;
-    case 16: km_rows<16>(dv, out, epoch, nmiss, lane, gw, nw, ins, ev, byp, hostb); break;
-    case 32: km_rows<32>(dv, out, epoch, nmiss, lane, gw, nw, ins, ev, byp, hostb); break;
-    case 64: km_rows<64>(dv, out, epoch, nmiss, lane, gw, nw, ins, ev, byp, hostb); break;
-    case 128: km_rows<128>(dv, out, epoch, nmiss, lane, gw, nw, ins, ev, byp, hostb); break;
-    case 256: km_rows<256>(dv, out, epoch, nmiss, lane, gw, nw, ins, ev, byp, hostb); break;
-    default: break;  // fleche_create only admits the widths above
+#define FL_KM(D, M) km_rows<D, M>(dv, out, epoch, nmiss, lane, gw, nw, ins, ev, byp, hostb)
+#define FL_KM_MS(D)                    \
+  switch (dv.km_m) {                   \
+    case 4: FL_KM(D, 4); break;        \
+    case 16: FL_KM(D, 16); break;      \
+    case 32: FL_KM(D, 32); break;      \
+    default: FL_KM(D, 8); break;       \
   }
+  switch (dv.dim) {  // fleche_create only admits these widths
+    case 8: FL_KM_MS(8); break;
+    case 16: FL_KM_MS(16); break;
+    case 32: FL_KM_MS(32); break;
+    case 64: FL_KM_MS(64); break;
+    case 128: if (dv.km_m <= 4) FL_KM(128, 4); else FL_KM(128, 8); break;
+    case 256: FL_KM(256, 4); break;
+    default: break;
+  }
+#undef FL_KM_MS
+#undef FL_KM
   ins = __reduce_add_sync(kFull, ins);
   ev = __reduce_add_sync(kFull, ev);
   byp = __reduce_add_sync(kFull, byp);
