@@ -49,19 +49,23 @@ typedef enum {
   FLECHE_ESTATE = -6  /* ctx poisoned by an earlier CUDA error                                */
 } fleche_status;
 
-#define FLECHE_MAX_TABLES 1024
+#define FLECHE_MAX_TABLES 512 /* per-call table arguments travel as kernel parameters (<= 32 KB) */
 
 typedef struct {
   int32_t num_tables;            /* n, 1 <= n <= FLECHE_MAX_TABLES                               */
   const int64_t* cardinalities;  /* [n] host array: c_t >= 1 rows of table t                    */
   const int32_t* dims;           /* [n] host array: d_t in {8, 16, 32, 64, 128, 256} (rows are moved
                                     as 16-byte vectors by warp-shaped kernels specialised per
-                                    width).  Round 1: all d_t must be equal (one slab class);
-                                    mixed dims return FLECHE_EINVAL.                              */
+                                    width).  One width for all tables -> uniform layout (32-way
+                                    sets of equal rows); mixed widths -> bytes layout (32-way sets
+                                    sharing a 4 KiB row region each: one byte budget for every
+                                    width, the flat cache's elastic per-table capacity, P:L801-804;
+                                    slabs per width as in Fig 5c).                    */
   uint64_t cache_bytes;          /* HBM budget for cached embedding ROWS (the paper expresses the
                                     cache size as a fraction of all table bytes);
-                                    capacity = floor(cache_bytes / (4 d)) rows.  The index
-                                    (8 B per row) and scratch are reported in index_bytes.       */
+                                    uniform: capacity = floor(cache_bytes / (4 d)) rows; bytes:
+                                    floor(cache_bytes / 4096) sets x 4096 B.  The index and the
+                                    scratch are reported separately in index_bytes.               */
   const float* const* host_tables;/* [n] host array of host pointers: E_t row-major c_t x d_t fp32,
                                     16-byte aligned, caller-owned, must outlive the ctx.  The ctx
                                     page-locks and maps them (cudaHostRegister Mapped|Portable)
@@ -124,6 +128,22 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out);
 fleche_status fleche_query(fleche_ctx* ctx, const int64_t* const* ids, const int64_t* lengths, float* out,
                            fleche_stream stream);
 
+/* One batch of multi-hot lookups with sum pooling per bag (pooling).
+ *   ids[t]     : DEVICE pointer to nnz[t] int64 IDs of table t (all bags, concatenated).
+ *   offsets[t] : DEVICE pointer to bags[t] + 1 int64 CSR offsets into ids[t]:
+ *                bag b = ids[t][offsets[t][b] .. offsets[t][b+1]); offsets[t][0] = 0 and
+ *                offsets[t][bags[t]] = nnz[t] (the caller guarantees this; not checked).
+ *   bags, nnz  : HOST arrays; sum_t nnz[t] <= max_lookups.
+ *   out        : DEVICE fp32, table t starts at float offset sum_{u<t} bags[u] * d_u; bag b's
+ *                row = fp32 sum of E_t[id] over its valid IDs, accumulated sequentially in
+ *                bag order (reading R16: the oracle's order, so results are bit-identical);
+ *                an empty bag gives a zero row; invalid IDs contribute nothing.
+ * Every ID is a lookup for the cache (hit/miss/insert as in fleche_query).  Enqueues
+ * 3 kernels (query, miss, pooling); the per-ID rows are staged in a ctx-owned buffer
+ * (max_lookups x max d floats, allocated at the first pooled call). */
+fleche_status fleche_query_pooled(fleche_ctx* ctx, const int64_t* const* ids, const int64_t* const* offsets,
+                                  const int64_t* bags, const int64_t* nnz, float* out, fleche_stream stream);
+
 /* Same lookups with HOST buffers: ids[t] are host pointers (ideally pinned), out is a
  * host buffer.  Enqueues host->device copies of the IDs, the query, and the
  * device->host copy of out on `stream` (ctx-owned device staging, allocated at the
@@ -145,14 +165,19 @@ const char* fleche_strerror(fleche_status status);
 /* Introspection for tests.
  * fleche_get_encoding: base[t] (first flat key of table t), fbits[t] (feature bits),
  *   *key_bits = minimal key width B_min of the size-aware code.
- * fleche_get_geometry: number of index sets S, capacity rows, row floats d.
+ * fleche_get_geometry: number of index sets S; uniform layout: capacity rows and row
+ *   floats d; bytes layout: rows = 0 and row_floats = -(floats of one set's region).
  * fleche_debug_snapshot: blocking copy of the index (keys[S*32], ts[S*32]; uint32,
- *   EMPTY key = 0xFFFFFFFF) and of the slab (S*32 rows x d floats; row of way w of set
- *   s at (s*32 + w) * d) into host buffers of at least the given element counts. */
+ *   EMPTY key = 0xFFFFFFFF) and of the slab (uniform: S*32 rows x d floats, row of way w
+ *   of set s at (s*32 + w) * d; bytes: S regions) into host buffers of at least the
+ *   given element counts.
+ * fleche_debug_locations: bytes layout only: loc[S*32] = (size << 8) | offset of each
+ *   way's row inside its set's region, both in 32-byte units. */
 fleche_status fleche_get_encoding(fleche_ctx* ctx, uint64_t* base, int32_t* fbits, int32_t* key_bits);
 fleche_status fleche_get_geometry(fleche_ctx* ctx, int64_t* sets, int64_t* rows, int32_t* row_floats);
 fleche_status fleche_debug_snapshot(fleche_ctx* ctx, uint32_t* keys, uint32_t* ts, size_t ways_cap, float* slab,
                                     size_t slab_floats_cap);
+fleche_status fleche_debug_locations(fleche_ctx* ctx, uint16_t* loc, size_t ways_cap);
 
 /* Diagnostics for measurement (bench.py).
  * fleche_set_profiling: when enabled, every later query records CUDA events on its

@@ -19,6 +19,7 @@ _lib = None
 
 MODE_GLOBAL = 0
 MODE_SETASSOC = 1
+MODE_SETBYTES = 2
 
 STAT_FIELDS = ["batches", "lookups", "hits", "misses", "invalid", "unique_keys", "unique_hits", "unique_misses",
                "inserted", "evicted", "bypassed", "occupancy_bytes", "capacity_bytes", "bypass_full"]
@@ -44,6 +45,8 @@ def lib():
         L.or_set_hash.argtypes = [u32, u32]
         L.or_create.restype = vp
         L.or_create.argtypes = [ctypes.c_int, vp, vp, vp, u64, ctypes.c_int, ctypes.c_double, u64, u32]
+        L.or_create_setbytes.restype = vp
+        L.or_create_setbytes.argtypes = [ctypes.c_int, vp, vp, vp, u64, ctypes.c_int, u64, ctypes.c_double, u64, u32]
         L.or_destroy.restype = None
         L.or_destroy.argtypes = [vp]
         L.or_query.restype = ctypes.c_int
@@ -91,7 +94,7 @@ class Oracle:
     """CPU reference cache.  ``tables`` are float32 [c_t, d_t] arrays (kept alive here)."""
 
     def __init__(self, cards, dims, tables, cache_bytes: int, mode: int = MODE_GLOBAL, admit_p: float = 1.0,
-                 admit_seed: int = 0, hash_seed: int = 0):
+                 admit_seed: int = 0, hash_seed: int = 0, ways: int = 32, set_bytes: int = 8192):
         self.n = len(cards)
         self.cards = np.ascontiguousarray(cards, dtype=np.int64)
         self.dims = np.ascontiguousarray(dims, dtype=np.int32)
@@ -99,8 +102,12 @@ class Oracle:
         for t, (c, d) in zip(self.tables, zip(cards, dims)):
             assert t.shape == (c, d)
         self._tp = _ptr_array(self.tables)
-        self.h = lib().or_create(self.n, self.cards.ctypes.data, self.dims.ctypes.data, self._tp, cache_bytes, mode,
-                                 admit_p, admit_seed, hash_seed)
+        if mode == MODE_SETBYTES:
+            self.h = lib().or_create_setbytes(self.n, self.cards.ctypes.data, self.dims.ctypes.data, self._tp,
+                                              cache_bytes, ways, set_bytes, admit_p, admit_seed, hash_seed)
+        else:
+            self.h = lib().or_create(self.n, self.cards.ctypes.data, self.dims.ctypes.data, self._tp, cache_bytes,
+                                     mode, admit_p, admit_seed, hash_seed)
         if not self.h:
             raise ValueError("or_create rejected the configuration")
 

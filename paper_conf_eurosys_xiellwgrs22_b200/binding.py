@@ -20,7 +20,7 @@ _lib = ctypes.CDLL(LIB_PATH)
 
 OK, EINVAL, ENOMEM, ECUDA, ENCCL, ERANGE, ESTATE = 0, -1, -2, -3, -4, -5, -6
 FLAG_L2_PREFETCH = 0x1
-MAX_TABLES = 1024
+MAX_TABLES = 512
 
 _vp, _i64, _i32, _u64, _u32 = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32, ctypes.c_uint64, ctypes.c_uint32
 
@@ -67,9 +67,13 @@ fleche_kernel_times = _sig("fleche_kernel_times", ctypes.c_int, [_vp, ctypes.POI
 fleche_probe_host_read = _sig("fleche_probe_host_read", ctypes.c_int, [_vp, _u64, _i32, _i64, _u64, _vp,
                                                                        ctypes.POINTER(ctypes.c_double)])
 
-EXPORTED = ["fleche_create", "fleche_query", "fleche_query_host", "fleche_stats", "fleche_reset_stats",
-            "fleche_destroy", "fleche_strerror", "fleche_get_encoding", "fleche_get_geometry",
-            "fleche_debug_snapshot", "fleche_set_profiling", "fleche_kernel_times", "fleche_probe_host_read"]
+fleche_query_pooled = _sig("fleche_query_pooled", ctypes.c_int, [_vp, _vp, _vp, _vp, _vp, _vp, _vp])
+fleche_debug_locations = _sig("fleche_debug_locations", ctypes.c_int, [_vp, _vp, ctypes.c_size_t])
+
+EXPORTED = ["fleche_create", "fleche_query", "fleche_query_pooled", "fleche_query_host", "fleche_stats",
+            "fleche_reset_stats", "fleche_destroy", "fleche_strerror", "fleche_get_encoding", "fleche_get_geometry",
+            "fleche_debug_snapshot", "fleche_debug_locations", "fleche_set_profiling", "fleche_kernel_times",
+            "fleche_probe_host_read"]
 
 
 def probe_host_read(host_ptr: int, nbytes: int, row_bytes: int, rows: int, seed: int = 1, stream=None) -> float:
@@ -155,6 +159,27 @@ class FlatCache:
         ip = (_vp * self.n)(*[_ptr(x) for x in ids])
         _check(fleche_query(self.h, ip, lp, _ptr(out), _stream_handle(stream)), "fleche_query")
 
+    def pooled_floats(self, bags) -> int:
+        return int(sum(int(b) * int(d) for b, d in zip(bags, self.dims)))
+
+    def query_pooled(self, ids, offsets, out, stream=None, bags=None, nnz=None):
+        """ids/offsets: lists of n device int64 tensors (CSR per table); out: device fp32 buffer."""
+        if bags is None:
+            bags = [int(o.numel()) - 1 for o in offsets]
+        if nnz is None:
+            nnz = [int(x.numel()) for x in ids]
+        bp = (_i64 * self.n)(*bags)
+        npp = (_i64 * self.n)(*nnz)
+        ip = (_vp * self.n)(*[_ptr(x) for x in ids])
+        op = (_vp * self.n)(*[_ptr(o) for o in offsets])
+        _check(fleche_query_pooled(self.h, ip, op, bp, npp, _ptr(out), _stream_handle(stream)), "fleche_query_pooled")
+
+    def locations(self):
+        sets, _, _ = self.geometry()
+        loc = np.empty(sets * 32, np.uint16)
+        _check(fleche_debug_locations(self.h, loc.ctypes.data, loc.size), "fleche_debug_locations")
+        return loc
+
     def query_host(self, ids, out, stream=None, lengths=None):
         """ids: list of n host int64 arrays (ideally pinned); out: host fp32 buffer."""
         if lengths is None:
@@ -196,10 +221,13 @@ class FlatCache:
         return int(s.value), int(r.value), int(d.value)
 
     def snapshot(self):
+        """keys, ts and the slab: uniform layout -> [S*32, d] rows; bytes layout -> [S, region floats]."""
         sets, rows, d = self.geometry()
         keys = np.empty(sets * 32, np.uint32)
         ts = np.empty(sets * 32, np.uint32)
-        slab = np.empty(sets * 32 * d, np.float32)
+        per = d if d > 0 else -d
+        nrow = sets * 32 if d > 0 else sets
+        slab = np.empty(nrow * per, np.float32)
         _check(fleche_debug_snapshot(self.h, keys.ctypes.data, ts.ctypes.data, keys.size, slab.ctypes.data, slab.size),
                "fleche_debug_snapshot")
-        return keys, ts, slab.reshape(sets * 32, d)
+        return keys, ts, slab.reshape(nrow, per)

@@ -9,6 +9,7 @@
 
 #include <algorithm>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <vector>
@@ -21,33 +22,39 @@ using namespace fl;
 struct fleche_ctx {
   int device = 0;
   int n = 0;
-  int dim = 0;
+  int max_dim = 0;
   int sm_count = 148;
   bool poisoned = false;
   int64_t max_lookups = 0;
   std::vector<int64_t> card;
   std::vector<int32_t> dims;
+  std::vector<int32_t> cls;      // width class of each table
+  std::vector<int32_t> cls_dim;  // row width of each class (ascending)
   std::vector<uint64_t> base;
   std::vector<int32_t> fbits;
   int key_bits = 0;
+  uint64_t capacity_bytes = 0;
   std::vector<std::pair<void*, size_t>> registered;  // host ranges we registered
   Dev dv{};
   TableInfo* d_tables = nullptr;
-  int ki_blocks = 0;
+  int km_blocks = 0;
   int km_bps = 4;  // KM CTAs per SM
+  size_t km_smem = 0;
   // host-side counters
   uint64_t batches = 0, lookups = 0, kernels = 0;
   // ordering across streams
   cudaStream_t last_stream = nullptr;
   bool have_last = false;
   cudaEvent_t chain_ev = nullptr;
-  // fleche_query_host staging (lazy)
+  // fleche_query_host staging and pooled staging (lazy)
   int64_t* d_ids_stage = nullptr;
   float* d_out_stage = nullptr;
+  float* d_pool_stage = nullptr;
   uint64_t index_bytes = 0;
   // profiling (fleche_set_profiling)
   bool profiling = false;
-  std::vector<cudaEvent_t> ev_pool;  // 3 per profiled query
+  std::vector<cudaEvent_t> ev_pool;  // 3 or 4 per profiled query
+  std::vector<int> ev_kinds;         // events recorded per profiled query (3 = one-hot, 4 = pooled)
   size_t ev_used = 0;
 };
 
@@ -104,8 +111,11 @@ uint32_t next_pow2(uint64_t x) {
   return (uint32_t)p;
 }
 
-// Page-lock and map the caller's tables.  Ranges are merged on page boundaries
-// (tables usually share one allocation, and a page may only be registered once).
+bool valid_dim(int d) { return d == 8 || d == 16 || d == 32 || d == 64 || d == 128 || d == 256; }
+
+// Page-lock and map the caller's tables.  Ranges that touch a common page are
+// registered together (tables usually share one allocation; a page can be
+// registered only once).
 fleche_status register_host(fleche_ctx* c, const float* const* host, std::vector<const float*>& dev_ptrs) {
   const uintptr_t pg = 4096;
   std::vector<std::pair<uintptr_t, uintptr_t>> r;
@@ -115,7 +125,7 @@ fleche_status register_host(fleche_ctx* c, const float* const* host, std::vector
   }
   std::sort(r.begin(), r.end());
   std::vector<std::pair<uintptr_t, uintptr_t>> m;
-  for (auto& x : r) {  // ranges that touch a common page are registered together
+  for (auto& x : r) {
     if (!m.empty() && (x.first & ~(pg - 1)) <= ((m.back().second - 1) & ~(pg - 1)))
       m.back().second = std::max(m.back().second, x.second);
     else
@@ -128,7 +138,7 @@ fleche_status register_host(fleche_ctx* c, const float* const* host, std::vector
     cudaGetLastError();
     cudaError_t e = cudaHostRegister(p, x.second - x.first, cudaHostRegisterMapped | cudaHostRegisterPortable);
     if (e == cudaErrorHostMemoryAlreadyRegistered) {
-      cudaGetLastError();  // caller pinned it already (cudaHostAlloc / earlier ctx)
+      cudaGetLastError();
       continue;
     }
     if (e != cudaSuccess) return poison(c, e, "cudaHostRegister");
@@ -144,8 +154,9 @@ fleche_status register_host(fleche_ctx* c, const float* const* host, std::vector
 }
 
 void free_all(fleche_ctx* c) {
-  void* ptrs[] = {c->dv.keys, c->dv.ts, c->dv.slab, c->dv.scratch, c->dv.dup_head, c->dv.miss, c->dv.dup,
-                  c->dv.ctl, c->dv.stats, c->d_tables, c->d_ids_stage, c->d_out_stage};
+  void* ptrs[] = {c->dv.keys, c->dv.ts, c->dv.loc, c->dv.lock, c->dv.slab, c->dv.scratch, c->dv.dup_head,
+                  c->dv.miss, c->dv.dup, c->dv.ctl, c->dv.stats, c->d_tables, c->d_ids_stage, c->d_out_stage,
+                  c->d_pool_stage};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   for (auto& r : c->registered) cudaHostUnregister(r.first);
@@ -172,13 +183,31 @@ fleche_status order_on(fleche_ctx* c, cudaStream_t s) {
   return FLECHE_OK;
 }
 
+fleche_status prof_event(fleche_ctx* c, cudaStream_t s, bool first, int kinds) {
+  if (!c->profiling) return FLECHE_OK;
+  if (c->ev_pool.size() <= c->ev_used) {
+    cudaEvent_t e;
+    FL_CUDA(c, cudaEventCreate(&e));
+    c->ev_pool.push_back(e);
+  }
+  if (first) c->ev_kinds.push_back(kinds);
+  FL_CUDA(c, cudaEventRecord(c->ev_pool[c->ev_used++], s));
+  return FLECHE_OK;
+}
+
+// KQ + KM for one batch of one-hot lookups into `out` (table-major rows).
 template <int MAXT>
 fleche_status launch_query(fleche_ctx* c, const int64_t* const* ids, const int64_t* lengths, float* out,
-                           cudaStream_t s, int64_t total) {
+                           cudaStream_t s, int64_t total, int nev) {
   QArgs<MAXT> qa;
   memset(&qa, 0, sizeof(qa));
   qa.n = c->n;
   qa.out = out;
+  KMArgs ka;
+  memset(&ka, 0, sizeof(ka));
+  ka.out = out;
+  ka.ncls = (int)c->cls_dim.size();
+  int64_t cls_len[8] = {0};
   int64_t acc = 0, oacc = 0;
   for (int t = 0; t < c->n; ++t) {
     qa.ids[t] = ids[t];
@@ -186,35 +215,34 @@ fleche_status launch_query(fleche_ctx* c, const int64_t* const* ids, const int64
     qa.out_off[t] = oacc;
     acc += lengths[t];
     oacc += lengths[t] * (int64_t)c->dims[t];
+    cls_len[c->cls[t]] += lengths[t];
   }
   qa.scan[c->n] = acc;
-  cudaEvent_t ev[3] = {nullptr, nullptr, nullptr};
-  if (c->profiling) {
-    while (c->ev_pool.size() < c->ev_used + 3) {
-      cudaEvent_t e;
-      FL_CUDA(c, cudaEventCreate(&e));
-      c->ev_pool.push_back(e);
-    }
-    for (int i = 0; i < 3; ++i) ev[i] = c->ev_pool[c->ev_used + i];
-    c->ev_used += 3;
-    FL_CUDA(c, cudaEventRecord(ev[0], s));
+  int64_t coff = 0;  // each width's region of the miss list: at most its lookups
+  for (int k = 0; k < ka.ncls; ++k) {
+    qa.cls_off[k] = ka.cls_off[k] = coff;
+    ka.cls_dim[k] = c->cls_dim[k];
+    coff += cls_len[k];
   }
+  fleche_status st = prof_event(c, s, true, nev);
+  if (st != FLECHE_OK) return st;
   if (total > 0) {
     const int64_t blocks = (total + 127) / 128;
     kq_kernel<MAXT><<<(unsigned)blocks, 128, 0, s>>>(qa, c->dv);
     c->kernels++;
   }
-  if (ev[1]) FL_CUDA(c, cudaEventRecord(ev[1], s));
-  km_kernel<<<c->ki_blocks, 128, 0, s>>>(c->dv, out);
+  if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
+  if (c->dv.bytes) km_kernel<true><<<c->km_blocks, 128, c->km_smem, s>>>(c->dv, ka);
+  else km_kernel<false><<<c->km_blocks, 128, 0, s>>>(c->dv, ka);
   c->kernels++;
-  if (ev[2]) FL_CUDA(c, cudaEventRecord(ev[2], s));
+  if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return poison(c, e, "kernel launch");
   return FLECHE_OK;
 }
 
 fleche_status query_impl(fleche_ctx* c, const int64_t* const* ids, const int64_t* lengths, float* out,
-                         cudaStream_t s) {
+                         cudaStream_t s, int nev = 3) {
   int64_t total = 0;
   for (int t = 0; t < c->n; ++t) {
     if (lengths[t] < 0) return FLECHE_EINVAL;
@@ -227,14 +255,44 @@ fleche_status query_impl(fleche_ctx* c, const int64_t* const* ids, const int64_t
   if (st != FLECHE_OK) return st;
   st = order_on(c, s);
   if (st != FLECHE_OK) return st;
-  if (c->n <= 32) st = launch_query<32>(c, ids, lengths, out, s, total);
-  else if (c->n <= 128) st = launch_query<128>(c, ids, lengths, out, s, total);
-  else st = launch_query<FLECHE_MAX_TABLES>(c, ids, lengths, out, s, total);
+  if (c->n <= 32) st = launch_query<32>(c, ids, lengths, out, s, total, nev);
+  else if (c->n <= 128) st = launch_query<128>(c, ids, lengths, out, s, total, nev);
+  else st = launch_query<FLECHE_MAX_TABLES>(c, ids, lengths, out, s, total, nev);
   if (st == FLECHE_OK) {
     c->batches++;
     c->lookups += (uint64_t)total;
   }
   return st;
+}
+
+template <int MAXT>
+fleche_status launch_pool(fleche_ctx* c, const int64_t* const* offsets, const int64_t* bags, const int64_t* nnz,
+                          float* out, cudaStream_t s) {
+  PArgs<MAXT> pa;
+  memset(&pa, 0, sizeof(pa));
+  pa.n = c->n;
+  pa.stage = c->d_pool_stage;
+  pa.out = out;
+  int64_t cs = 0, so = 0, oo = 0;
+  for (int t = 0; t < c->n; ++t) {
+    pa.offs[t] = offsets[t];
+    pa.cscan[t] = cs;
+    pa.stage_off[t] = so;
+    pa.out_off[t] = oo;
+    cs += bags[t] * (int64_t)(c->dims[t] / 4);
+    so += nnz[t] * (int64_t)c->dims[t];
+    oo += bags[t] * (int64_t)c->dims[t];
+  }
+  pa.cscan[c->n] = cs;
+  if (cs > 0) {
+    kp_kernel<MAXT><<<(unsigned)((cs + 255) / 256), 256, 0, s>>>(pa, c->d_tables);
+    c->kernels++;
+  }
+  fleche_status st = prof_event(c, s, false, 0);
+  if (st != FLECHE_OK) return st;
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return poison(c, e, "kernel launch");
+  return FLECHE_OK;
 }
 
 }  // namespace
@@ -259,24 +317,29 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   *out = nullptr;
   const int n = cfg->num_tables;
   if (n < 1 || n > FLECHE_MAX_TABLES || !cfg->cardinalities || !cfg->dims || !cfg->host_tables) return FLECHE_EINVAL;
-  if (cfg->max_lookups < 1 || cfg->max_lookups > (int64_t(1) << 31) || (cfg->flags & ~FLECHE_FLAG_L2_PREFETCH)) return FLECHE_EINVAL;
+  if (cfg->max_lookups < 1 || cfg->max_lookups > (int64_t(1) << 31) || (cfg->flags & ~FLECHE_FLAG_L2_PREFETCH))
+    return FLECHE_EINVAL;
   for (int t = 0; t < n; ++t) {
-    const int d = cfg->dims[t];
-    if (cfg->cardinalities[t] < 1 || d != cfg->dims[0]) return FLECHE_EINVAL;
-    if (d != 8 && d != 16 && d != 32 && d != 64 && d != 128 && d != 256) return FLECHE_EINVAL;
+    if (cfg->cardinalities[t] < 1 || !valid_dim(cfg->dims[t])) return FLECHE_EINVAL;
     if (!cfg->host_tables[t] || ((uintptr_t)cfg->host_tables[t] & 15u)) return FLECHE_EINVAL;
   }
   fleche_ctx* c = new (std::nothrow) fleche_ctx();
   if (!c) return FLECHE_ENOMEM;
   c->device = cfg->device;
   c->n = n;
-  c->dim = cfg->dims[0];
   c->max_lookups = cfg->max_lookups;
   c->card.assign(cfg->cardinalities, cfg->cardinalities + n);
   c->dims.assign(cfg->dims, cfg->dims + n);
   c->key_bits = size_aware_code(c->card, c->base, c->fbits);
-  const uint64_t rows = cfg->cache_bytes / (4ull * (uint64_t)c->dim);
-  if (c->key_bits < 0 || rows > 0xFFFFFFE0ull) {
+  for (int t = 0; t < n; ++t)
+    if (std::find(c->cls_dim.begin(), c->cls_dim.end(), c->dims[t]) == c->cls_dim.end()) c->cls_dim.push_back(c->dims[t]);
+  std::sort(c->cls_dim.begin(), c->cls_dim.end());
+  c->cls.resize(n);
+  for (int t = 0; t < n; ++t)
+    c->cls[t] = (int)(std::find(c->cls_dim.begin(), c->cls_dim.end(), c->dims[t]) - c->cls_dim.begin());
+  c->max_dim = c->cls_dim.back();
+  const bool bytes = c->cls_dim.size() > 1;
+  if (c->key_bits < 0) {
     delete c;
     return FLECHE_EINVAL;
   }
@@ -288,12 +351,31 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   if (cudaSetDevice(c->device) != cudaSuccess) return fail(FLECHE_EINVAL);
   cudaDeviceGetAttribute(&c->sm_count, cudaDevAttrMultiProcessorCount, c->device);
 
-  const uint64_t sets = std::max<uint64_t>(1, (rows + 31) / 32);
-  const uint32_t scr_n = next_pow2(std::max<uint64_t>(1024, 2ull * (uint64_t)cfg->max_lookups));
   Dev& dv = c->dv;
+  uint64_t sets, rows = 0;
+  size_t slab_bytes;
+  if (!bytes) {  // uniform layout: way w of set s = slab row 32s + w
+    rows = cfg->cache_bytes / (4ull * (uint64_t)c->max_dim);
+    if (rows > 0xFFFFFFE0ull) return fail(FLECHE_EINVAL);
+    sets = std::max<uint64_t>(1, (rows + 31) / 32);
+    slab_bytes = (size_t)sets * 32u * (size_t)c->max_dim * 4u;
+    c->capacity_bytes = rows * 4ull * (uint64_t)c->max_dim;
+  } else {       // bytes layout: every set owns a set_bytes region (R22)
+    uint64_t set_bytes = 4096;
+    if (const char* e = getenv("FLECHE_SET_BYTES")) set_bytes = strtoull(e, nullptr, 10);
+    if (set_bytes < 1024 || set_bytes > 4096 || (set_bytes & 31)) return fail(FLECHE_EINVAL);
+    sets = cfg->cache_bytes / set_bytes;
+    dv.set_units = sets ? (uint32_t)(set_bytes / 32) : 0u;  // a budget below one set caches nothing
+    sets = std::max<uint64_t>(1, sets);
+    if (sets > 0xFFFFFFF0ull / 32) return fail(FLECHE_EINVAL);
+    slab_bytes = (size_t)sets * set_bytes;
+    c->capacity_bytes = dv.set_units ? sets * set_bytes : 0;
+  }
+  const uint32_t scr_n = next_pow2(std::max<uint64_t>(1024, 2ull * (uint64_t)cfg->max_lookups));
+  dv.bytes = bytes ? 1 : 0;
   dv.sets = (uint32_t)sets;
   dv.rows = (uint32_t)rows;
-  dv.dim = c->dim;
+  dv.dim = c->max_dim;
   dv.hash_seed = cfg->hash_seed;
   dv.scr_mask = scr_n - 1;
   const double p = cfg->admit_prob;
@@ -301,33 +383,36 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   dv.admit_thr = dv.admit_all ? ~0ull : (uint64_t)ldexp(p, 64);
   dv.admit_seed = cfg->admit_seed;
   dv.prefetch = (cfg->flags & FLECHE_FLAG_L2_PREFETCH) ? 1 : 0;
-  dv.km_m = c->dim <= 32 ? 16 : 8;
+  dv.km_m = c->max_dim <= 32 ? 16 : 8;
   if (const char* e = getenv("FLECHE_KM_M")) dv.km_m = atoi(e);  // tuning knob (bench sweeps)
-  if (const char* e = getenv("FLECHE_KM_BLOCKS_PER_SM")) c->km_bps = atoi(e);
+  if (bytes) dv.km_m = std::min(dv.km_m, 8);                     // smem staging holds <= 4 KB of rows
+  if (const char* e = getenv("FLECHE_KM_BLOCKS_PER_SM")) c->km_bps = std::max(1, atoi(e));
 #ifdef FLECHE_EXPERIMENTS
   if (const char* e = getenv("FLECHE_EXP_MODE")) dv.exp_mode = atoi(e);
 #endif
 
-  auto alloc = [&](void** p, size_t bytes) { return cudaMalloc(p, bytes) == cudaSuccess; };
+  auto alloc = [&](void** ptr, size_t b) { return cudaMalloc(ptr, std::max<size_t>(b, 16)) == cudaSuccess; };
   const size_t ways = (size_t)sets * 32u;
-  bool ok = alloc((void**)&dv.keys, ways * 4) && alloc((void**)&dv.ts, ways * 4) &&
-            alloc((void**)&dv.slab, ways * (size_t)c->dim * 4) &&
+  bool ok = alloc((void**)&dv.keys, ways * 4) && alloc((void**)&dv.ts, ways * 4) && alloc((void**)&dv.slab, slab_bytes) &&
             alloc((void**)&dv.scratch, (size_t)scr_n * 8) && alloc((void**)&dv.dup_head, (size_t)scr_n * 8) &&
             alloc((void**)&dv.miss, (size_t)cfg->max_lookups * sizeof(MissRec)) &&
-            alloc((void**)&dv.dup, (size_t)cfg->max_lookups * sizeof(DupRec)) &&
-            alloc((void**)&dv.ctl, sizeof(Ctl)) &&
+            alloc((void**)&dv.dup, (size_t)cfg->max_lookups * sizeof(DupRec)) && alloc((void**)&dv.ctl, sizeof(Ctl)) &&
             alloc((void**)&dv.stats, sizeof(unsigned long long) * kStripes * kNumCtr) &&
             alloc((void**)&c->d_tables, sizeof(TableInfo) * n);
+  if (ok && bytes) ok = alloc((void**)&dv.loc, ways * 2) && alloc((void**)&dv.lock, (size_t)sets * 4);
   if (!ok) {
     cudaGetLastError();
     return fail(FLECHE_ENOMEM);
   }
-  c->index_bytes = ways * 8 + (size_t)scr_n * 16 + (size_t)cfg->max_lookups * (sizeof(MissRec) + sizeof(DupRec));
+  c->index_bytes = ways * (bytes ? 10 : 8) + (bytes ? (size_t)sets * 4 : 0) + (size_t)scr_n * 16 +
+                   (size_t)cfg->max_lookups * (sizeof(MissRec) + sizeof(DupRec));
   dv.tables = c->d_tables;
   if (cudaMemset(dv.keys, 0xFF, ways * 4) != cudaSuccess || cudaMemset(dv.ts, 0, ways * 4) != cudaSuccess ||
       cudaMemset(dv.scratch, 0, (size_t)scr_n * 8) != cudaSuccess ||
       cudaMemset(dv.dup_head, 0, (size_t)scr_n * 8) != cudaSuccess ||
       cudaMemset(dv.stats, 0, sizeof(unsigned long long) * kStripes * kNumCtr) != cudaSuccess)
+    return fail(FLECHE_ECUDA);
+  if (bytes && (cudaMemset(dv.loc, 0, ways * 2) != cudaSuccess || cudaMemset(dv.lock, 0, (size_t)sets * 4) != cudaSuccess))
     return fail(FLECHE_ECUDA);
   Ctl ctl{};
   ctl.epoch = 1;
@@ -336,13 +421,14 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   std::vector<const float*> dptr;
   if (register_host(c, cfg->host_tables, dptr) != FLECHE_OK) return fail(FLECHE_ECUDA);
   std::vector<TableInfo> ti(n);
-  for (int t = 0; t < n; ++t) ti[t] = TableInfo{dptr[t], c->card[t], (uint32_t)c->base[t], c->dims[t]};
+  for (int t = 0; t < n; ++t) ti[t] = TableInfo{dptr[t], c->card[t], (uint32_t)c->base[t], c->dims[t], c->cls[t], 0};
   if (cudaMemcpy(c->d_tables, ti.data(), sizeof(TableInfo) * n, cudaMemcpyHostToDevice) != cudaSuccess)
     return fail(FLECHE_ECUDA);
   if (cudaEventCreateWithFlags(&c->chain_ev, cudaEventDisableTiming) != cudaSuccess) return fail(FLECHE_ECUDA);
-  // KI: enough warps for the expected unique misses, capped at 4 CTAs (32 warps) per SM
-  c->ki_blocks = (int)std::min<int64_t>((int64_t)c->km_bps * c->sm_count,
-                                         std::max<int64_t>(1, (cfg->max_lookups + 255) / 256));
+  // KM: enough warps for the expected unique misses, km_bps CTAs of 4 warps per SM
+  c->km_blocks = (int)std::min<int64_t>((int64_t)c->km_bps * c->sm_count,
+                                        std::max<int64_t>(1, (cfg->max_lookups + 255) / 256));
+  c->km_smem = bytes ? (size_t)kKmWarps * kKmSmemF4 * sizeof(float4) : 0;
   if (cudaDeviceSynchronize() != cudaSuccess) return fail(FLECHE_ECUDA);
   *out = c;
   return FLECHE_OK;
@@ -355,14 +441,37 @@ fleche_status fleche_query(fleche_ctx* c, const int64_t* const* ids, const int64
   return query_impl(c, ids, lengths, out, (cudaStream_t)stream);
 }
 
+fleche_status fleche_query_pooled(fleche_ctx* c, const int64_t* const* ids, const int64_t* const* offsets,
+                                  const int64_t* bags, const int64_t* nnz, float* out, fleche_stream stream) {
+  if (!c || !ids || !offsets || !bags || !nnz) return FLECHE_EINVAL;
+  if (c->poisoned) return FLECHE_ESTATE;
+  int64_t total_bags = 0;
+  for (int t = 0; t < c->n; ++t) {
+    if (bags[t] < 0 || nnz[t] < 0 || (bags[t] > 0 && !offsets[t])) return FLECHE_EINVAL;
+    total_bags += bags[t];
+  }
+  if (total_bags > 0 && (!out || ((uintptr_t)out & 15u))) return FLECHE_EINVAL;
+  fleche_status st = ensure_device(c);
+  if (st != FLECHE_OK) return st;
+  if (!c->d_pool_stage) FL_CUDA(c, cudaMalloc((void**)&c->d_pool_stage, (size_t)c->max_lookups * c->max_dim * 4));
+  cudaStream_t s = (cudaStream_t)stream;
+  // one-hot lookups of every ID into the staging rows (A1-A8), then bag sums (KP)
+  st = query_impl(c, ids, nnz, c->d_pool_stage, s, 4);
+  if (st != FLECHE_OK) return st;
+  if (c->n <= 32) return launch_pool<32>(c, offsets, bags, nnz, out, s);
+  if (c->n <= 128) return launch_pool<128>(c, offsets, bags, nnz, out, s);
+  return launch_pool<FLECHE_MAX_TABLES>(c, offsets, bags, nnz, out, s);
+}
+
 fleche_status fleche_query_host(fleche_ctx* c, const int64_t* const* ids, const int64_t* lengths, float* out,
                                 fleche_stream stream) {
   if (!c || !ids || !lengths) return FLECHE_EINVAL;
   if (c->poisoned) return FLECHE_ESTATE;
-  int64_t total = 0;
+  int64_t total = 0, out_floats = 0;
   for (int t = 0; t < c->n; ++t) {
     if (lengths[t] < 0 || (lengths[t] > 0 && !ids[t])) return FLECHE_EINVAL;
     total += lengths[t];
+    out_floats += lengths[t] * (int64_t)c->dims[t];
   }
   if (total > c->max_lookups || (total > 0 && !out)) return FLECHE_EINVAL;
   fleche_status st = ensure_device(c);
@@ -370,7 +479,7 @@ fleche_status fleche_query_host(fleche_ctx* c, const int64_t* const* ids, const 
   cudaStream_t s = (cudaStream_t)stream;
   if (!c->d_ids_stage) {
     FL_CUDA(c, cudaMalloc((void**)&c->d_ids_stage, (size_t)c->max_lookups * 8));
-    FL_CUDA(c, cudaMalloc((void**)&c->d_out_stage, (size_t)c->max_lookups * (size_t)c->dim * 4));
+    FL_CUDA(c, cudaMalloc((void**)&c->d_out_stage, (size_t)c->max_lookups * (size_t)c->max_dim * 4));
   }
   st = order_on(c, s);
   if (st != FLECHE_OK) return st;
@@ -392,8 +501,8 @@ fleche_status fleche_query_host(fleche_ctx* c, const int64_t* const* ids, const 
     FL_CUDA(c, cudaMemcpyAsync(c->d_ids_stage, first, (size_t)total * 8, cudaMemcpyHostToDevice, s));
   st = query_impl(c, dids.data(), lengths, c->d_out_stage, s);
   if (st != FLECHE_OK) return st;
-  if (total > 0)
-    FL_CUDA(c, cudaMemcpyAsync(out, c->d_out_stage, (size_t)total * (size_t)c->dim * 4, cudaMemcpyDeviceToHost, s));
+  if (out_floats > 0)
+    FL_CUDA(c, cudaMemcpyAsync(out, c->d_out_stage, (size_t)out_floats * 4, cudaMemcpyDeviceToHost, s));
   return FLECHE_OK;
 }
 
@@ -422,8 +531,8 @@ fleche_status fleche_stats(fleche_ctx* c, fleche_stats_t* out) {
   out->inserted = v[C_INSERTED];
   out->evicted = v[C_EVICTED];
   out->bypassed = v[C_BYPASSED];
-  out->occupancy_bytes = (uint64_t)ctl.occ_rows * 4ull * (uint64_t)c->dim;
-  out->capacity_bytes = (uint64_t)c->dv.rows * 4ull * (uint64_t)c->dim;
+  out->occupancy_bytes = (uint64_t)ctl.occ_bytes;
+  out->capacity_bytes = c->capacity_bytes;
   out->index_bytes = c->index_bytes;
   out->host_bytes_fetched = v[C_HOSTBYTES];
   out->kernels_launched = c->kernels;
@@ -467,8 +576,8 @@ fleche_status fleche_get_encoding(fleche_ctx* c, uint64_t* base, int32_t* fbits,
 fleche_status fleche_get_geometry(fleche_ctx* c, int64_t* sets, int64_t* rows, int32_t* row_floats) {
   if (!c) return FLECHE_EINVAL;
   if (sets) *sets = c->dv.sets;
-  if (rows) *rows = c->dv.rows;
-  if (row_floats) *row_floats = c->dim;
+  if (rows) *rows = c->dv.bytes ? 0 : c->dv.rows;
+  if (row_floats) *row_floats = c->dv.bytes ? -(int32_t)(c->dv.set_units * 8) : c->max_dim;
   return FLECHE_OK;
 }
 
@@ -477,20 +586,29 @@ fleche_status fleche_debug_snapshot(fleche_ctx* c, uint32_t* keys, uint32_t* ts,
   if (!c) return FLECHE_EINVAL;
   if (c->poisoned) return FLECHE_ESTATE;
   const size_t ways = (size_t)c->dv.sets * 32u;
+  const size_t slab_floats = c->dv.bytes ? (size_t)c->dv.sets * c->dv.set_units * 8u : ways * (size_t)c->max_dim;
   if ((keys || ts) && ways_cap < ways) return FLECHE_EINVAL;
-  if (slab && slab_floats_cap < ways * (size_t)c->dim) return FLECHE_EINVAL;
+  if (slab && slab_floats_cap < slab_floats) return FLECHE_EINVAL;
   fleche_status st = ensure_device(c);
   if (st != FLECHE_OK) return st;
   if (c->have_last) FL_CUDA(c, cudaStreamSynchronize(c->last_stream));
   if (keys) FL_CUDA(c, cudaMemcpy(keys, c->dv.keys, ways * 4, cudaMemcpyDeviceToHost));
   if (ts) FL_CUDA(c, cudaMemcpy(ts, c->dv.ts, ways * 4, cudaMemcpyDeviceToHost));
-  if (slab) FL_CUDA(c, cudaMemcpy(slab, c->dv.slab, ways * (size_t)c->dim * 4, cudaMemcpyDeviceToHost));
+  if (slab && slab_floats) FL_CUDA(c, cudaMemcpy(slab, c->dv.slab, slab_floats * 4, cudaMemcpyDeviceToHost));
   return FLECHE_OK;
 }
 
-}  // extern "C"
-
-extern "C" {
+fleche_status fleche_debug_locations(fleche_ctx* c, uint16_t* loc, size_t ways_cap) {
+  if (!c || !loc) return FLECHE_EINVAL;
+  if (c->poisoned) return FLECHE_ESTATE;
+  const size_t ways = (size_t)c->dv.sets * 32u;
+  if (!c->dv.bytes || ways_cap < ways) return FLECHE_EINVAL;
+  fleche_status st = ensure_device(c);
+  if (st != FLECHE_OK) return st;
+  if (c->have_last) FL_CUDA(c, cudaStreamSynchronize(c->last_stream));
+  FL_CUDA(c, cudaMemcpy(loc, c->dv.loc, ways * 2, cudaMemcpyDeviceToHost));
+  return FLECHE_OK;
+}
 
 fleche_status fleche_set_profiling(fleche_ctx* c, int enable) {
   if (!c) return FLECHE_EINVAL;
@@ -502,18 +620,21 @@ fleche_status fleche_kernel_times(fleche_ctx* c, double* kq_ms, double* ki_ms, u
   if (!c) return FLECHE_EINVAL;
   if (c->poisoned) return FLECHE_ESTATE;
   double a = 0, b = 0;
-  for (size_t i = 0; i + 3 <= c->ev_used; i += 3) {
+  size_t i = 0;
+  for (int k : c->ev_kinds) {  // events: [start, after KQ, after KM (, after KP)]
     float x = 0, y = 0;
-    FL_CUDA(c, cudaEventSynchronize(c->ev_pool[i + 2]));
+    FL_CUDA(c, cudaEventSynchronize(c->ev_pool[i + k - 1]));
     FL_CUDA(c, cudaEventElapsedTime(&x, c->ev_pool[i], c->ev_pool[i + 1]));
-    FL_CUDA(c, cudaEventElapsedTime(&y, c->ev_pool[i + 1], c->ev_pool[i + 2]));
+    FL_CUDA(c, cudaEventElapsedTime(&y, c->ev_pool[i + 1], c->ev_pool[i + k - 1]));
     a += x;
     b += y;
+    i += k;
   }
   if (kq_ms) *kq_ms = a;
   if (ki_ms) *ki_ms = b;
-  if (queries) *queries = c->ev_used / 3;
+  if (queries) *queries = c->ev_kinds.size();
   c->ev_used = 0;
+  c->ev_kinds.clear();
   return FLECHE_OK;
 }
 
@@ -539,7 +660,7 @@ fleche_status fleche_probe_host_read(const void* host, uint64_t bytes, int32_t r
     else if (D == 128) probe_host_kernel<128><<<blocks, 128, 0, s>>>((const float*)dev, span, rows, sd, sink);
     else probe_host_kernel<256><<<blocks, 128, 0, s>>>((const float*)dev, span, rows, sd, sink);
   };
-  launch(seed ^ 0x5555);  // warm-up (TLB, clocks)
+  launch(seed ^ 0x5555);  // warm-up (clocks)
   cudaEventRecord(e0, s);
   launch(seed);
   cudaEventRecord(e1, s);

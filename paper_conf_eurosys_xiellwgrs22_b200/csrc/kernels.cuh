@@ -1,28 +1,35 @@
 // kernels.cuh — device side of the B200 flat embedding cache (sm_100a).
 //
-// Two kernels per batch (the paper's "1 -> 2" after decoupling):
+// Two kernels per one-hot batch (the paper's "1 -> 2" after decoupling):
 //
 //   KQ  fused, self-identified query kernel: one lane per
 //       lookup; each warp finds its table from the prefix offsets in shared memory,
 //       re-encodes (table, id) to a flat key, probes its 32-way set with
 //       a warp-cooperative ballot (index of P:L513-528), refreshes the hit way's
 //       timestamp (approximate LRU), claims each unique missed key in an
-//       epoch-tagged scratch table (dedup) and appends it to the miss
-//       list, chains duplicate misses to their key, and copies hit rows from the HBM
-//       slab into `out` with 16-byte vectors.  KQ never touches the host link.
+//       epoch-tagged scratch table (dedup) and appends it to its row
+//       width's miss list, chains duplicate misses to their key, and copies hit rows
+//       from the HBM slab into `out` with 16-byte vectors.  KQ never touches the host.
 //   KM  miss kernel (unified index + replacement, P:L855-860, P:L653-666,
-//       P:L985-988): each warp takes up to 32 unique misses, issues all their
-//       zero-copy host-row loads at once (pinned, mapped host tables), and while those
-//       are in flight picks each miss's victim way (argmin (ts, key) over ways not
-//       touched in this batch: epoch protection) and claims it with a CAS
-//       on the way's timestamp; then writes the row to the owner's `out` position, to
-//       every duplicate position (restore) and to the claimed slab slot,
-//       and publishes the key.  The last CTA advances the device-resident epoch, so a
-//       captured CUDA graph replays correctly.
+//       P:L985-988): each warp takes up to M unique misses of one row width, issues
+//       all their zero-copy host-row loads at once (pinned, mapped host tables) and,
+//       while those are in flight, admits and places each miss: victim =
+//       argmin (ts, key) over ways not touched in this batch (epoch protection,
+//       P:L663-666).  Rows then go to the owner's `out` position, every duplicate
+//       position (restore) and the slab.  The last CTA advances the
+//       device-resident epoch, so a captured CUDA graph replays correctly.
+//   KP  pooling kernel (pooled queries only): bag sums of the staged
+//       one-hot rows, accumulated in fp32 in bag order.
 //
-// The hit copy (KQ, HBM-bound) is decoupled from the miss handling (KM, host-link
-// bound): no lock is held across a copy and miss handling never waits on
-// an index lock.
+// Two index layouts (flat cache, Fig 5c: one pool, slabs per row width):
+//   uniform (all tables share one row width d): way w of set s holds slab row 32s+w;
+//           CAS on the victim's timestamp claims it, no locks.
+//   bytes   (mixed widths): every set owns a set_units x 32 B region of the slab and
+//           at most 32 rows whose sizes sum to <= the region; an insert evicts until
+//           both limits admit the row, places it first-fit (compacting the region when
+//           fragmented) under a per-set lock.  One byte budget is shared by all widths,
+//           so the per-width capacity follows the workload (the flat cache's elastic
+//           rescaling) with no per-class partition to tune.
 #pragma once
 #include <cstdint>
 
@@ -31,6 +38,11 @@ namespace fl {
 constexpr uint32_t kEmpty = 0xFFFFFFFFu;
 constexpr unsigned kFull = 0xFFFFFFFFu;
 constexpr int kStripes = 64;  // stats counters are striped to spread L2 atomics
+constexpr int kMaxCls = 6;    // row widths 8, 16, 32, 64, 128, 256 floats
+constexpr int kDupSlot = 7;   // Ctl::counts column of duplicate misses
+constexpr int kKmWarps = 4;     // KM CTA = 4 warps
+constexpr int kKmStageF4 = 256; // bytes layout, per warp: staged rows of a chunk (<= 4 KB) ...
+constexpr int kKmSmemF4 = 512;  // ... + the compaction buffer of one set region (<= 4 KB)
 
 enum Ctr : int {
   C_HITS = 0,
@@ -51,6 +63,8 @@ struct TableInfo {
   int64_t card;       // c_t
   uint32_t base;      // first flat key of table t (size-aware coding)
   int32_t dim;        // d_t
+  int32_t cls;        // width class (index into the per-call class regions)
+  int32_t pad;
 };
 
 struct MissRec {  // one unique missed key (its owner lookup)
@@ -72,26 +86,30 @@ struct Ctl {
   uint32_t done;   // KM CTA arrival counter
   uint32_t err_invalid;
   uint32_t pad;
-  uint32_t counts[2][4];  // [epoch & 1][0 = unique misses, 1 = duplicate misses]
-  long long occ_rows;     // rows currently cached
+  uint32_t counts[2][8];  // [epoch & 1][class 0..5: unique misses; 7: duplicate misses]
+  long long occ_bytes;    // row bytes currently cached
 };
 
 struct Dev {
-  uint32_t* keys;  // [sets][32] flat keys, kEmpty = free way
-  uint32_t* ts;    // [sets][32] batch epoch of last touch (0 = never)
-  float* slab;     // [sets*32][dim] rows; way w of set s at row s*32 + w
+  uint32_t* keys;   // [sets][32] flat keys, kEmpty = free way
+  uint32_t* ts;     // [sets][32] batch epoch of last touch (0 = never)
+  uint16_t* loc;    // bytes layout: [sets][32] (size units << 8 | offset units), 32 B units
+  uint32_t* lock;   // bytes layout: [sets] insert locks
+  float* slab;      // uniform: [sets*32][dim];  bytes: [sets][set_units * 8]
   unsigned long long* scratch;   // [scr_mask+1] (epoch << 32 | fk) dedup tags
   unsigned long long* dup_head;  // [scr_mask+1] (epoch << 32 | first duplicate + 1)
-  MissRec* miss;                 // [max_lookups]
+  MissRec* miss;                 // [max_lookups], split into per-class regions per call
   DupRec* dup;                   // [max_lookups]
   Ctl* ctl;
   unsigned long long* stats;  // [kStripes][kNumCtr]
   const TableInfo* tables;    // [n]
   uint32_t sets, rows, scr_mask, hash_seed;
-  int32_t dim, admit_all;
+  int32_t dim, admit_all;     // dim: row width of the uniform layout
   uint64_t admit_thr, admit_seed;
   int32_t prefetch;  // KQ starts each unique miss's host-row transfer into L2
   int32_t km_m;      // unique misses per KM warp iteration (4, 8, 16, 32)
+  int32_t bytes;     // 0 = uniform layout, 1 = bytes layout
+  uint32_t set_units;  // bytes layout: region of a set in 32 B units (<= 256)
 #ifdef FLECHE_EXPERIMENTS
   int32_t exp_mode;  // timing experiments only (libfleche_exp.so); breaks semantics
   int32_t exp_pad;
@@ -103,8 +121,30 @@ struct QArgs {
   const int64_t* ids[MAXT];  // per-table device ID arrays
   int64_t scan[MAXT + 1];    // exclusive prefix of lengths
   int64_t out_off[MAXT];     // float offset of O_t in out
+  int64_t cls_off[8];        // start of each class's region of the miss list
   float* out;
   int32_t n;
+  int32_t pad;
+};
+
+struct KMArgs {
+  float* out;
+  int64_t cls_off[8];
+  int32_t cls_dim[8];
+  int32_t ncls;
+  int32_t pad;
+};
+
+template <int MAXT>
+struct PArgs {                  // pooling: column slots of table t = bags_t * d_t / 4
+  const int64_t* offs[MAXT];    // CSR bag offsets of table t (device), bags_t + 1 entries
+  int64_t cscan[MAXT + 1];      // exclusive prefix of column slots
+  int64_t stage_off[MAXT];      // float offset of table t's staged rows
+  int64_t out_off[MAXT];        // float offset of table t's pooled rows in out
+  const float* stage;
+  float* out;
+  int32_t n;
+  int32_t pad;
 };
 
 __device__ __forceinline__ uint32_t fmix32(uint32_t h) {
@@ -135,6 +175,11 @@ __device__ __forceinline__ float4 ld_nc_v4(const float* p) {
   asm volatile("ld.global.nc.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p));
   return v;
 }
+__device__ __forceinline__ float4 ld_cg_v4(const float* p) {
+  float4 v;
+  asm volatile("ld.global.cg.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p) : "memory");
+  return v;
+}
 __device__ __forceinline__ uint32_t ld_nc_u32(const uint32_t* p) {
   uint32_t v;
   asm volatile("ld.global.nc.u32 %0, [%1];" : "=r"(v) : "l"(p));
@@ -143,6 +188,11 @@ __device__ __forceinline__ uint32_t ld_nc_u32(const uint32_t* p) {
 __device__ __forceinline__ uint32_t ld_cg_u32(const uint32_t* p) {
   uint32_t v;
   asm volatile("ld.global.cg.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ uint32_t ld_cg_u16(const uint16_t* p) {
+  unsigned short v;
+  asm volatile("ld.global.cg.u16 %0, [%1];" : "=h"(v) : "l"(p) : "memory");
   return v;
 }
 __device__ __forceinline__ uint4 ld_cg_v4u(const uint32_t* p) {
@@ -157,6 +207,14 @@ __device__ __forceinline__ unsigned long long ld_cg_u64(const unsigned long long
 }
 __device__ __forceinline__ void st_v4(float* p, float4 v) {
   asm volatile("st.global.v4.f32 [%0], {%1,%2,%3,%4};" ::"l"(p), "f"(v.x), "f"(v.y), "f"(v.z), "f"(v.w) : "memory");
+}
+__device__ __forceinline__ unsigned long long warp_min_u64(unsigned long long x) {
+#pragma unroll
+  for (int o = 16; o; o >>= 1) {
+    const unsigned long long y = __shfl_xor_sync(kFull, x, o);
+    x = y < x ? y : x;
+  }
+  return x;
 }
 
 // Copy the 32 rows named by the warp's lanes (src may be null = zero row; dst null =
@@ -194,8 +252,7 @@ __device__ __forceinline__ void gather_rows(const float* src, float* dst, int la
   }
 }
 
-// Fallback for warps whose lanes have different row widths or widths that are not a
-// power of two: one row at a time, whole warp.
+// Fallback for warps whose lanes have different row widths: one row at a time.
 __device__ __forceinline__ void gather_rows_any(const float* src, float* dst, int d, int lane) {
 #pragma unroll 1
   for (int r = 0; r < 32; ++r) {
@@ -239,6 +296,18 @@ struct RowBuf {
       if (o && r < M) {
 #pragma unroll
         for (int k = 0; k < VPL; ++k) st_v4(o + 4 * (sub + k * LPR), v[p][k]);
+      }
+    }
+  }
+  // row r -> smem[r * VEC ...]
+  __device__ __forceinline__ void to_smem(float4* sm, int lane) const {
+    const int sub = lane % LPR, rs = lane / LPR;
+#pragma unroll
+    for (int p = 0; p < PASSES; ++p) {
+      const int r = p * RPP + rs;
+      if (r < M) {
+#pragma unroll
+        for (int k = 0; k < VPL; ++k) sm[r * VEC + sub + k * LPR] = v[p][k];
       }
     }
   }
@@ -300,7 +369,15 @@ __global__ void __launch_bounds__(128) kq_kernel(const __grid_constant__ QArgs<M
     const int64_t off = active ? qa.out_off[t] + j * (int64_t)d : 0;
 
     // A4 hit gather from the HBM slab (zero row for an invalid ID); misses are KM's
-    const float* src = hit ? dv.slab + (size_t)slot * (size_t)d : nullptr;
+    const float* src = nullptr;
+    if (hit) {
+      if (!dv.bytes) {
+        src = dv.slab + (size_t)slot * (size_t)d;
+      } else {
+        const uint32_t l = ld_nc_u32((const uint32_t*)(dv.loc + (slot & ~1u))) >> ((slot & 1u) * 16);
+        src = dv.slab + ((size_t)s * dv.set_units + (l & 0xFFu)) * 8u;
+      }
+    }
     float* dst = (active && !miss) ? qa.out + off : nullptr;
     const int d0 = __shfl_sync(kFull, d, 0);
     const bool uni = __all_sync(kFull, !active || d == d0);
@@ -344,14 +421,16 @@ __global__ void __launch_bounds__(128) kq_kernel(const __grid_constant__ QArgs<M
     const unsigned own_m = __ballot_sync(kFull, kind == 1);
     const unsigned dup_m = __ballot_sync(kFull, kind == 2);
     const unsigned lt = (1u << lane) - 1u;
-    if (own_m) {
+    if (own_m) {  // append to this width's region of the miss list, aggregated per class
+      const int cls = ti->cls;
+      const unsigned grp = __match_any_sync(kFull, kind == 1 ? cls : 64 + lane);
+      const int leader = __ffs(grp) - 1;
       uint32_t b = 0;
-      if (lane == __ffs(own_m) - 1) b = atomicAdd(&dv.ctl->counts[par][0], (uint32_t)__popc(own_m));
-      b = __shfl_sync(kFull, b, __ffs(own_m) - 1);
+      if (kind == 1 && lane == leader) b = atomicAdd(&dv.ctl->counts[par][cls], (uint32_t)__popc(grp));
+      b = __shfl_sync(kFull, b, leader);
       if (kind == 1) {
-        dv.miss[b + __popc(own_m & lt)] = MissRec{off, fk, scr, t, 0};
-        // start the host-link transfer now: KM's loads of this row then hit L2
-        if (dv.prefetch) {
+        dv.miss[qa.cls_off[cls] + b + __popc(grp & lt)] = MissRec{off, fk, scr, t, 0};
+        if (dv.prefetch) {  // experimental: start the host-link transfer now
           const float* hrow = ti->host + (size_t)id * (size_t)d;
           asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(hrow), "r"(4u * (unsigned)d) : "memory");
         }
@@ -359,7 +438,7 @@ __global__ void __launch_bounds__(128) kq_kernel(const __grid_constant__ QArgs<M
     }
     if (dup_m) {
       uint32_t b = 0;
-      if (lane == __ffs(dup_m) - 1) b = atomicAdd(&dv.ctl->counts[par][1], (uint32_t)__popc(dup_m));
+      if (lane == __ffs(dup_m) - 1) b = atomicAdd(&dv.ctl->counts[par][kDupSlot], (uint32_t)__popc(dup_m));
       b = __shfl_sync(kFull, b, __ffs(dup_m) - 1);
       if (kind == 2) {  // push onto the key's duplicate chain (epoch-tagged head)
         const uint32_t idx = b + __popc(dup_m & lt);
@@ -395,10 +474,10 @@ __global__ void __launch_bounds__(128) kq_kernel(const __grid_constant__ QArgs<M
     atomicAdd(dv.stats + (blockIdx.x % kStripes) * kNumCtr + threadIdx.x, s_ctr[threadIdx.x]);
 }
 
-// Victim way for flat key fk in its set: argmin (ts, key) over ways with ts < epoch,
-// claimed by CAS(ts: old -> epoch).  Returns the slot, or -1 if every way of the set
-// was read or written in this batch (epoch protection: bypass).  *old_key = the
-// evicted key (kEmpty if the way was free).  One lane, 16 vector loads, no warp sync.
+// Uniform layout: victim way for fk in its set = argmin (ts, key) over ways with
+// ts < epoch, claimed by CAS(ts: old -> epoch).  Returns the slot, or -1 if every way
+// of the set was read or written in this batch (epoch protection: bypass).  One lane,
+// 16 vector loads, no warp synchronisation.
 __device__ __forceinline__ int64_t claim_victim(const Dev& dv, uint32_t fk, uint32_t epoch, uint32_t* old_key) {
   const uint32_t s = set_of(dv, fk);
   const int nways = ways_in(dv, s);
@@ -427,18 +506,116 @@ __device__ __forceinline__ int64_t claim_victim(const Dev& dv, uint32_t fk, uint
   }
 }
 
-// KM for row width D: each warp iteration handles M unique misses.
-template <int D, int M>
-__device__ __forceinline__ void km_rows(const Dev& dv, float* __restrict__ out, uint32_t epoch, uint32_t nmiss,
-                                        int lane, uint32_t gw, uint32_t nw, unsigned& ins, unsigned& ev,
-                                        unsigned& byp, unsigned long long& hostb) {
+// Bytes layout: warp-cooperative insert of one row (units x 32 B, staged in smem)
+// into fk's set under the set's lock.  Evicts argmin (ts, key) among rows not touched
+// in this batch until a way is free and the row fits the set's byte budget; places it
+// first-fit, compacting the set's region through `cbuf` (set_units * 2 float4 of
+// smem) when free space is fragmented.  Returns false (bypass) if no candidate is
+// left; evictions already made stay made (as in the oracle's MODE_SETBYTES).
+__device__ bool bytes_insert(const Dev& dv, uint32_t fk, int units, const float4* row, uint32_t epoch, int lane,
+                             unsigned& ev, long long& docc, float4* cbuf) {
+  const uint32_t s = set_of(dv, fk);
+  const int SU = (int)dv.set_units;
+  uint32_t* lk = dv.lock + s;
+  if (lane == 0) {
+    while (atomicCAS(lk, 0u, 1u) != 0u) __nanosleep(32);
+  }
+  __syncwarp();
+  __threadfence();
+  uint32_t* kp = dv.keys + (size_t)s * 32u + lane;
+  uint32_t* tp = dv.ts + (size_t)s * 32u + lane;
+  uint16_t* lp = dv.loc + (size_t)s * 32u + lane;
+  uint32_t k = ld_cg_u32(kp);
+  const uint32_t t = ld_cg_u32(tp);
+  uint32_t l = ld_cg_u16(lp);
+  bool live = k != kEmpty;
+  int my_sz = live ? (int)(l >> 8) : 0;
+  int used = __reduce_add_sync(kFull, (unsigned)my_sz);
+  bool ok = true;
+  while (true) {
+    const int nlive = __popc(__ballot_sync(kFull, live));
+    if (nlive < 32 && used + units <= SU) break;
+    const unsigned long long rank = (live && t < epoch) ? (((unsigned long long)t << 32) | k) : ~0ull;
+    const unsigned long long best = warp_min_u64(rank);
+    if (best == ~0ull) { ok = false; break; }
+    const int v = __ffs(__ballot_sync(kFull, rank == best)) - 1;
+    const int vsz = __shfl_sync(kFull, my_sz, v);
+    used -= vsz;
+    if (lane == 0) { ++ev; docc -= 32ll * vsz; }
+    if (lane == v) { live = false; my_sz = 0; k = kEmpty; *kp = kEmpty; }
+  }
+  if (ok) {
+    // occupancy bitmap of the region (SU <= 256 units -> 8 words)
+    const int my_off = (int)(l & 0xFFu);
+    uint32_t words[8];
+#pragma unroll
+    for (int w = 0; w < 8; ++w) {
+      uint32_t mine = 0;
+      if (live) {
+        const int lo = max(my_off, 32 * w), hi = min(my_off + my_sz, 32 * w + 32);
+        if (hi > lo) mine = (hi - lo == 32) ? kFull : (((1u << (hi - lo)) - 1u) << (lo - 32 * w));
+      }
+      words[w] = __reduce_or_sync(kFull, mine);
+    }
+    int start = -1;
+    for (int base = 0; base < SU && start < 0; base += 32) {
+      const int p = base + lane;
+      bool fits = p + units <= SU;
+      for (int u = 0; u < units && fits; ++u) fits = !((words[(p + u) >> 5] >> ((p + u) & 31)) & 1u);
+      const unsigned b = __ballot_sync(kFull, fits);
+      if (b) start = base + __ffs(b) - 1;
+    }
+    if (start < 0) {  // fragmented: pack the live rows to the front through smem
+      float* region = dv.slab + (size_t)s * SU * 8u;
+      for (int c = lane; c < SU * 2; c += 32) cbuf[c] = ld_cg_v4(region + 4 * c);
+      __syncwarp();
+      int incl = my_sz;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const int y = __shfl_up_sync(kFull, incl, o);
+        if (lane >= o) incl += y;
+      }
+      const int new_off = incl - my_sz;
+      for (int w = 0; w < 32; ++w) {
+        const int wsz = __shfl_sync(kFull, my_sz, w);
+        if (!wsz) continue;
+        const int wo = __shfl_sync(kFull, my_off, w), wn = __shfl_sync(kFull, new_off, w);
+        for (int c = lane; c < wsz * 2; c += 32) st_v4(region + (size_t)(wn * 2 + c) * 4, cbuf[wo * 2 + c]);
+      }
+      if (live) *lp = (uint16_t)((my_sz << 8) | new_off);
+      start = used;
+      __syncwarp();
+    }
+    float* dst = dv.slab + ((size_t)s * SU + start) * 8u;
+    for (int c = lane; c < units * 2; c += 32) st_v4(dst + 4 * c, row[c]);
+    const int fw = __ffs(~__ballot_sync(kFull, live)) - 1;
+    if (lane == fw) {
+      *kp = fk;
+      *tp = epoch;
+      *lp = (uint16_t)((units << 8) | start);
+    }
+    if (lane == 0) docc += 32ll * units;
+  }
+  __syncwarp();
+  __threadfence();
+  if (lane == 0) atomicExch(lk, 0u);
+  __syncwarp();
+  return ok;
+}
+
+// KM for row width D: each warp iteration handles M unique misses of this class.
+template <bool BYTES, int D, int M>
+__device__ __forceinline__ void km_rows(const Dev& dv, float* __restrict__ out, const MissRec* __restrict__ mlist,
+                                        uint32_t epoch, uint32_t nmiss, int lane, uint32_t gw, uint32_t nw,
+                                        unsigned& ins, unsigned& ev, unsigned& byp, long long& docc,
+                                        unsigned long long& hostb, float4* wsm) {
   for (uint32_t base = gw * M; base < nmiss; base += nw * M) {
     const uint32_t k = base + lane;
     bool has = lane < M && k < nmiss;
     MissRec m{};
     const float* src = nullptr;
     if (has) {
-      m = dv.miss[k];
+      m = mlist[k];
       const TableInfo* ti = dv.tables + m.t;
       src = ti->host + (size_t)(m.fk - ti->base) * D;  // unified index: computed host address
     }
@@ -449,30 +626,48 @@ __device__ __forceinline__ void km_rows(const Dev& dv, float* __restrict__ out, 
     // A6: all of this warp's host-row loads go out now (zero-copy over the host link)
     RowBuf<D, M> rb;
     rb.load(src, lane);
-    // A7 while they are in flight: admission + victim claim (L2 round trips only)
-    float* slab_dst = nullptr;
-    uint32_t fkey = kEmpty;
+    bool admit = false;
     if (has) {
-      bool admit = true;
-      if (!dv.admit_all)
-        admit = splitmix64(dv.admit_seed ^ (uint64_t)m.fk ^ ((uint64_t)(epoch - 1u) << 32)) < dv.admit_thr;
-      int64_t slot = -1;
-      uint32_t old_key = kEmpty;
-      if (admit) slot = claim_victim(dv, m.fk, epoch, &old_key);
-      if (slot >= 0) {
-        ++ins;
-        if (old_key != kEmpty) ++ev;
-        slab_dst = dv.slab + (size_t)slot * D;
-        fkey = (uint32_t)slot;
-      } else {
-        ++byp;
-      }
+      admit = dv.admit_all ||
+              splitmix64(dv.admit_seed ^ (uint64_t)m.fk ^ ((uint64_t)(epoch - 1u) << 32)) < dv.admit_thr;
       hostb += 4ull * D;
     }
-    // rows land: owner position, slab slot, then the key is published
-    rb.store(has ? out + m.off : nullptr, lane);
-    rb.store(slab_dst, lane);
-    if (slab_dst) dv.keys[fkey] = m.fk;
+    if constexpr (!BYTES) {
+      // A7 while the loads are in flight: victim claim (L2 round trips only)
+      float* slab_dst = nullptr;
+      uint32_t slot32 = 0;
+      if (has) {
+        int64_t slot = -1;
+        uint32_t old_key = kEmpty;
+        if (admit) slot = claim_victim(dv, m.fk, epoch, &old_key);
+        if (slot >= 0) {
+          ++ins;
+          docc += 4ll * D;
+          if (old_key != kEmpty) { ++ev; docc -= 4ll * D; }
+          slab_dst = dv.slab + (size_t)slot * D;
+          slot32 = (uint32_t)slot;
+        } else {
+          ++byp;
+        }
+      }
+      rb.store(has ? out + m.off : nullptr, lane);
+      rb.store(slab_dst, lane);
+      if (slab_dst) dv.keys[slot32] = m.fk;
+    } else {
+      rb.store(has ? out + m.off : nullptr, lane);
+      rb.to_smem(wsm, lane);
+      __syncwarp();
+      for (int r = 0; r < M; ++r) {  // inserts of this chunk, one set lock at a time
+        if (!__shfl_sync(kFull, (int)has, r)) continue;
+        const uint32_t fk = __shfl_sync(kFull, m.fk, r);
+        if (!__shfl_sync(kFull, (int)admit, r)) {
+          if (lane == 0) ++byp;
+          continue;
+        }
+        const bool ok = bytes_insert(dv, fk, D / 8, wsm + r * (D / 4), epoch, lane, ev, docc, wsm + kKmStageF4);
+        if (lane == 0) { if (ok) ++ins; else ++byp; }
+      }
+    }
     // A8 restore: walk each miss's duplicate chain
     uint32_t p = 0;
     if (has) {
@@ -488,24 +683,33 @@ __device__ __forceinline__ void km_rows(const Dev& dv, float* __restrict__ out, 
       }
       rb.store(o, lane);
     }
+    __syncwarp();
   }
 }
 
-__global__ void __launch_bounds__(128) km_kernel(const __grid_constant__ Dev dv, float* __restrict__ out) {
+
+template <bool BYTES>
+__global__ void __launch_bounds__(128, 4) km_kernel(const __grid_constant__ Dev dv, const __grid_constant__ KMArgs ka) {
   __shared__ unsigned long long s_ctr[kNumCtr];
+  extern __shared__ float4 s_dyn[];
   if (threadIdx.x < kNumCtr) s_ctr[threadIdx.x] = 0;
   __syncthreads();
   const uint32_t epoch = *(volatile uint32_t*)&dv.ctl->epoch;
   const int par = epoch & 1u;
-  const uint32_t nmiss = *(volatile uint32_t*)&dv.ctl->counts[par][0];
   const int lane = threadIdx.x & 31;
   // block-interleaved warp numbering: consecutive miss chunks land on different SMs,
   // so the host-link loads of a batch are spread over the whole GPU
   const uint32_t gw = (threadIdx.x >> 5) * gridDim.x + blockIdx.x;
   const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
+  float4* wsm = BYTES ? s_dyn + (threadIdx.x >> 5) * kKmSmemF4 : nullptr;
   unsigned ins = 0, ev = 0, byp = 0;
+  long long docc = 0;
   unsigned long long hostb = 0;
-#define FL_KM(D, M) km_rows<D, M>(dv, out, epoch, nmiss, lane, gw, nw, ins, ev, byp, hostb)
+  for (int c = 0; c < ka.ncls; ++c) {
+    const uint32_t nmiss = *(volatile uint32_t*)&dv.ctl->counts[par][c];
+    if (!nmiss) continue;
+    const MissRec* ml = dv.miss + ka.cls_off[c];
+#define FL_KM(D, M) km_rows<BYTES, D, M>(dv, ka.out, ml, epoch, nmiss, lane, gw, nw, ins, ev, byp, docc, hostb, wsm)
 #define FL_KM_MS(D)                    \
   switch (dv.km_m) {                   \
     case 4: FL_KM(D, 4); break;        \
@@ -513,43 +717,80 @@ __global__ void __launch_bounds__(128) km_kernel(const __grid_constant__ Dev dv,
     case 32: FL_KM(D, 32); break;      \
     default: FL_KM(D, 8); break;       \
   }
-  switch (dv.dim) {  // fleche_create only admits these widths
-    case 8: FL_KM_MS(8); break;
-    case 16: FL_KM_MS(16); break;
-    case 32: FL_KM_MS(32); break;
-    case 64: FL_KM_MS(64); break;
-    case 128: if (dv.km_m <= 4) FL_KM(128, 4); else FL_KM(128, 8); break;
-    case 256: FL_KM(256, 4); break;
-    default: break;
-  }
+    switch (ka.cls_dim[c]) {  // fleche_create only admits these widths
+      case 8: FL_KM_MS(8); break;
+      case 16: FL_KM_MS(16); break;
+      case 32: FL_KM_MS(32); break;
+      case 64: FL_KM_MS(64); break;
+      case 128: if (dv.km_m <= 4) FL_KM(128, 4); else FL_KM(128, 8); break;
+      case 256: FL_KM(256, 4); break;
+      default: break;
+    }
 #undef FL_KM_MS
 #undef FL_KM
+  }
   ins = __reduce_add_sync(kFull, ins);
   ev = __reduce_add_sync(kFull, ev);
   byp = __reduce_add_sync(kFull, byp);
-  for (int o = 16; o; o >>= 1) hostb += __shfl_xor_sync(kFull, hostb, o);
+#pragma unroll
+  for (int o = 16; o; o >>= 1) {
+    hostb += __shfl_xor_sync(kFull, hostb, o);
+    docc += __shfl_xor_sync(kFull, docc, o);
+  }
   if (lane == 0) {
     if (ins) atomicAdd(&s_ctr[C_INSERTED], (unsigned long long)ins);
     if (ev) atomicAdd(&s_ctr[C_EVICTED], (unsigned long long)ev);
     if (byp) atomicAdd(&s_ctr[C_BYPASSED], (unsigned long long)byp);
     if (hostb) atomicAdd(&s_ctr[C_HOSTBYTES], hostb);
+    if (docc) atomicAdd((unsigned long long*)&dv.ctl->occ_bytes, (unsigned long long)docc);
   }
   __syncthreads();
   if (threadIdx.x < kNumCtr && s_ctr[threadIdx.x])
     atomicAdd(dv.stats + (blockIdx.x % kStripes) * kNumCtr + threadIdx.x, s_ctr[threadIdx.x]);
   if (threadIdx.x == 0) {
-    const long long docc = (long long)s_ctr[C_INSERTED] - (long long)s_ctr[C_EVICTED];
-    if (docc) atomicAdd((unsigned long long*)&dv.ctl->occ_rows, (unsigned long long)docc);
     __threadfence();
     const uint32_t prev = atomicAdd(&dv.ctl->done, 1u);
     if (prev == gridDim.x - 1) {  // last CTA: reset next batch's counters, advance the epoch
-      dv.ctl->counts[par ^ 1][0] = 0;
-      dv.ctl->counts[par ^ 1][1] = 0;
+#pragma unroll
+      for (int c = 0; c < 8; ++c) dv.ctl->counts[par ^ 1][c] = 0;
       dv.ctl->done = 0;
       __threadfence();
       *(volatile uint32_t*)&dv.ctl->epoch = epoch + 1u;
     }
   }
+}
+
+// Pooling: one thread per (bag, 4-float column); sums the bag's staged
+// rows sequentially in bag order in fp32 (the oracle's order, so results are
+// bit-identical for any values).  An empty bag gives a zero row.
+template <int MAXT>
+__global__ void __launch_bounds__(256) kp_kernel(const __grid_constant__ PArgs<MAXT> pa, const TableInfo* __restrict__ tables) {
+  __shared__ int64_t s_scan[MAXT + 1];
+  for (int i = threadIdx.x; i <= pa.n; i += blockDim.x) s_scan[i] = pa.cscan[i];
+  __syncthreads();
+  const int64_t g = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (g >= s_scan[pa.n]) return;
+  int lo = 0, hi = pa.n;
+  while (hi - lo > 1) {
+    const int mid = (lo + hi) >> 1;
+    if (s_scan[mid] <= g) lo = mid; else hi = mid;
+  }
+  const int t = lo;
+  const int vec = tables[t].dim / 4;
+  const int64_t local = g - s_scan[t];
+  const int64_t bag = local / vec;
+  const int c = (int)(local % vec);
+  const int64_t k0 = pa.offs[t][bag], k1 = pa.offs[t][bag + 1];
+  const float* st = pa.stage + pa.stage_off[t] + 4 * c;
+  float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+  for (int64_t k = k0; k < k1; ++k) {
+    const float4 x = *reinterpret_cast<const float4*>(st + k * 4 * vec);
+    acc.x = __fadd_rn(acc.x, x.x);
+    acc.y = __fadd_rn(acc.y, x.y);
+    acc.z = __fadd_rn(acc.z, x.z);
+    acc.w = __fadd_rn(acc.w, x.w);
+  }
+  *reinterpret_cast<float4*>(pa.out + pa.out_off[t] + bag * 4 * vec + 4 * c) = acc;
 }
 
 // Host-link probe: the miss-fetch access pattern (one row per lane, 16-byte vector
