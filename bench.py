@@ -29,7 +29,7 @@ import numpy as np  # noqa: E402
 
 from workload import configs  # noqa: E402
 
-PREFILL = {"cfg0": 20, "cfg1": 150, "cfg2": 300, "cfg5": 60}
+PREFILL = {"cfg0": 20, "cfg1": 150, "cfg2": 300, "cfg4": 30, "cfg5": 60}  # >= 2x the Che fill time
 HASH_SEED = 0x9E3779B9
 
 
@@ -119,26 +119,31 @@ class ClockSampler:
                 "reasons": sorted(seen), "samples": len(sel)}
 
 
-def algorithmic_bytes(st: dict, n_queries: int, d: int) -> dict:
-    """Per-launch algorithmic bytes of KQ and KI."""
+def algorithmic_bytes(st: dict, n_queries: int, row: float, row_miss: float, pooled_out: float = 0) -> dict:
+    """Per-launch algorithmic bytes of KQ and KM.
+
+    row: lookup-weighted mean row bytes; row_miss: mean row bytes of unique misses
+    (= host bytes / unique misses, from the run's own counters); pooled_out: bytes of
+    pooled output rows per batch (0 for one-hot)."""
     q = max(n_queries, 1)
     N = st["lookups"] / q
     U = st["unique_keys"] / q
     Uh = st["unique_hits"] / q
     Um = st["unique_misses"] / q
     Ui = st["inserted"] / q
-    Nd = (st["misses"] - st["unique_misses"]) / q  # duplicate misses (restored in KI)
+    Nd = (st["misses"] - st["unique_misses"]) / q  # duplicate misses (restored in KM)
     Nm = st["misses"] / q  # missed lookups (owners + duplicates)
-    row = 4 * d
     # KQ: IDs in, one 128 B set line per unique key, hit rows read + ts sector touched,
     #     out rows written for every non-missed lookup, 8 B dedup tag + 24 B record per unique miss
     kq_hbm = N * 8 + U * 128 + Uh * (row + 32) + (N - Nm) * row + Um * (8 + 24) + Nd * 24
     # KM: miss record in, host row in (host link), owner + duplicate out rows written,
     #     per insert: the set's key+ts lines (256 B) read, the row and key/ts written
-    km_host = Um * row
-    km_hbm = Um * 24 + Nd * 16 + (Um + Nd) * row + Ui * (256 + row + 8)
+    km_host = Um * row_miss
+    km_hbm = Um * 24 + Nd * 16 + (Um * row_miss + Nd * row) + Ui * (256 + row_miss + 8)
+    # KP (pooled only): staged rows read once, pooled rows written
+    kp_hbm = (N * row + pooled_out) if pooled_out else 0
     return {"N": N, "U": U, "U_hit": Uh, "U_miss": Um, "U_ins": Ui, "kq_hbm": kq_hbm, "km_host": km_host,
-            "km_hbm": km_hbm}
+            "km_hbm": km_hbm + kp_hbm, "kp_hbm": kp_hbm}
 
 
 def run_reference(args, w, P, W, K):
@@ -221,8 +226,10 @@ def main():
         import torch.distributed as dist
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     dev = torch.device("cuda", local)
-    N = w.batch_size * w.n
+    b0 = w.batch(0, rank=rank)
+    N = int(b0.lookups * (1.25 if w.pooled else 1))  # max_lookups (bag lengths vary per batch)
     d = w.dims[0]
+    uniform = len(set(w.dims)) == 1
 
     # host tier: every table in one buffer, page-locked + mapped by fleche_create
     log("host tier")
@@ -234,35 +241,64 @@ def main():
     stream = torch.cuda.current_stream()
 
     def gen_batch(b):
-        return np.concatenate(w.batch(b, rank=rank).ids)
+        return w.batch(b, rank=rank)
 
-    lens = [w.batch_size] * w.n
+    class DevBatch:
+        """One batch resident in HBM: flat IDs (+ flat CSR offsets when pooled)."""
 
-    def views(t):
-        return [t[i * w.batch_size:(i + 1) * w.batch_size] for i in range(w.n)]
+        def __init__(self, bt):
+            self.lens = [int(x.size) for x in bt.ids]
+            self.ids = torch.from_numpy(np.concatenate(bt.ids)).to(dev)
+            self.idv, o = [], 0
+            for L in self.lens:
+                self.idv.append(self.ids[o:o + L])
+                o += L
+            self.bags = None
+            if bt.offsets is not None:
+                self.bags = [int(x.size) - 1 for x in bt.offsets]
+                self.offs = torch.from_numpy(np.concatenate(bt.offsets)).to(dev)
+                self.offv, o = [], 0
+                for x in bt.offsets:
+                    self.offv.append(self.offs[o:o + x.size])
+                    o += x.size
+
+        def out_floats(self):
+            return cache.pooled_floats(self.bags) if self.bags is not None else cache.out_floats(self.lens)
+
+        def run(self, out):
+            if self.bags is not None:
+                cache.query_pooled(self.idv, self.offv, out, bags=self.bags, nnz=self.lens)
+            else:
+                cache.query(self.idv, out, lengths=self.lens)
+
+    out_max = int(DevBatch(b0).out_floats() * 1.25)
+    outs = [torch.empty(out_max, dtype=torch.float32, device=dev) for _ in range(4)]  # 4 x out > L2 when large
 
     # steady state: untimed prefill batches
-    stage = torch.empty(N, dtype=torch.int64, device=dev)
-    outs = [torch.empty(N * d, dtype=torch.float32, device=dev) for _ in range(4)]  # 4 x out > L2 when N*d*4 large
     log("prefill")
     for b in range(P):
-        stage.copy_(torch.from_numpy(gen_batch(b)))
-        cache.query(views(stage), outs[b % 4])
+        DevBatch(gen_batch(b)).run(outs[b % 4])
+        if b % 16 == 15:
+            torch.cuda.synchronize()
     torch.cuda.synchronize()
 
-    # pre-generated device-resident batches for warm-up, timed and profiled passes
+    # pre-generated device-resident batches for warm-up, timed and profiled passes (at most
+    # ~8 GB of them; beyond that the timed steps cycle through the pre-generated batches)
     log("pregen")
     KP = min(K, 300)
-    ids_dev = torch.empty((W + K + KP, N), dtype=torch.int64, device=dev)
-    for i in range(W + K + KP):
-        ids_dev[i].copy_(torch.from_numpy(gen_batch(P + i)))
+    per_step = b0.lookups * 8 * (1.1 if w.pooled else 1.0)
+    R = int(min(W + K + KP, max(8, 8e9 // per_step)))
+    pre = [DevBatch(gen_batch(P + i)) for i in range(R)]
     torch.cuda.synchronize()
+
+    def step(i, out):
+        pre[i % R].run(out)
 
     log("timed")
     clock = ClockSampler(local)
     clock.start()
     for i in range(W):
-        cache.query(views(ids_dev[i]), outs[i % 4])
+        step(i, outs[i % 4])
     torch.cuda.synchronize()
     if dist:
         dist.barrier()
@@ -272,7 +308,7 @@ def main():
     tw0 = time.perf_counter()
     e0.record(stream)
     for k in range(K):
-        cache.query(views(ids_dev[W + k]), outs[k % 4])
+        step(W + k, outs[k % 4])
     e1.record(stream)
     torch.cuda.synchronize()
     tw1 = time.perf_counter()
@@ -298,14 +334,18 @@ def main():
     cache.set_profiling(True)
     sp0 = cache.stats()
     for k in range(KP):
-        cache.query(views(ids_dev[W + K + k]), outs[k % 4])
+        step(W + K + k, outs[k % 4])
     torch.cuda.synchronize()
     kq_ms, ki_ms, nq = cache.kernel_times()
     sp1 = cache.stats()
     cache.set_profiling(False)
     dsp = {k: sp1[k] - sp0[k] for k in fl.STAT_FIELDS}
     kq_avg, ki_avg = kq_ms / nq, ki_ms / nq
-    ab = algorithmic_bytes(dsp, nq, d)
+    # lookup-weighted and miss-weighted mean row bytes (uniform configs: both 4d)
+    row_lk = sum(L * 4 * dd for L, dd in zip(pre[0].lens, w.dims)) / max(1, sum(pre[0].lens))
+    row_ms = dsp["host_bytes_fetched"] / max(1, dsp["unique_misses"])
+    ab = algorithmic_bytes(dsp, nq, row_lk, row_ms, pooled_out=(
+        sum(b * 4 * dd for b, dd in zip(pre[0].bags, w.dims)) if w.pooled else 0))
 
     # host-link peaks, both measured in-run with KM's access pattern (16 B vector loads,
     # one row per lane) over rows of 4d bytes: (a) uniformly random rows over the WHOLE host
@@ -314,15 +354,19 @@ def main():
     # (b) random rows inside a 1 GiB window = the link's bandwidth
     log("host probe")
     hp = int(hostbuf.ctypes.data)
-    host_rand = fl.binding.probe_host_read(hp, int(hostbuf.nbytes), 4 * d, 1 << 21, 7)
-    host_link = fl.binding.probe_host_read(hp, min(1 << 30, int(hostbuf.nbytes)), 4 * d, 1 << 21, 9)
+    prow = min((128, 256, 512, 1024), key=lambda r: abs(r - row_ms))
+    host_rand = fl.binding.probe_host_read(hp, int(hostbuf.nbytes), prow, 1 << 21, 7)
+    host_link = fl.binding.probe_host_read(hp, min(1 << 30, int(hostbuf.nbytes)), prow, 1 << 21, 9)
+    if prow != round(row_ms):  # mixed widths: the large-span ceiling is a row rate; scale to the mean miss row
+        host_rand *= row_ms / prow
+        host_link *= row_ms / prow
     hbm_peak = float(peaks().get("hbm_gbs", 6650.0))
     kern = {
         "kq_kernel": {"ms": kq_avg, "bound": "hbm", "bytes": ab["kq_hbm"], "peak": hbm_peak,
                       "peak_source": "MEASURED_PEAKS.json hbm_gbs (of measured)"},
         "km_kernel": {"ms": ki_avg, "bound": "host_link", "bytes": ab["km_host"], "peak": host_rand,
-                      "peak_source": "measured in-run: random-row zero-copy read over the whole host tier",
-                      "hbm_bytes": ab["km_hbm"]},
+                      "peak_source": f"measured in-run: random {prow} B-row zero-copy read over the whole host tier",
+                      "hbm_bytes": ab["km_hbm"], "includes": "km_kernel + kp_kernel" if w.pooled else "km_kernel"},
     }
     for kd in kern.values():
         kd["achieved"] = kd["bytes"] / (kd["ms"] * 1e-3) / 1e9
@@ -343,7 +387,7 @@ def main():
     lat = []
     for k in range(min(200, K)):
         t0 = time.perf_counter()
-        cache.query(views(ids_dev[W + k]), outs[k % 4])
+        step(W + k, outs[k % 4])
         stream.synchronize()
         lat.append((time.perf_counter() - t0) * 1e6)
     lat.sort()
@@ -351,10 +395,11 @@ def main():
     # end to end through the host-buffer entry point: H2D ids + query + D2H out per step
     log("e2e")
     e2e = None
-    if not args.no_e2e:
+    if not args.no_e2e and not w.pooled:
         KE = min(K, 100)
-        hids = [torch.from_numpy(gen_batch(P + W + K + KP + i)).pin_memory() for i in range(KE)]
-        hout = torch.empty(N * d, dtype=torch.float32).pin_memory()
+        lens = [w.batch_size] * w.n
+        hids = [torch.from_numpy(np.concatenate(gen_batch(P + W + K + KP + i).ids)).pin_memory() for i in range(KE)]
+        hout = torch.empty(cache.out_floats(lens), dtype=torch.float32).pin_memory()
         hv = [[h.numpy()[i * w.batch_size:(i + 1) * w.batch_size] for i in range(w.n)] for h in hids]
         torch.cuda.synchronize()
         if dist:
@@ -370,8 +415,9 @@ def main():
             t = torch.tensor([ems], device=dev)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             ems = float(t.item())
-        e2e = {"value": KE * N * world / (ems * 1e-3) / 1e6, "unit": "Mkeys/s", "h2d_bytes_per_step": N * 8,
-               "d2h_bytes_per_step": N * d * 4, "steps": KE,
+        NL = sum(lens)
+        e2e = {"value": KE * NL * world / (ems * 1e-3) / 1e6, "unit": "Mkeys/s", "h2d_bytes_per_step": NL * 8,
+               "d2h_bytes_per_step": cache.out_floats(lens) * 4, "steps": KE,
                "note": "fleche_query_host: pinned host IDs -> HBM, query, full output -> pinned host"}
 
     log("cpu baseline")
@@ -384,14 +430,17 @@ def main():
             "metric": "embedding lookups/s", "value": value, "unit": "Mkeys/s", "n_gpus": world, "steps": K,
             "warmup": W, "ms_per_step": ms_max / K, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
             "dtype": "f32", "data": "synthetic",
-            "config": {"workload": f"{w.name}: {w.n} tables, dim {d}, batch {w.batch_size} per GPU, cache "
-                                   f"{w.cache_frac:.0%} of table bytes, Zipf a={w.skews[0]}",
-                       "tables": w.n, "dim": d, "batch": w.batch_size, "lookups_per_step": N,
+            "config": {"workload": f"{w.name}: {w.n} tables, dim {d if uniform else 'mixed 8-128'}, "
+                                   f"{'bags' if w.pooled else 'batch'} {w.batch_size} per table per GPU"
+                                   f"{' (multi-hot, sum-pooled)' if w.pooled else ''}, cache "
+                                   f"{w.cache_frac:.0%} of table bytes, Zipf a={min(w.skews):.2f}-{max(w.skews):.2f}",
+                       "tables": w.n, "dim": d if uniform else sorted(set(w.dims)), "batch": w.batch_size,
+                       "lookups_per_step": dst["lookups"] / K,
                        "cache_bytes": w.cache_bytes, "host_table_bytes": w.table_bytes,
                        "parallelism": f"replicated x{world}" if world > 1 else "single GPU",
-                       "prefill_batches": P,
+                       "prefill_batches": P, "distinct_timed_batches": min(R, K),
                        "l2": "inputs larger than L2: fresh ID batch per step, 4 rotating output buffers "
-                             f"({4 * N * d * 4 / 1e6:.0f} MB), {w.cache_bytes / 1e6:.0f} MB slab"},
+                             f"({4 * out_max * 4 / 1e6:.0f} MB), {w.cache_bytes / 1e6:.0f} MB slab"},
             "hit_ratio": hit, "hit_ratio_unique": uhit,
             "unique_misses_per_step": dst["unique_misses"] / K,
             "p50_batch_latency_us": lat[len(lat) // 2], "p99_batch_latency_us": lat[int(len(lat) * 0.99) - 1],

@@ -219,7 +219,7 @@ EXPORT void flg_gen_bag_ids(uint64_t s_id, uint64_t s_perm, int64_t b, int64_t t
   perm_init(&p, s_perm, t, c);
 #ifdef _OPENMP
   if (nthreads <= 0) nthreads = omp_get_max_threads();
-#pragma omp parallel for schedule(static, 1024) num_threads(nthreads) if (bags > 16384)
+#pragma omp parallel for schedule(static, 256) num_threads(nthreads) if (bags >= 4096)
 #endif
   for (int64_t i = 0; i < bags; ++i) {
     for (int64_t k = offsets[i]; k < offsets[i + 1]; ++k) {
