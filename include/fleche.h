@@ -87,6 +87,15 @@ typedef struct {
  * (cp.async.bulk.prefetch.L2) so the miss kernel's loads hit L2.  Off by default: it
  * measured slower on B200 (profiles/README.md, round 1). */
 #define FLECHE_FLAG_L2_PREFETCH 0x1u
+/* Baseline / ablation modes (the paper's comparison point):
+ * STATIC_PER_TABLE: replace the flat cache by one static cache per table, each with
+ *   floor(frac * c_t) rows where frac = cache_bytes / sum_t 4 c_t d_t ("the same
+ *   proportion of cache size for all embedding tables"; reading R17), each a
+ *   32-way set-associative partition of its own (uniform layout per table);
+ * PER_TABLE_LAUNCH: launch the query kernel once per table (n launches instead of one
+ *   self-identified launch; the kernel-maintenance cost of P:L479-497). */
+#define FLECHE_FLAG_STATIC_PER_TABLE 0x2u
+#define FLECHE_FLAG_PER_TABLE_LAUNCH 0x4u
 
 typedef struct {
   uint64_t batches;            /* query calls                                                       */

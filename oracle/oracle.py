@@ -112,9 +112,12 @@ class Oracle:
             raise ValueError("or_create rejected the configuration")
 
     def __del__(self):
-        if getattr(self, "h", None):
-            lib().or_destroy(self.h)
-            self.h = None
+        try:
+            if getattr(self, "h", None) and _lib is not None:
+                _lib.or_destroy(self.h)
+                self.h = None
+        except Exception:  # interpreter shutdown
+            pass
 
     def out_size(self, lens) -> int:
         return int(sum(int(l) * int(d) for l, d in zip(lens, self.dims)))

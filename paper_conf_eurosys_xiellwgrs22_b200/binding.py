@@ -225,6 +225,10 @@ class FlatCache:
         sets, rows, d = self.geometry()
         keys = np.empty(sets * 32, np.uint32)
         ts = np.empty(sets * 32, np.uint32)
+        if d == 0:  # static per-table partitions: flat slab (rows of each table's width)
+            _check(fleche_debug_snapshot(self.h, keys.ctypes.data, ts.ctypes.data, keys.size, 0, 0),
+                   "fleche_debug_snapshot")
+            return keys, ts, None
         per = d if d > 0 else -d
         nrow = sets * 32 if d > 0 else sets
         slab = np.empty(nrow * per, np.float32)

@@ -34,11 +34,13 @@ struct fleche_ctx {
   std::vector<int32_t> fbits;
   int key_bits = 0;
   uint64_t capacity_bytes = 0;
+  uint64_t slab_floats = 0;
   std::vector<std::pair<void*, size_t>> registered;  // host ranges we registered
   Dev dv{};
   TableInfo* d_tables = nullptr;
   int km_blocks = 0;
   int km_bps = 4;  // KM CTAs per SM
+  bool per_table_launch = false;
   size_t km_smem = 0;
   // host-side counters
   uint64_t batches = 0, lookups = 0, kernels = 0;
@@ -155,6 +157,7 @@ fleche_status register_host(fleche_ctx* c, const float* const* host, std::vector
 
 void free_all(fleche_ctx* c) {
   void* ptrs[] = {c->dv.keys, c->dv.ts, c->dv.loc, c->dv.lock, c->dv.slab, c->dv.scratch, c->dv.dup_head,
+                  c->dv.firstpos, c->dv.ipos,
                   c->dv.miss, c->dv.dup, c->dv.ctl, c->dv.stats, c->d_tables, c->d_ids_stage, c->d_out_stage,
                   c->d_pool_stage};
   for (void* p : ptrs)
@@ -226,10 +229,27 @@ fleche_status launch_query(fleche_ctx* c, const int64_t* const* ids, const int64
   }
   fleche_status st = prof_event(c, s, true, nev);
   if (st != FLECHE_OK) return st;
-  if (total > 0) {
+  if (total > 0 && !c->per_table_launch) {
     const int64_t blocks = (total + 127) / 128;
     kq_kernel<MAXT><<<(unsigned)blocks, 128, 0, s>>>(qa, c->dv);
     c->kernels++;
+  } else if (total > 0) {  // ablation: one query launch per table (n launches)
+    QArgs<32> q1;
+    memset(&q1, 0, sizeof(q1));
+    q1.n = 1;
+    q1.out = out;
+    for (int k = 0; k < 8; ++k) q1.cls_off[k] = qa.cls_off[k];
+    for (int t = 0; t < c->n; ++t) {
+      if (lengths[t] == 0) continue;
+      q1.t0 = t;
+      q1.g0 = qa.scan[t];
+      q1.ids[0] = ids[t];
+      q1.scan[0] = 0;
+      q1.scan[1] = lengths[t];
+      q1.out_off[0] = qa.out_off[t];
+      kq_kernel<32><<<(unsigned)((lengths[t] + 127) / 128), 128, 0, s>>>(q1, c->dv);
+      c->kernels++;
+    }
   }
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
   if (c->dv.bytes) km_kernel<true><<<c->km_blocks, 128, c->km_smem, s>>>(c->dv, ka);
@@ -317,8 +337,8 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   *out = nullptr;
   const int n = cfg->num_tables;
   if (n < 1 || n > FLECHE_MAX_TABLES || !cfg->cardinalities || !cfg->dims || !cfg->host_tables) return FLECHE_EINVAL;
-  if (cfg->max_lookups < 1 || cfg->max_lookups > (int64_t(1) << 31) || (cfg->flags & ~FLECHE_FLAG_L2_PREFETCH))
-    return FLECHE_EINVAL;
+  const uint32_t known = FLECHE_FLAG_L2_PREFETCH | FLECHE_FLAG_STATIC_PER_TABLE | FLECHE_FLAG_PER_TABLE_LAUNCH;
+  if (cfg->max_lookups < 1 || cfg->max_lookups > (int64_t(1) << 31) || (cfg->flags & ~known)) return FLECHE_EINVAL;
   for (int t = 0; t < n; ++t) {
     if (cfg->cardinalities[t] < 1 || !valid_dim(cfg->dims[t])) return FLECHE_EINVAL;
     if (!cfg->host_tables[t] || ((uintptr_t)cfg->host_tables[t] & 15u)) return FLECHE_EINVAL;
@@ -338,7 +358,9 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   for (int t = 0; t < n; ++t)
     c->cls[t] = (int)(std::find(c->cls_dim.begin(), c->cls_dim.end(), c->dims[t]) - c->cls_dim.begin());
   c->max_dim = c->cls_dim.back();
-  const bool bytes = c->cls_dim.size() > 1;
+  const bool part = (cfg->flags & FLECHE_FLAG_STATIC_PER_TABLE) != 0;
+  const bool bytes = c->cls_dim.size() > 1 && !part;
+  c->per_table_launch = (cfg->flags & FLECHE_FLAG_PER_TABLE_LAUNCH) != 0;
   if (c->key_bits < 0) {
     delete c;
     return FLECHE_EINVAL;
@@ -354,7 +376,27 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   Dev& dv = c->dv;
   uint64_t sets, rows = 0;
   size_t slab_bytes;
-  if (!bytes) {  // uniform layout: way w of set s = slab row 32s + w
+  std::vector<uint32_t> p_off(n, 0), p_sets(n, 0), p_rows(n, 0);
+  std::vector<int64_t> p_slab(n, 0);
+  if (part) {  // static per-table partitions: rows_t = floor(frac * c_t), frac = cache / table bytes
+    unsigned __int128 tot = 0;
+    for (int t = 0; t < n; ++t) tot += (unsigned __int128)c->card[t] * (uint64_t)c->dims[t] * 4u;
+    uint64_t set_acc = 0, floats = 0;
+    c->capacity_bytes = 0;
+    for (int t = 0; t < n; ++t) {
+      const uint64_t r = (uint64_t)(((unsigned __int128)cfg->cache_bytes * (uint64_t)c->card[t]) / tot);
+      p_rows[t] = (uint32_t)std::min<uint64_t>(r, 0xFFFFFFE0ull);
+      p_sets[t] = (p_rows[t] + 31) / 32;
+      p_off[t] = (uint32_t)set_acc;
+      p_slab[t] = (int64_t)floats;
+      set_acc += p_sets[t];
+      floats += (uint64_t)p_sets[t] * 32u * (uint64_t)c->dims[t];
+      c->capacity_bytes += (uint64_t)p_rows[t] * 4u * (uint64_t)c->dims[t];
+    }
+    if (set_acc + 1 > 0xFFFFFFF0ull / 32) return fail(FLECHE_EINVAL);
+    sets = set_acc + 1;  // + one padding set (a 0-row partition points past the last one)
+    slab_bytes = (size_t)floats * 4u;
+  } else if (!bytes) {  // uniform layout: way w of set s = slab row 32s + w
     rows = cfg->cache_bytes / (4ull * (uint64_t)c->max_dim);
     if (rows > 0xFFFFFFE0ull) return fail(FLECHE_EINVAL);
     sets = std::max<uint64_t>(1, (rows + 31) / 32);
@@ -372,7 +414,9 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
     c->capacity_bytes = dv.set_units ? sets * set_bytes : 0;
   }
   const uint32_t scr_n = next_pow2(std::max<uint64_t>(1024, 2ull * (uint64_t)cfg->max_lookups));
+  c->slab_floats = slab_bytes / 4;
   dv.bytes = bytes ? 1 : 0;
+  dv.part = part ? 1 : 0;
   dv.sets = (uint32_t)sets;
   dv.rows = (uint32_t)rows;
   dv.dim = c->max_dim;
@@ -399,12 +443,14 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
             alloc((void**)&dv.dup, (size_t)cfg->max_lookups * sizeof(DupRec)) && alloc((void**)&dv.ctl, sizeof(Ctl)) &&
             alloc((void**)&dv.stats, sizeof(unsigned long long) * kStripes * kNumCtr) &&
             alloc((void**)&c->d_tables, sizeof(TableInfo) * n);
+  if (ok) ok = alloc((void**)&dv.firstpos, (size_t)scr_n * 8);
   if (ok && bytes) ok = alloc((void**)&dv.loc, ways * 2) && alloc((void**)&dv.lock, (size_t)sets * 4);
+  if (ok && !bytes) ok = alloc((void**)&dv.ipos, ways * 8);
   if (!ok) {
     cudaGetLastError();
     return fail(FLECHE_ENOMEM);
   }
-  c->index_bytes = ways * (bytes ? 10 : 8) + (bytes ? (size_t)sets * 4 : 0) + (size_t)scr_n * 16 +
+  c->index_bytes = ways * (bytes ? 10 : 16) + (bytes ? (size_t)sets * 4 : 0) + (size_t)scr_n * 24 +
                    (size_t)cfg->max_lookups * (sizeof(MissRec) + sizeof(DupRec));
   dv.tables = c->d_tables;
   if (cudaMemset(dv.keys, 0xFF, ways * 4) != cudaSuccess || cudaMemset(dv.ts, 0, ways * 4) != cudaSuccess ||
@@ -414,6 +460,8 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
     return fail(FLECHE_ECUDA);
   if (bytes && (cudaMemset(dv.loc, 0, ways * 2) != cudaSuccess || cudaMemset(dv.lock, 0, (size_t)sets * 4) != cudaSuccess))
     return fail(FLECHE_ECUDA);
+  if (!bytes && cudaMemset(dv.ipos, 0, ways * 8) != cudaSuccess) return fail(FLECHE_ECUDA);
+  if (cudaMemset(dv.firstpos, 0xFF, (size_t)scr_n * 8) != cudaSuccess) return fail(FLECHE_ECUDA);
   Ctl ctl{};
   ctl.epoch = 1;
   if (cudaMemcpy(dv.ctl, &ctl, sizeof(Ctl), cudaMemcpyHostToDevice) != cudaSuccess) return fail(FLECHE_ECUDA);
@@ -421,7 +469,9 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   std::vector<const float*> dptr;
   if (register_host(c, cfg->host_tables, dptr) != FLECHE_OK) return fail(FLECHE_ECUDA);
   std::vector<TableInfo> ti(n);
-  for (int t = 0; t < n; ++t) ti[t] = TableInfo{dptr[t], c->card[t], (uint32_t)c->base[t], c->dims[t], c->cls[t], 0};
+  for (int t = 0; t < n; ++t)
+    ti[t] = TableInfo{dptr[t], c->card[t], (uint32_t)c->base[t], c->dims[t], c->cls[t], p_off[t], p_sets[t],
+                      p_rows[t], p_slab[t]};
   if (cudaMemcpy(c->d_tables, ti.data(), sizeof(TableInfo) * n, cudaMemcpyHostToDevice) != cudaSuccess)
     return fail(FLECHE_ECUDA);
   if (cudaEventCreateWithFlags(&c->chain_ev, cudaEventDisableTiming) != cudaSuccess) return fail(FLECHE_ECUDA);
@@ -576,8 +626,8 @@ fleche_status fleche_get_encoding(fleche_ctx* c, uint64_t* base, int32_t* fbits,
 fleche_status fleche_get_geometry(fleche_ctx* c, int64_t* sets, int64_t* rows, int32_t* row_floats) {
   if (!c) return FLECHE_EINVAL;
   if (sets) *sets = c->dv.sets;
-  if (rows) *rows = c->dv.bytes ? 0 : c->dv.rows;
-  if (row_floats) *row_floats = c->dv.bytes ? -(int32_t)(c->dv.set_units * 8) : c->max_dim;
+  if (rows) *rows = (c->dv.bytes || c->dv.part) ? 0 : c->dv.rows;
+  if (row_floats) *row_floats = c->dv.part ? 0 : (c->dv.bytes ? -(int32_t)(c->dv.set_units * 8) : c->max_dim);
   return FLECHE_OK;
 }
 
@@ -586,7 +636,7 @@ fleche_status fleche_debug_snapshot(fleche_ctx* c, uint32_t* keys, uint32_t* ts,
   if (!c) return FLECHE_EINVAL;
   if (c->poisoned) return FLECHE_ESTATE;
   const size_t ways = (size_t)c->dv.sets * 32u;
-  const size_t slab_floats = c->dv.bytes ? (size_t)c->dv.sets * c->dv.set_units * 8u : ways * (size_t)c->max_dim;
+  const size_t slab_floats = c->slab_floats;
   if ((keys || ts) && ways_cap < ways) return FLECHE_EINVAL;
   if (slab && slab_floats_cap < slab_floats) return FLECHE_EINVAL;
   fleche_status st = ensure_device(c);

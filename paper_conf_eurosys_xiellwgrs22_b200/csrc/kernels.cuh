@@ -64,7 +64,10 @@ struct TableInfo {
   uint32_t base;      // first flat key of table t (size-aware coding)
   int32_t dim;        // d_t
   int32_t cls;        // width class (index into the per-call class regions)
-  int32_t pad;
+  uint32_t set_off;   // static per-table mode: first set of table t's partition
+  uint32_t sets;      //   number of sets of the partition
+  uint32_t rows;      //   capacity rows of the partition (last set may be partial)
+  int64_t slab_off;   //   float offset of the partition's rows in the slab
 };
 
 struct MissRec {  // one unique missed key (its owner lookup)
@@ -98,6 +101,8 @@ struct Dev {
   float* slab;      // uniform: [sets*32][dim];  bytes: [sets][set_units * 8]
   unsigned long long* scratch;   // [scr_mask+1] (epoch << 32 | fk) dedup tags
   unsigned long long* dup_head;  // [scr_mask+1] (epoch << 32 | first duplicate + 1)
+  unsigned long long* firstpos;  // [scr_mask+1] (~epoch << 32 | first occurrence of the key in the batch)
+  unsigned long long* ipos;      // uniform layout: [sets][32] (epoch << 32 | inserter's first occurrence << 1 | busy)
   MissRec* miss;                 // [max_lookups], split into per-class regions per call
   DupRec* dup;                   // [max_lookups]
   Ctl* ctl;
@@ -110,6 +115,8 @@ struct Dev {
   int32_t km_m;      // unique misses per KM warp iteration (4, 8, 16, 32)
   int32_t bytes;     // 0 = uniform layout, 1 = bytes layout
   uint32_t set_units;  // bytes layout: region of a set in 32 B units (<= 256)
+  int32_t part;      // static per-table partitions (HugeCTR-like baseline, NEXT-1)
+  int32_t t0;        // unused padding slot
 #ifdef FLECHE_EXPERIMENTS
   int32_t exp_mode;  // timing experiments only (libfleche_exp.so); breaks semantics
   int32_t exp_pad;
@@ -123,8 +130,9 @@ struct QArgs {
   int64_t out_off[MAXT];     // float offset of O_t in out
   int64_t cls_off[8];        // start of each class's region of the miss list
   float* out;
+  int64_t g0;                // batch position of this launch's first lookup (per-table launches)
   int32_t n;
-  int32_t pad;
+  int32_t t0;                // first table of this launch (per-table launches: t0 = t, n = 1)
 };
 
 struct KMArgs {
@@ -161,6 +169,20 @@ __device__ __forceinline__ uint32_t set_of(const Dev& dv, uint32_t fk) {
 __device__ __forceinline__ int ways_in(const Dev& dv, uint32_t s) {
   const uint32_t lo = s * 32u;
   return dv.rows - lo >= 32u ? 32 : (int)(dv.rows - lo);
+}
+// Static per-table mode: table t's keys live only in its own partition of sets.
+__device__ __forceinline__ uint32_t set_of_t(const Dev& dv, const TableInfo* ti, uint32_t fk) {
+  return dv.part ? ti->set_off + __umulhi(fmix32(fk ^ dv.hash_seed), ti->sets) : set_of(dv, fk);
+}
+__device__ __forceinline__ int ways_in_t(const Dev& dv, const TableInfo* ti, uint32_t s) {
+  if (!dv.part) return ways_in(dv, s);
+  const uint32_t lo = (s - ti->set_off) * 32u;
+  return ti->rows <= lo ? 0 : (ti->rows - lo >= 32u ? 32 : (int)(ti->rows - lo));
+}
+// Uniform layout: slab row of a slot (global slot = 32 * set + way).
+__device__ __forceinline__ float* slot_row(const Dev& dv, const TableInfo* ti, uint32_t slot, int d) {
+  return dv.part ? dv.slab + ti->slab_off + (size_t)(slot - ti->set_off * 32u) * (size_t)d
+                 : dv.slab + (size_t)slot * (size_t)d;
 }
 __device__ __forceinline__ uint32_t scr_hash(uint32_t fk) { return fmix32(fk * 0x9E3779B1u + 0x632BE5ABu); }
 __device__ __forceinline__ uint64_t splitmix64(uint64_t x) {
@@ -339,7 +361,7 @@ __global__ void __launch_bounds__(128) kq_kernel(const __grid_constant__ QArgs<M
       t = lo;
     }
     const int64_t j = g - s_scan[t];
-    const TableInfo* ti = dv.tables + t;
+    const TableInfo* ti = dv.tables + qa.t0 + t;
     const int64_t id = active ? qa.ids[t][j] : -1;
     const int64_t card = ti->card;
     const int d = ti->dim;
@@ -347,7 +369,7 @@ __global__ void __launch_bounds__(128) kq_kernel(const __grid_constant__ QArgs<M
     // A2 re-encode to the flat key (size-aware code: fk = base_t + id)
     const bool valid = active && id >= 0 && id < card;
     const uint32_t fk = valid ? ti->base + (uint32_t)id : kEmpty;
-    const uint32_t s = valid ? set_of(dv, fk) : 0u;
+    const uint32_t s = valid ? set_of_t(dv, ti, fk) : 0u;
 
     // A3 probe: lane k holds way k of each of the warp's 32 sets (one 128 B line each)
     uint32_t kw[32];
@@ -372,7 +394,7 @@ __global__ void __launch_bounds__(128) kq_kernel(const __grid_constant__ QArgs<M
     const float* src = nullptr;
     if (hit) {
       if (!dv.bytes) {
-        src = dv.slab + (size_t)slot * (size_t)d;
+        src = slot_row(dv, ti, slot, d);
       } else {
         const uint32_t l = ld_nc_u32((const uint32_t*)(dv.loc + (slot & ~1u))) >> ((slot & 1u) * 16);
         src = dv.slab + ((size_t)s * dv.set_units + (l & 0xFFu)) * 8u;
@@ -415,6 +437,8 @@ __global__ void __launch_bounds__(128) kq_kernel(const __grid_constant__ QArgs<M
         cur = ld_cg_u64(dv.scratch + h);
       }
       scr = h;
+      // first occurrence of the key in canonical (table-major) order: the insert priority
+      atomicMin(dv.firstpos + h, ((unsigned long long)(~epoch) << 32) | (uint32_t)(qa.g0 + g));
     }
 
     const int par = epoch & 1u;
@@ -429,7 +453,7 @@ __global__ void __launch_bounds__(128) kq_kernel(const __grid_constant__ QArgs<M
       if (kind == 1 && lane == leader) b = atomicAdd(&dv.ctl->counts[par][cls], (uint32_t)__popc(grp));
       b = __shfl_sync(kFull, b, leader);
       if (kind == 1) {
-        dv.miss[qa.cls_off[cls] + b + __popc(grp & lt)] = MissRec{off, fk, scr, t, 0};
+        dv.miss[qa.cls_off[cls] + b + __popc(grp & lt)] = MissRec{off, fk, scr, qa.t0 + t, 0};
         if (dv.prefetch) {  // experimental: start the host-link transfer now
           const float* hrow = ti->host + (size_t)id * (size_t)d;
           asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(hrow), "r"(4u * (unsigned)d) : "memory");
@@ -474,15 +498,26 @@ __global__ void __launch_bounds__(128) kq_kernel(const __grid_constant__ QArgs<M
     atomicAdd(dv.stats + (blockIdx.x % kStripes) * kNumCtr + threadIdx.x, s_ctr[threadIdx.x]);
 }
 
-// Uniform layout: victim way for fk in its set = argmin (ts, key) over ways with
-// ts < epoch, claimed by CAS(ts: old -> epoch).  Returns the slot, or -1 if every way
-// of the set was read or written in this batch (epoch protection: bypass).  One lane,
-// 16 vector loads, no warp synchronisation.
-__device__ __forceinline__ int64_t claim_victim(const Dev& dv, uint32_t fk, uint32_t epoch, uint32_t* old_key) {
-  const uint32_t s = set_of(dv, fk);
-  const int nways = ways_in(dv, s);
+// Uniform layout: claim a way for fk (first occurrence `pos` in the batch).
+//  * victim = argmin (ts, key) over ways not read or written in this batch, claimed by a
+//    CAS on its insert word ipos (epoch << 32 | pos << 1 | BUSY), then ts := epoch;
+//  * no such way left: take over the way inserted in this batch by the miss with the
+//    LARGEST first-occurrence position, if that is larger than ours.
+// The set then ends up holding exactly the set's earliest-occurring misses, with exactly
+// the argmin-(ts, key) candidates evicted -- what the oracle's first-occurrence insert
+// order produces (reading R7) -- whatever order the warps run in.
+// Returns the slot (>= 0), kClaimBypass, or kClaimRetry (the way to take over is still
+// being written by its claimer: try again after this warp's own writes).  One lane.
+constexpr int64_t kClaimBypass = -1, kClaimRetry = -2;
+__device__ __forceinline__ int64_t claim_victim(const Dev& dv, const TableInfo* ti, uint32_t fk, uint32_t epoch,
+                                                uint32_t pos, uint32_t* old_key, bool* took_over) {
+  const uint32_t s = set_of_t(dv, ti, fk);
+  const int nways = ways_in_t(dv, ti, s);
+  if (nways <= 0) return kClaimBypass;
   const uint32_t* kp = dv.keys + (size_t)s * 32u;
   uint32_t* tp = dv.ts + (size_t)s * 32u;
+  unsigned long long* ip = dv.ipos + (size_t)s * 32u;
+  const unsigned long long mine = ((unsigned long long)epoch << 32) | ((unsigned long long)pos << 1) | 1ull;
   while (true) {
     uint32_t kk[32], tt[32];
 #pragma unroll
@@ -498,11 +533,29 @@ __device__ __forceinline__ int64_t claim_victim(const Dev& dv, uint32_t fk, uint
       const unsigned long long r = ((unsigned long long)tt[w] << 32) | kk[w];
       if (w < nways && tt[w] < epoch && r < best) { best = r; bw = w; }
     }
-    if (bw < 0) return -1;
-    if (atomicCAS(tp + bw, (uint32_t)(best >> 32), epoch) == (uint32_t)(best >> 32)) {
-      *old_key = (uint32_t)best;
+    if (bw >= 0) {
+      const unsigned long long cur = ld_cg_u64(ip + bw);
+      if ((uint32_t)(cur >> 32) == epoch) continue;  // claimed an instant ago; its ts is on the way
+      if (atomicCAS(ip + bw, cur, mine) != cur) continue;
+      tp[bw] = epoch;
+      *old_key = kk[bw];
+      *took_over = false;
       return (int64_t)s * 32 + bw;
     }
+    // every way was read or written in this batch: the latest-occurring insert of this
+    // batch gives way if we occur earlier
+    unsigned long long worst = 0;
+    int ww = -1;
+    for (int w = 0; w < nways; ++w) {
+      const unsigned long long v = ld_cg_u64(ip + w);
+      if ((uint32_t)(v >> 32) == epoch && (v | 1ull) > (worst | 1ull)) { worst = v; ww = w; }
+    }
+    if (ww < 0 || ((worst >> 1) & 0x7FFFFFFFull) <= pos) return kClaimBypass;
+    if (worst & 1ull) return kClaimRetry;  // still being written by its claimer
+    if (atomicCAS(ip + ww, worst, mine) != worst) continue;
+    *old_key = kk[ww];
+    *took_over = true;
+    return (int64_t)s * 32 + ww;
   }
 }
 
@@ -634,25 +687,41 @@ __device__ __forceinline__ void km_rows(const Dev& dv, float* __restrict__ out, 
     }
     if constexpr (!BYTES) {
       // A7 while the loads are in flight: victim claim (L2 round trips only)
-      float* slab_dst = nullptr;
-      uint32_t slot32 = 0;
-      if (has) {
-        int64_t slot = -1;
-        uint32_t old_key = kEmpty;
-        if (admit) slot = claim_victim(dv, m.fk, epoch, &old_key);
-        if (slot >= 0) {
-          ++ins;
-          docc += 4ll * D;
-          if (old_key != kEmpty) { ++ev; docc -= 4ll * D; }
-          slab_dst = dv.slab + (size_t)slot * D;
-          slot32 = (uint32_t)slot;
-        } else {
-          ++byp;
-        }
-      }
       rb.store(has ? out + m.off : nullptr, lane);
-      rb.store(slab_dst, lane);
-      if (slab_dst) dv.keys[slot32] = m.fk;
+      bool pending = has && admit;
+      if (has && !admit) ++byp;
+      const TableInfo* ti = dv.tables + (has ? m.t : 0);
+      const uint32_t pos = pending ? (uint32_t)ld_cg_u64(dv.firstpos + m.scr) : 0u;
+      while (__any_sync(kFull, pending)) {  // rounds: a lane may wait for a way its warp still writes
+        float* slab_dst = nullptr;
+        int64_t slot = kClaimRetry;
+        if (pending) {
+          uint32_t old_key = kEmpty;
+          bool took = false;
+          slot = claim_victim(dv, ti, m.fk, epoch, pos, &old_key, &took);
+          if (slot >= 0) {
+            pending = false;
+            if (took) {
+              ++byp;  // the later-occurring miss we displaced is bypassed; our insert replaces its
+            } else {
+              ++ins;
+              docc += 4ll * D;
+              if (old_key != kEmpty) { ++ev; docc -= 4ll * D; }
+            }
+            slab_dst = slot_row(dv, ti, (uint32_t)slot, D);
+          } else if (slot == kClaimBypass) {
+            pending = false;
+            ++byp;
+          }
+        }
+        rb.store(slab_dst, lane);
+        if (slab_dst) {  // row -> key -> release the way (clears BUSY)
+          dv.keys[slot] = m.fk;
+          __threadfence();
+          *(volatile unsigned long long*)(dv.ipos + slot) = ((unsigned long long)epoch << 32) | ((unsigned long long)pos << 1);
+        }
+        if (slot == kClaimRetry && pending) __nanosleep(100);
+      }
     } else {
       rb.store(has ? out + m.off : nullptr, lane);
       rb.to_smem(wsm, lane);
