@@ -156,7 +156,7 @@ fleche_status register_host(fleche_ctx* c, const float* const* host, std::vector
 }
 
 void free_all(fleche_ctx* c) {
-  void* ptrs[] = {c->dv.keys, c->dv.ts, c->dv.loc, c->dv.lock, c->dv.slab, c->dv.scratch, c->dv.dup_head,
+  void* ptrs[] = {c->dv.keys, c->dv.ts, c->dv.loc, c->dv.lock, c->dv.slab, c->dv.scratch, c->dv.owner_off,
                   c->dv.firstpos, c->dv.ipos,
                   c->dv.miss, c->dv.dup, c->dv.ctl, c->dv.stats, c->d_tables, c->d_ids_stage, c->d_out_stage,
                   c->d_pool_stage};
@@ -254,7 +254,8 @@ fleche_status launch_query(fleche_ctx* c, const int64_t* const* ids, const int64
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
   if (c->dv.bytes) km_kernel<true><<<c->km_blocks, 128, c->km_smem, s>>>(c->dv, ka);
   else km_kernel<false><<<c->km_blocks, 128, 0, s>>>(c->dv, ka);
-  c->kernels++;
+  kd_kernel<<<c->km_blocks, 128, 0, s>>>(c->dv, out);
+  c->kernels += 2;
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return poison(c, e, "kernel launch");
@@ -438,7 +439,7 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   auto alloc = [&](void** ptr, size_t b) { return cudaMalloc(ptr, std::max<size_t>(b, 16)) == cudaSuccess; };
   const size_t ways = (size_t)sets * 32u;
   bool ok = alloc((void**)&dv.keys, ways * 4) && alloc((void**)&dv.ts, ways * 4) && alloc((void**)&dv.slab, slab_bytes) &&
-            alloc((void**)&dv.scratch, (size_t)scr_n * 8) && alloc((void**)&dv.dup_head, (size_t)scr_n * 8) &&
+            alloc((void**)&dv.scratch, (size_t)scr_n * 8) && alloc((void**)&dv.owner_off, (size_t)scr_n * 8) &&
             alloc((void**)&dv.miss, (size_t)cfg->max_lookups * sizeof(MissRec)) &&
             alloc((void**)&dv.dup, (size_t)cfg->max_lookups * sizeof(DupRec)) && alloc((void**)&dv.ctl, sizeof(Ctl)) &&
             alloc((void**)&dv.stats, sizeof(unsigned long long) * kStripes * kNumCtr) &&
@@ -455,7 +456,6 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   dv.tables = c->d_tables;
   if (cudaMemset(dv.keys, 0xFF, ways * 4) != cudaSuccess || cudaMemset(dv.ts, 0, ways * 4) != cudaSuccess ||
       cudaMemset(dv.scratch, 0, (size_t)scr_n * 8) != cudaSuccess ||
-      cudaMemset(dv.dup_head, 0, (size_t)scr_n * 8) != cudaSuccess ||
       cudaMemset(dv.stats, 0, sizeof(unsigned long long) * kStripes * kNumCtr) != cudaSuccess)
     return fail(FLECHE_ECUDA);
   if (bytes && (cudaMemset(dv.loc, 0, ways * 2) != cudaSuccess || cudaMemset(dv.lock, 0, (size_t)sets * 4) != cudaSuccess))

@@ -80,8 +80,8 @@ struct MissRec {  // one unique missed key (its owner lookup)
 
 struct DupRec {  // a later occurrence of a missed key in the same batch
   int64_t off;   // float offset of the duplicate's row in `out`
-  uint32_t next; // next duplicate + 1 (0 = end of chain)
-  uint32_t pad;
+  uint32_t scr;  // scratch slot of the key -> its owner's row (owner_off)
+  int32_t dim;   // row width
 };
 
 struct Ctl {
@@ -100,7 +100,7 @@ struct Dev {
   uint32_t* lock;   // bytes layout: [sets] insert locks
   float* slab;      // uniform: [sets*32][dim];  bytes: [sets][set_units * 8]
   unsigned long long* scratch;   // [scr_mask+1] (epoch << 32 | fk) dedup tags
-  unsigned long long* dup_head;  // [scr_mask+1] (epoch << 32 | first duplicate + 1)
+  int64_t* owner_off;            // [scr_mask+1] float offset in `out` of the key's owner row
   unsigned long long* firstpos;  // [scr_mask+1] (~epoch << 32 | first occurrence of the key in the batch)
   unsigned long long* ipos;      // uniform layout: [sets][32] (epoch << 32 | inserter's first occurrence << 1 | busy)
   MissRec* miss;                 // [max_lookups], split into per-class regions per call
@@ -454,6 +454,7 @@ __global__ void __launch_bounds__(128) kq_kernel(const __grid_constant__ QArgs<M
       b = __shfl_sync(kFull, b, leader);
       if (kind == 1) {
         dv.miss[qa.cls_off[cls] + b + __popc(grp & lt)] = MissRec{off, fk, scr, qa.t0 + t, 0};
+        dv.owner_off[scr] = off;
         if (dv.prefetch) {  // experimental: start the host-link transfer now
           const float* hrow = ti->host + (size_t)id * (size_t)d;
           asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(hrow), "r"(4u * (unsigned)d) : "memory");
@@ -464,18 +465,7 @@ __global__ void __launch_bounds__(128) kq_kernel(const __grid_constant__ QArgs<M
       uint32_t b = 0;
       if (lane == __ffs(dup_m) - 1) b = atomicAdd(&dv.ctl->counts[par][kDupSlot], (uint32_t)__popc(dup_m));
       b = __shfl_sync(kFull, b, __ffs(dup_m) - 1);
-      if (kind == 2) {  // push onto the key's duplicate chain (epoch-tagged head)
-        const uint32_t idx = b + __popc(dup_m & lt);
-        unsigned long long old = ld_cg_u64(dv.dup_head + scr);
-        while (true) {
-          const uint32_t next = ((uint32_t)(old >> 32) == epoch) ? (uint32_t)old : 0u;
-          dv.dup[idx] = DupRec{off, next, 0};
-          const unsigned long long nw = ((unsigned long long)epoch << 32) | (idx + 1u);
-          const unsigned long long prev = atomicCAS(dv.dup_head + scr, old, nw);
-          if (prev == old) break;
-          old = prev;
-        }
-      }
+      if (kind == 2) dv.dup[b + __popc(dup_m & lt)] = DupRec{off, scr, d};  // restored by KD
     }
 
     // A9 stats, warp-aggregated then block-aggregated
@@ -737,21 +727,6 @@ __device__ __forceinline__ void km_rows(const Dev& dv, float* __restrict__ out, 
         if (lane == 0) { if (ok) ++ins; else ++byp; }
       }
     }
-    // A8 restore: walk each miss's duplicate chain
-    uint32_t p = 0;
-    if (has) {
-      const unsigned long long h = ld_cg_u64(dv.dup_head + m.scr);
-      p = ((uint32_t)(h >> 32) == epoch) ? (uint32_t)h : 0u;
-    }
-    while (__any_sync(kFull, p != 0)) {
-      float* o = nullptr;
-      if (p) {
-        const DupRec r = dv.dup[p - 1];
-        o = out + r.off;
-        p = r.next;
-      }
-      rb.store(o, lane);
-    }
     __syncwarp();
   }
 }
@@ -816,6 +791,24 @@ __global__ void __launch_bounds__(128, 4) km_kernel(const __grid_constant__ Dev 
   __syncthreads();
   if (threadIdx.x < kNumCtr && s_ctr[threadIdx.x])
     atomicAdd(dv.stats + (blockIdx.x % kStripes) * kNumCtr + threadIdx.x, s_ctr[threadIdx.x]);
+}
+
+// KD restore: every duplicate occurrence of a missed key copies its owner's
+// row (written by KM) in parallel; then the last CTA closes the batch: resets the next
+// batch's counters and advances the device-resident epoch (graph-replay safe).
+__global__ void __launch_bounds__(128) kd_kernel(const __grid_constant__ Dev dv, float* __restrict__ out) {
+  const uint32_t epoch = *(volatile uint32_t*)&dv.ctl->epoch;
+  const int par = epoch & 1u;
+  const uint32_t ndup = *(volatile uint32_t*)&dv.ctl->counts[par][kDupSlot];
+  const int lane = threadIdx.x & 31;
+  const uint32_t gw = (threadIdx.x >> 5) * gridDim.x + blockIdx.x;
+  const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
+  for (uint32_t k = gw; k < ndup; k += nw) {
+    const DupRec r = dv.dup[k];
+    const float* src = out + dv.owner_off[r.scr];
+    for (int c = lane; c < r.dim / 4; c += 32) st_v4(out + r.off + 4 * c, ld_cg_v4(src + 4 * c));
+  }
+  __syncthreads();
   if (threadIdx.x == 0) {
     __threadfence();
     const uint32_t prev = atomicAdd(&dv.ctl->done, 1u);

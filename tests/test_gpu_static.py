@@ -91,7 +91,7 @@ def test_per_table_launch_matches_fused_exactly():
     assert sa["bypassed"] == 0
     for k in H.STAT_KEYS_EXACT:
         assert sa[k] == sc[k], k
-    assert sc["kernels_launched"] == 15 * (w.n + 1) and sa["kernels_launched"] == 30
+    assert sc["kernels_launched"] == 15 * (w.n + 2) and sa["kernels_launched"] == 45  # KQ(s) + KM + KD
 
 
 def test_flat_beats_static_on_skewed_table_sizes():
