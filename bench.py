@@ -234,7 +234,14 @@ def main():
     # host tier: every table in one buffer, page-locked + mapped by fleche_create
     log("host tier")
     t_gen = time.time()
-    hostbuf, tabs = w.make_tables()
+    shm_cleanup = None
+    if dist:  # one copy per node in /dev/shm, mapped by every local rank
+        from workload import shm
+        hostbuf, tabs, shm_cleanup = shm.shared_tables(
+            f"fleche_{w.name}_{os.environ.get('MASTER_PORT', '0')}", w.cards, w.dims, w.value_mode, local,
+            dist.barrier)
+    else:
+        hostbuf, tabs = w.make_tables()
     t_gen = time.time() - t_gen
     log("create")
     cache = fl.FlatCache(w.cards, w.dims, tabs, w.cache_bytes, N, local, 1.0, 0, HASH_SEED, args.flags)
@@ -449,6 +456,9 @@ def main():
             "host_tier_gen_s": t_gen,
         }), flush=True)
     if dist:
+        dist.barrier()
+        if shm_cleanup:
+            shm_cleanup()
         dist.destroy_process_group()
 
 
