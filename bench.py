@@ -45,6 +45,8 @@ def parse():
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=15.0, help="oracle sample budget")
     p.add_argument("--flags", type=int, default=0, help="fleche_config.flags (ablations)")
+    p.add_argument("--mode", default="replicated", choices=["replicated", "sharded"],
+                   help="multi-GPU partitioning: per-GPU replicated caches, or one key-sharded cache (NCCL all-to-all)")
     return p.parse_args()
 
 
@@ -244,7 +246,19 @@ def main():
         hostbuf, tabs = w.make_tables()
     t_gen = time.time() - t_gen
     log("create")
-    cache = fl.FlatCache(w.cards, w.dims, tabs, w.cache_bytes, N, local, 1.0, 0, HASH_SEED, args.flags)
+    sharded = args.mode == "sharded"
+    if sharded and (w.pooled or not uniform):
+        raise SystemExit("--mode sharded supports one-hot, uniform-width configs (cfg1, cfg2, cfg5)")
+    cache = fl.FlatCache(w.cards, w.dims, tabs, w.cache_bytes, N * (world if sharded else 1), local, 1.0, 0,
+                         HASH_SEED, args.flags)
+    shard = None
+    if sharded:
+        if dist is None:
+            import torch.distributed as dist
+            dist.init_process_group("nccl", init_method="tcp://127.0.0.1:%d" % (29600 + os.getpid() % 300),
+                                    rank=0, world_size=1, device_id=torch.device("cuda", local))
+        from paper_conf_eurosys_xiellwgrs22_b200.sharded import ShardedCache
+        shard = ShardedCache(cache, row_floats=d)
     stream = torch.cuda.current_stream()
 
     def gen_batch(b):
@@ -275,6 +289,8 @@ def main():
         def run(self, out):
             if self.bags is not None:
                 cache.query_pooled(self.idv, self.offv, out, bags=self.bags, nnz=self.lens)
+            elif shard is not None:
+                shard.query(self.idv, out, lengths=self.lens)
             else:
                 cache.query(self.idv, out, lengths=self.lens)
 
@@ -310,6 +326,7 @@ def main():
     if dist:
         dist.barrier()
     s0 = cache.stats()
+    r0 = cache.shard_stats() if sharded else None
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     torch.cuda.synchronize()
     tw0 = time.perf_counter()
@@ -332,9 +349,16 @@ def main():
         ms_max = float(t.item())
     dst = {k: s1[k] - s0[k] for k in fl.STAT_FIELDS}
     keys_total = dst["lookups"] * world
-    value = keys_total / (ms_max * 1e-3) / 1e6
     hit = dst["hits"] / max(1, dst["hits"] + dst["misses"])
     uhit = dst["unique_hits"] / max(1, dst["unique_keys"])
+    if sharded:  # requester side: this rank's batch lookups and how many hit at their owner
+        r1 = cache.shard_stats()
+        dr = {k: r1[k] - r0[k] for k in r1}
+        keys_total = dr["lookups"] * world
+        hit = dr["hits"] / max(1, dr["lookups"] - dr["invalid"])
+        uhit = dst["unique_hits"] / max(1, dst["unique_keys"])  # at this rank as an owner
+        dst["unique_misses_owner"] = dst["unique_misses"]
+    value = keys_total / (ms_max * 1e-3) / 1e6
 
     # per-kernel device time (profiled pass: CUDA events on the launching stream)
     log("profiled pass")
@@ -402,7 +426,7 @@ def main():
     # end to end through the host-buffer entry point: H2D ids + query + D2H out per step
     log("e2e")
     e2e = None
-    if not args.no_e2e and not w.pooled:
+    if not args.no_e2e and not w.pooled and not sharded:
         KE = min(K, 100)
         lens = [w.batch_size] * w.n
         hids = [torch.from_numpy(np.concatenate(gen_batch(P + W + K + KP + i).ids)).pin_memory() for i in range(KE)]
@@ -444,7 +468,8 @@ def main():
                        "tables": w.n, "dim": d if uniform else sorted(set(w.dims)), "batch": w.batch_size,
                        "lookups_per_step": dst["lookups"] / K,
                        "cache_bytes": w.cache_bytes, "host_table_bytes": w.table_bytes,
-                       "parallelism": f"replicated x{world}" if world > 1 else "single GPU",
+                       "parallelism": (f"key-sharded x{world} (NCCL all-to-all)" if sharded else
+                                       (f"replicated x{world}" if world > 1 else "single GPU")),
                        "prefill_batches": P, "distinct_timed_batches": min(R, K),
                        "l2": "inputs larger than L2: fresh ID batch per step, 4 rotating output buffers "
                              f"({4 * out_max * 4 / 1e6:.0f} MB), {w.cache_bytes / 1e6:.0f} MB slab"},

@@ -188,6 +188,34 @@ fleche_status fleche_debug_snapshot(fleche_ctx* ctx, uint32_t* keys, uint32_t* t
                                     size_t slab_floats_cap);
 fleche_status fleche_debug_locations(fleche_ctx* ctx, uint16_t* loc, size_t ways_cap);
 
+/* Key-sharded multi-GPU mode (the paper leaves multi-GPU caching to
+ * future work).  Rank r of G caches only the keys it OWNS:
+ * owner(fk) = (fmix32(fk ^ owner_seed ^ 0x85EBCA77) * G) >> 32, so the G per-GPU
+ * budgets aggregate.  One batch on every rank (all calls on the same stream):
+ *   1. fleche_route(ids, lengths, G, seed, send_keys, send_counts): dedups the batch's
+ *      valid flat keys and writes them grouped by owner (send_keys[sum counts], uint32
+ *      flat keys, DEVICE) with per-owner counts (send_counts[G], int64, DEVICE).
+ *   2. the caller exchanges counts and keys with an all-to-all (NCCL over NVLink);
+ *   3. fleche_query_keys(recv_keys, R, rows, flags): the owner answers R flat keys
+ *      (its share of every rank's batch) with the ordinary query/miss/restore kernels:
+ *      rows[R x d] fp32 (DEVICE, row g answers key g), hit_flags[R] (DEVICE, 1 = hit;
+ *      may be NULL); this is one batch (epoch) of the owner's cache;
+ *   4. the caller returns rows (and flags) with an all-to-all, owners in rank order,
+ *      each owner's rows in the order the keys were sent;
+ *   5. fleche_restore(rows_back, flags_back, out): out (layout of fleche_query for the
+ *      lengths of step 1) gets every lookup's row; invalid IDs give a zero row.
+ * Uniform row widths only (FLECHE_EINVAL otherwise); G <= 64.
+ * fleche_shard_stats: requester-side counters: lookups routed, lookups whose key hit
+ * at its owner, invalid IDs, unique keys routed (summed over batches). */
+fleche_status fleche_route(fleche_ctx* ctx, const int64_t* const* ids, const int64_t* lengths, int32_t world,
+                           uint32_t owner_seed, uint32_t* send_keys, int64_t* send_counts, fleche_stream stream);
+fleche_status fleche_query_keys(fleche_ctx* ctx, const uint32_t* keys, int64_t count, float* rows,
+                                uint8_t* hit_flags, fleche_stream stream);
+fleche_status fleche_restore(fleche_ctx* ctx, const float* rows, const uint8_t* hit_flags, float* out,
+                             fleche_stream stream);
+fleche_status fleche_shard_stats(fleche_ctx* ctx, uint64_t* lookups, uint64_t* hits, uint64_t* invalid,
+                                 uint64_t* unique_routed);
+
 /* Diagnostics for measurement (bench.py).
  * fleche_set_profiling: when enabled, every later query records CUDA events on its
  *   stream around each of its kernels (adds ~3 event records per call).

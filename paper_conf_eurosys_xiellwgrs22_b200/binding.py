@@ -68,12 +68,17 @@ fleche_probe_host_read = _sig("fleche_probe_host_read", ctypes.c_int, [_vp, _u64
                                                                        ctypes.POINTER(ctypes.c_double)])
 
 fleche_query_pooled = _sig("fleche_query_pooled", ctypes.c_int, [_vp, _vp, _vp, _vp, _vp, _vp, _vp])
+fleche_route = _sig("fleche_route", ctypes.c_int, [_vp, _vp, _vp, _i32, _u32, _vp, _vp, _vp])
+fleche_query_keys = _sig("fleche_query_keys", ctypes.c_int, [_vp, _vp, _i64, _vp, _vp, _vp])
+fleche_restore = _sig("fleche_restore", ctypes.c_int, [_vp, _vp, _vp, _vp, _vp])
+fleche_shard_stats = _sig("fleche_shard_stats", ctypes.c_int, [_vp, ctypes.POINTER(_u64), ctypes.POINTER(_u64),
+                                                               ctypes.POINTER(_u64), ctypes.POINTER(_u64)])
 fleche_debug_locations = _sig("fleche_debug_locations", ctypes.c_int, [_vp, _vp, ctypes.c_size_t])
 
 EXPORTED = ["fleche_create", "fleche_query", "fleche_query_pooled", "fleche_query_host", "fleche_stats",
             "fleche_reset_stats", "fleche_destroy", "fleche_strerror", "fleche_get_encoding", "fleche_get_geometry",
             "fleche_debug_snapshot", "fleche_debug_locations", "fleche_set_profiling", "fleche_kernel_times",
-            "fleche_probe_host_read"]
+            "fleche_probe_host_read", "fleche_route", "fleche_query_keys", "fleche_restore", "fleche_shard_stats"]
 
 
 def probe_host_read(host_ptr: int, nbytes: int, row_bytes: int, rows: int, seed: int = 1, stream=None) -> float:
@@ -173,6 +178,28 @@ class FlatCache:
         ip = (_vp * self.n)(*[_ptr(x) for x in ids])
         op = (_vp * self.n)(*[_ptr(o) for o in offsets])
         _check(fleche_query_pooled(self.h, ip, op, bp, npp, _ptr(out), _stream_handle(stream)), "fleche_query_pooled")
+
+    # ---- key-sharded building blocks (see include/fleche.h and sharded.py)
+    def route(self, ids, world, owner_seed, send_keys, send_counts, stream=None, lengths=None):
+        if lengths is None:
+            lengths = [int(x.numel()) for x in ids]
+        lp = (_i64 * self.n)(*lengths)
+        ip = (_vp * self.n)(*[_ptr(x) for x in ids])
+        _check(fleche_route(self.h, ip, lp, int(world), int(owner_seed), _ptr(send_keys), _ptr(send_counts),
+                            _stream_handle(stream)), "fleche_route")
+
+    def query_keys(self, keys, count, rows, hit_flags=None, stream=None):
+        _check(fleche_query_keys(self.h, _ptr(keys), int(count), _ptr(rows), _ptr(hit_flags), _stream_handle(stream)),
+               "fleche_query_keys")
+
+    def restore(self, rows, hit_flags, out, stream=None):
+        _check(fleche_restore(self.h, _ptr(rows), _ptr(hit_flags), _ptr(out), _stream_handle(stream)),
+               "fleche_restore")
+
+    def shard_stats(self) -> dict:
+        v = [_u64() for _ in range(4)]
+        _check(fleche_shard_stats(self.h, *[ctypes.byref(x) for x in v]), "fleche_shard_stats")
+        return dict(zip(["lookups", "hits", "invalid", "unique_routed"], [int(x.value) for x in v]))
 
     def locations(self):
         sets, _, _ = self.geometry()

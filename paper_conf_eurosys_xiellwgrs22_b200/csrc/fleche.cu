@@ -16,6 +16,7 @@
 
 #include "fleche.h"
 #include "kernels.cuh"
+#include "shard.cuh"
 
 using namespace fl;
 
@@ -58,6 +59,12 @@ struct fleche_ctx {
   std::vector<cudaEvent_t> ev_pool;  // 3 or 4 per profiled query
   std::vector<int> ev_kinds;         // events recorded per profiled query (3 = one-hot, 4 = pooled)
   size_t ev_used = 0;
+  // key-sharded mode (lazy): routing state and the last routed batch's geometry
+  uint64_t* d_kdec = nullptr;
+  RouteDev rd{};
+  bool rd_ready = false;
+  uint32_t repoch = 0;
+  std::vector<int64_t> route_len;
 };
 
 namespace {
@@ -159,7 +166,8 @@ void free_all(fleche_ctx* c) {
   void* ptrs[] = {c->dv.keys, c->dv.ts, c->dv.loc, c->dv.lock, c->dv.slab, c->dv.scratch, c->dv.owner_off,
                   c->dv.firstpos, c->dv.ipos,
                   c->dv.miss, c->dv.dup, c->dv.ctl, c->dv.stats, c->d_tables, c->d_ids_stage, c->d_out_stage,
-                  c->d_pool_stage};
+                  c->d_pool_stage, c->d_kdec, c->rd.scratch, c->rd.slotval, c->rd.inv, c->rd.region, c->rd.cnt,
+                  c->rd.prefix, c->rd.done, c->rd.stats};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   for (auto& r : c->registered) cudaHostUnregister(r.first);
@@ -454,6 +462,15 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   c->index_bytes = ways * (bytes ? 10 : 16) + (bytes ? (size_t)sets * 4 : 0) + (size_t)scr_n * 24 +
                    (size_t)cfg->max_lookups * (sizeof(MissRec) + sizeof(DupRec));
   dv.tables = c->d_tables;
+  {  // flat key -> table decoding table (prefix match of the size-aware code), for key-sharded queries
+    std::vector<uint64_t> kd(n);
+    for (int t = 0; t < n; ++t) kd[t] = (c->base[t] << 16) | (uint64_t)t;
+    std::sort(kd.begin(), kd.end());
+    if (!alloc((void**)&c->d_kdec, 8ull * n) || cudaMemcpy(c->d_kdec, kd.data(), 8ull * n, cudaMemcpyHostToDevice) != cudaSuccess)
+      return fail(FLECHE_ENOMEM);
+    dv.kdec = c->d_kdec;
+    dv.ntables = n;
+  }
   if (cudaMemset(dv.keys, 0xFF, ways * 4) != cudaSuccess || cudaMemset(dv.ts, 0, ways * 4) != cudaSuccess ||
       cudaMemset(dv.scratch, 0, (size_t)scr_n * 8) != cudaSuccess ||
       cudaMemset(dv.stats, 0, sizeof(unsigned long long) * kStripes * kNumCtr) != cudaSuccess)
@@ -722,6 +739,213 @@ fleche_status fleche_probe_host_read(const void* host, uint64_t bytes, int32_t r
   cudaFree(sink);
   if (e != cudaSuccess) return FLECHE_ECUDA;
   *gbps = (double)rows * (double)row_bytes / ((double)ms * 1e-3) / 1e9;
+  return FLECHE_OK;
+}
+
+}  // extern "C"
+
+// ---------------------------------------------------------------- key-sharded mode
+namespace {
+
+template <int MAXT>
+fleche_status launch_keys(fleche_ctx* c, const uint32_t* keys, int64_t count, float* rows, uint8_t* flags,
+                          cudaStream_t s) {
+  QArgs<MAXT> qa;
+  memset(&qa, 0, sizeof(qa));  // out_off[t] = 0: row g of `rows` answers keys[g]
+  qa.n = 1;
+  qa.scan[1] = count;
+  qa.out = rows;
+  qa.fkeys = keys;
+  qa.hit_flags = flags;
+  KMArgs ka;
+  memset(&ka, 0, sizeof(ka));
+  ka.out = rows;
+  ka.ncls = 1;
+  ka.cls_dim[0] = c->max_dim;
+  fleche_status st = prof_event(c, s, true, 3);
+  if (st != FLECHE_OK) return st;
+  if (count > 0) {
+    kq_kernel<MAXT><<<(unsigned)((count + 127) / 128), 128, 0, s>>>(qa, c->dv);
+    c->kernels++;
+  }
+  if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
+  km_kernel<false><<<c->km_blocks, 128, 0, s>>>(c->dv, ka);
+  kd_kernel<<<c->km_blocks, 128, 0, s>>>(c->dv, rows);
+  c->kernels += 2;
+  if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return poison(c, e, "kernel launch");
+  return FLECHE_OK;
+}
+
+template <int MAXT>
+void fill_rargs(fleche_ctx* c, RArgs<MAXT>& ra, const int64_t* const* ids, const int64_t* lengths) {
+  memset(&ra, 0, sizeof(ra));
+  ra.n = c->n;
+  ra.repoch = c->repoch;
+  int64_t acc = 0, oacc = 0;
+  for (int t = 0; t < c->n; ++t) {
+    if (ids) ra.ids[t] = ids[t];
+    ra.scan[t] = acc;
+    ra.out_off[t] = oacc;
+    acc += lengths[t];
+    oacc += lengths[t] * (int64_t)c->dims[t];
+  }
+  ra.scan[c->n] = acc;
+}
+
+template <int MAXT>
+fleche_status launch_route(fleche_ctx* c, const int64_t* const* ids, const int64_t* lengths, int64_t total,
+                           uint32_t* send_keys, int64_t* send_counts, cudaStream_t s) {
+  RArgs<MAXT> ra;
+  fill_rargs<MAXT>(c, ra, ids, lengths);
+  if (total > 0) {
+    kr_kernel<MAXT><<<(unsigned)((total + 127) / 128), 128, 0, s>>>(ra, c->rd, c->d_tables);
+    c->kernels++;
+  }
+  kpk_kernel<<<std::max(1, std::min(2 * c->sm_count, (int)((total + 255) / 256))), 256, 0, s>>>(c->rd, send_keys,
+                                                                                              send_counts);
+  c->kernels++;
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return poison(c, e, "kernel launch");
+  return FLECHE_OK;
+}
+
+template <int MAXT, int D>
+fleche_status launch_restore_d(fleche_ctx* c, const float* rows, const uint8_t* flags, float* out, cudaStream_t s) {
+  RArgs<MAXT> ra;
+  fill_rargs<MAXT>(c, ra, nullptr, c->route_len.data());
+  const int64_t total = ra.scan[c->n];
+  if (total > 0) {
+    krs_kernel<MAXT, D><<<(unsigned)((total + 127) / 128), 128, 0, s>>>(ra, c->rd, rows, flags, out);
+    c->kernels++;
+  }
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return poison(c, e, "kernel launch");
+  return FLECHE_OK;
+}
+
+template <int MAXT>
+fleche_status launch_restore(fleche_ctx* c, const float* rows, const uint8_t* flags, float* out, cudaStream_t s) {
+  switch (c->max_dim) {
+    case 8: return launch_restore_d<MAXT, 8>(c, rows, flags, out, s);
+    case 16: return launch_restore_d<MAXT, 16>(c, rows, flags, out, s);
+    case 32: return launch_restore_d<MAXT, 32>(c, rows, flags, out, s);
+    case 64: return launch_restore_d<MAXT, 64>(c, rows, flags, out, s);
+    case 128: return launch_restore_d<MAXT, 128>(c, rows, flags, out, s);
+    default: return launch_restore_d<MAXT, 256>(c, rows, flags, out, s);
+  }
+}
+
+bool uniform_dims(const fleche_ctx* c) { return c->cls_dim.size() == 1; }
+
+}  // namespace
+
+extern "C" {
+
+fleche_status fleche_route(fleche_ctx* c, const int64_t* const* ids, const int64_t* lengths, int32_t world,
+                           uint32_t owner_seed, uint32_t* send_keys, int64_t* send_counts, fleche_stream stream) {
+  if (!c || !ids || !lengths || !send_keys || !send_counts || world < 1 || world > kMaxWorld) return FLECHE_EINVAL;
+  if (c->poisoned) return FLECHE_ESTATE;
+  if (!uniform_dims(c)) return FLECHE_EINVAL;
+  int64_t total = 0;
+  for (int t = 0; t < c->n; ++t) {
+    if (lengths[t] < 0 || (lengths[t] > 0 && !ids[t])) return FLECHE_EINVAL;
+    total += lengths[t];
+  }
+  if (total > c->max_lookups) return FLECHE_EINVAL;
+  fleche_status st = ensure_device(c);
+  if (st != FLECHE_OK) return st;
+  cudaStream_t s = (cudaStream_t)stream;
+  if (!c->rd_ready || c->rd.world != world) {
+    if (c->rd_ready) FL_CUDA(c, cudaStreamSynchronize(c->last_stream));
+    void* ptrs[] = {c->rd.scratch, c->rd.slotval, c->rd.inv, c->rd.region, c->rd.cnt, c->rd.prefix, c->rd.done,
+                    c->rd.stats};
+    for (void* p : ptrs)
+      if (p) cudaFree(p);
+    const uint32_t scr_n = next_pow2(std::max<uint64_t>(1024, 2ull * (uint64_t)c->max_lookups));
+    RouteDev& rd = c->rd;
+    rd = RouteDev{};
+    rd.mask = scr_n - 1;
+    rd.cap = (uint32_t)c->max_lookups;
+    rd.world = world;
+    rd.owner_seed = owner_seed;
+    FL_CUDA(c, cudaMalloc((void**)&rd.scratch, (size_t)scr_n * 8));
+    FL_CUDA(c, cudaMalloc((void**)&rd.slotval, (size_t)scr_n * 8));
+    FL_CUDA(c, cudaMalloc((void**)&rd.inv, (size_t)c->max_lookups * 4));
+    FL_CUDA(c, cudaMalloc((void**)&rd.region, (size_t)world * c->max_lookups * 4));
+    FL_CUDA(c, cudaMalloc((void**)&rd.cnt, kMaxWorld * 4));
+    FL_CUDA(c, cudaMalloc((void**)&rd.prefix, (kMaxWorld + 1) * 8));
+    FL_CUDA(c, cudaMalloc((void**)&rd.done, 4));
+    FL_CUDA(c, cudaMalloc((void**)&rd.stats, 4 * 8));
+    FL_CUDA(c, cudaMemset(rd.scratch, 0, (size_t)scr_n * 8));
+    FL_CUDA(c, cudaMemset(rd.cnt, 0, kMaxWorld * 4));
+    FL_CUDA(c, cudaMemset(rd.done, 0, 4));
+    FL_CUDA(c, cudaMemset(rd.stats, 0, 32));
+    FL_CUDA(c, cudaDeviceSynchronize());
+    c->rd_ready = true;
+    c->repoch = 0;
+  }
+  c->rd.owner_seed = owner_seed;
+  st = order_on(c, s);
+  if (st != FLECHE_OK) return st;
+  ++c->repoch;
+  c->route_len.assign(lengths, lengths + c->n);
+  if (c->n <= 32) return launch_route<32>(c, ids, lengths, total, send_keys, send_counts, s);
+  if (c->n <= 128) return launch_route<128>(c, ids, lengths, total, send_keys, send_counts, s);
+  return launch_route<FLECHE_MAX_TABLES>(c, ids, lengths, total, send_keys, send_counts, s);
+}
+
+fleche_status fleche_query_keys(fleche_ctx* c, const uint32_t* keys, int64_t count, float* rows, uint8_t* hit_flags,
+                                fleche_stream stream) {
+  if (!c || count < 0 || (count > 0 && (!keys || !rows))) return FLECHE_EINVAL;
+  if (c->poisoned) return FLECHE_ESTATE;
+  if (!uniform_dims(c) || c->dv.part || count > c->max_lookups || ((uintptr_t)rows & 15u)) return FLECHE_EINVAL;
+  fleche_status st = ensure_device(c);
+  if (st != FLECHE_OK) return st;
+  cudaStream_t s = (cudaStream_t)stream;
+  st = order_on(c, s);
+  if (st != FLECHE_OK) return st;
+  if (c->n <= 32) st = launch_keys<32>(c, keys, count, rows, hit_flags, s);
+  else if (c->n <= 128) st = launch_keys<128>(c, keys, count, rows, hit_flags, s);
+  else st = launch_keys<FLECHE_MAX_TABLES>(c, keys, count, rows, hit_flags, s);
+  if (st == FLECHE_OK) {
+    c->batches++;
+    c->lookups += (uint64_t)count;
+  }
+  return st;
+}
+
+fleche_status fleche_restore(fleche_ctx* c, const float* rows, const uint8_t* hit_flags, float* out,
+                             fleche_stream stream) {
+  if (!c || !out || ((uintptr_t)out & 15u)) return FLECHE_EINVAL;
+  if (c->poisoned) return FLECHE_ESTATE;
+  if (!c->rd_ready) return FLECHE_EINVAL;
+  fleche_status st = ensure_device(c);
+  if (st != FLECHE_OK) return st;
+  cudaStream_t s = (cudaStream_t)stream;
+  st = order_on(c, s);
+  if (st != FLECHE_OK) return st;
+  if (c->n <= 32) return launch_restore<32>(c, rows, hit_flags, out, s);
+  if (c->n <= 128) return launch_restore<128>(c, rows, hit_flags, out, s);
+  return launch_restore<FLECHE_MAX_TABLES>(c, rows, hit_flags, out, s);
+}
+
+fleche_status fleche_shard_stats(fleche_ctx* c, uint64_t* lookups, uint64_t* hits, uint64_t* invalid,
+                                 uint64_t* unique_routed) {
+  if (!c) return FLECHE_EINVAL;
+  if (c->poisoned) return FLECHE_ESTATE;
+  unsigned long long v[4] = {0, 0, 0, 0};
+  if (c->rd_ready) {
+    fleche_status st = ensure_device(c);
+    if (st != FLECHE_OK) return st;
+    if (c->have_last) FL_CUDA(c, cudaStreamSynchronize(c->last_stream));
+    FL_CUDA(c, cudaMemcpy(v, c->rd.stats, sizeof(v), cudaMemcpyDeviceToHost));
+  }
+  if (lookups) *lookups = v[0];
+  if (hits) *hits = v[1];
+  if (invalid) *invalid = v[2];
+  if (unique_routed) *unique_routed = v[3];
   return FLECHE_OK;
 }
 

@@ -116,7 +116,8 @@ struct Dev {
   int32_t bytes;     // 0 = uniform layout, 1 = bytes layout
   uint32_t set_units;  // bytes layout: region of a set in 32 B units (<= 256)
   int32_t part;      // static per-table partitions (HugeCTR-like baseline, NEXT-1)
-  int32_t t0;        // unused padding slot
+  int32_t ntables;
+  const uint64_t* kdec;  // [ntables] (base_t << 16 | t) sorted by base: flat key -> table
 #ifdef FLECHE_EXPERIMENTS
   int32_t exp_mode;  // timing experiments only (libfleche_exp.so); breaks semantics
   int32_t exp_pad;
@@ -131,6 +132,8 @@ struct QArgs {
   int64_t cls_off[8];        // start of each class's region of the miss list
   float* out;
   int64_t g0;                // batch position of this launch's first lookup (per-table launches)
+  const uint32_t* fkeys;     // key-sharded owner side: flat keys instead of per-table IDs
+  uint8_t* hit_flags;        // optional per-lookup hit flags (key-sharded)
   int32_t n;
   int32_t t0;                // first table of this launch (per-table launches: t0 = t, n = 1)
 };
@@ -352,17 +355,32 @@ __global__ void __launch_bounds__(128) kq_kernel(const __grid_constant__ QArgs<M
 
     // A1 self-identification: largest t with scan[t] <= g (reading R14)
     int t = 0;
-    if (active) {
-      int lo = 0, hi = qa.n;
+    int64_t j = 0, id = -1;
+    if (!qa.fkeys) {
+      if (active) {
+        int lo = 0, hi = qa.n;
+        while (hi - lo > 1) {
+          const int mid = (lo + hi) >> 1;
+          if (s_scan[mid] <= g) lo = mid; else hi = mid;
+        }
+        t = lo;
+      }
+      j = g - s_scan[t];
+      if (active) id = qa.ids[t][j];
+    } else if (active) {
+      // key-sharded owner side: lookups arrive as flat keys; decode the table by prefix
+      // match (largest base <= fk, the canonical size-aware code) and id = fk - base_t
+      const uint32_t fk0 = qa.fkeys[g];
+      int lo = 0, hi = dv.ntables;
       while (hi - lo > 1) {
         const int mid = (lo + hi) >> 1;
-        if (s_scan[mid] <= g) lo = mid; else hi = mid;
+        if ((uint32_t)(dv.kdec[mid] >> 16) <= fk0) lo = mid; else hi = mid;
       }
-      t = lo;
+      t = (int)(dv.kdec[lo] & 0xFFFFu);
+      id = (int64_t)(fk0 - (uint32_t)(dv.kdec[lo] >> 16));
+      j = g;
     }
-    const int64_t j = g - s_scan[t];
     const TableInfo* ti = dv.tables + qa.t0 + t;
-    const int64_t id = active ? qa.ids[t][j] : -1;
     const int64_t card = ti->card;
     const int d = ti->dim;
 
@@ -467,6 +485,8 @@ __global__ void __launch_bounds__(128) kq_kernel(const __grid_constant__ QArgs<M
       b = __shfl_sync(kFull, b, __ffs(dup_m) - 1);
       if (kind == 2) dv.dup[b + __popc(dup_m & lt)] = DupRec{off, scr, d};  // restored by KD
     }
+
+    if (qa.hit_flags && active) qa.hit_flags[g] = hit ? 1 : 0;  // key-sharded: per-key hit back to requester
 
     // A9 stats, warp-aggregated then block-aggregated
     const unsigned hm = __ballot_sync(kFull, hit), mm = __ballot_sync(kFull, miss);

@@ -88,3 +88,63 @@ def test_replicated_two_ranks_cover_the_global_batch():
                 assert np.array_equal(got[off:off + 64 * d].reshape(64, d), ref)
                 off += 64 * d
     assert not os.path.exists(os.path.join("/dev/shm", name))
+
+
+# ------------------------------------------------------------------ key-sharded plumbing
+def _sharded_worker(rank, world, port, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        from paper_conf_eurosys_xiellwgrs22_b200.sharded import ShardedCache
+        from tests.shard_double import ShardDouble
+        w = configs.get("cfg0").with_(batch_size=40, invalid_ppm=20000)
+        _, tabs = w.make_tables()
+        dbl = ShardDouble(w.cards, w.dims, tabs, max_lookups=w.batch_size * w.n * world)
+        sc = ShardedCache(dbl, row_floats=w.dims[0], device=torch.device("cpu"))
+        res = []
+        for b in range(3):
+            bt = w.batch(b, rank=rank)
+            out = torch.zeros(sum(x.size * d for x, d in zip(bt.ids, w.dims)))
+            ex = sc.query([torch.from_numpy(x) for x in bt.ids], out)
+            res.append((out.numpy().tolist(), ex))
+        gathered = [None] * world
+        dist.all_gather_object(gathered, res)
+        if rank == 0:
+            q.put(gathered)
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.timeout(300)
+def test_sharded_plumbing_two_ranks():
+    # ranks exchange keys and rows with all-to-alls (gloo here, NCCL on GPUs); every
+    # rank's output must be the plain definition for its own shard of the batch, and the
+    # keys each rank sends must equal the keys the owners receive
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_sharded_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    gathered = q.get(timeout=240)
+    for p in procs:
+        p.join(60)
+        assert p.exitcode == 0
+    w = configs.get("cfg0").with_(batch_size=40, invalid_ppm=20000)
+    _, tabs = w.make_tables()
+    for b in range(3):
+        sent = sum(gathered[r][b][1]["sent_keys"] for r in range(world))
+        recv = sum(gathered[r][b][1]["recv_keys"] for r in range(world))
+        assert sent == recv > 0
+        for r in range(world):
+            got = np.array(gathered[r][b][0], np.float32)
+            bt = w.batch(b, rank=r)
+            off = 0
+            for t, ids in enumerate(bt.ids):
+                d = w.dims[t]
+                ref = np.zeros((ids.size, d), np.float32)
+                ok = (ids >= 0) & (ids < w.cards[t])
+                ref[ok] = tabs[t][ids[ok]]
+                assert np.array_equal(got[off:off + ids.size * d].reshape(ids.size, d), ref)
+                off += ids.size * d

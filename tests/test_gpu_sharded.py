@@ -1,0 +1,89 @@
+"""Key-sharded mode on one B200: the routing kernel's owner grouping, and a one-rank NCCL
+group running the full route -> all-to-all -> owner query -> all-to-all -> restore path
+(needs a GPU; multi-rank plumbing is covered on CPU by tests/test_dist_cpu.py)."""
+import socket
+
+import numpy as np
+import pytest
+
+from oracle import oracle as O
+from tests import harness as H
+from tests.shard_double import owner_of
+from workload import configs
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _need_gpu():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+
+
+def _tables(w):
+    return [np.ascontiguousarray(t) for t in w.make_tables()[1]]
+
+
+@pytest.mark.parametrize("world", [1, 3, 8])
+def test_route_groups_unique_keys_by_owner(world):
+    import paper_conf_eurosys_xiellwgrs22_b200 as fl
+    w = configs.get("cfg0").with_(invalid_ppm=5000)
+    tabs = _tables(w)
+    gpu = fl.FlatCache(w.cards, w.dims, tabs, w.cache_bytes, w.batch_size * w.n, 0, 1.0, 0, H.HASH_SEED)
+    _, base, _ = O.encode(w.cards)
+    seed = 0x2545F491
+    for b in range(3):
+        bt = w.batch(b)
+        ids = [torch.from_numpy(x).cuda() for x in bt.ids]
+        sk = torch.empty(w.batch_size * w.n, dtype=torch.int32, device="cuda")
+        sc = torch.empty(world, dtype=torch.int64, device="cuda")
+        gpu.route(ids, world, seed, sk, sc)
+        torch.cuda.synchronize()
+        counts = sc.cpu().numpy()
+        keys = sk[:counts.sum()].cpu().numpy().view(np.uint32).astype(np.int64)
+        ref = set()
+        for t, x in enumerate(bt.ids):
+            ok = (x >= 0) & (x < w.cards[t])
+            ref |= set((int(base[t]) + x[ok]).tolist())
+        assert len(keys) == len(set(keys.tolist())) == len(ref) and set(keys.tolist()) == ref
+        off = 0
+        for o, c in enumerate(counts):
+            assert (owner_of(keys[off:off + c], seed, world) == o).all()
+            off += c
+
+
+def test_sharded_one_rank_nccl_bit_exact_and_exact_hits():
+    import torch.distributed as dist
+
+    import paper_conf_eurosys_xiellwgrs22_b200 as fl
+    from paper_conf_eurosys_xiellwgrs22_b200.sharded import ShardedCache
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    dist.init_process_group("nccl", init_method=f"tcp://127.0.0.1:{port}", rank=0, world_size=1,
+                            device_id=torch.device("cuda", 0))
+    try:
+        w = configs.get("cfg0").with_(cache_frac=0.25, invalid_ppm=3000)
+        tabs = _tables(w)
+        gpu = fl.FlatCache(w.cards, w.dims, tabs, w.cache_bytes, w.batch_size * w.n, 0, 1.0, 0, H.HASH_SEED)
+        sc = ShardedCache(gpu, row_floats=w.dims[0])
+        orc = O.Oracle(w.cards, w.dims, tabs, w.cache_bytes, O.MODE_SETASSOC, hash_seed=H.HASH_SEED)
+        for b in range(20):
+            bt = w.batch(b)
+            ids = [torch.from_numpy(x).cuda() for x in bt.ids]
+            out = torch.full((gpu.out_floats([x.size for x in bt.ids]),), float("nan"), device="cuda")
+            sc.query(ids, out)
+            torch.cuda.synchronize()
+            ref = orc.query(bt.ids)
+            assert H.bits_equal(out.cpu().numpy(), ref), b
+        so, ss, sg = orc.stats(), gpu.shard_stats(), gpu.stats()
+        # one rank owns every key: per-lookup hits, unique keys, inserts equal the oracle's
+        assert ss["hits"] == so["hits"] and ss["invalid"] == so["invalid"] and ss["lookups"] == so["lookups"]
+        assert ss["unique_routed"] == so["unique_keys"] == sg["lookups"]
+        for k in ("unique_hits", "unique_misses", "inserted", "evicted"):
+            assert sg[k] == so[k], k
+    finally:
+        dist.destroy_process_group()
