@@ -229,6 +229,9 @@ fleche_status fleche_shard_stats(fleche_ctx* ctx, uint64_t* lookups, uint64_t* h
  *   with CUDA events on `stream`; *gbps = rows * row_bytes / time.  Blocking. */
 fleche_status fleche_set_profiling(fleche_ctx* ctx, int enable);
 fleche_status fleche_kernel_times(fleche_ctx* ctx, double* kq_ms, double* ki_ms, uint64_t* queries);
+/* Same accumulation split per kernel: ms4 = {query (KQ), miss (KM), restore (KD),
+ * pooling (KP; 0 for one-hot)} summed over the profiled queries; resets. */
+fleche_status fleche_kernel_times_ex(fleche_ctx* ctx, double* ms4, uint64_t* queries);
 fleche_status fleche_probe_host_read(const void* host, uint64_t bytes, int32_t row_bytes, int64_t rows, uint64_t seed,
                                      fleche_stream stream, double* gbps);
 

@@ -64,6 +64,7 @@ fleche_set_profiling = _sig("fleche_set_profiling", ctypes.c_int, [_vp, ctypes.c
 fleche_kernel_times = _sig("fleche_kernel_times", ctypes.c_int, [_vp, ctypes.POINTER(ctypes.c_double),
                                                                  ctypes.POINTER(ctypes.c_double),
                                                                  ctypes.POINTER(_u64)])
+fleche_kernel_times_ex = _sig("fleche_kernel_times_ex", ctypes.c_int, [_vp, _vp, ctypes.POINTER(_u64)])
 fleche_probe_host_read = _sig("fleche_probe_host_read", ctypes.c_int, [_vp, _u64, _i32, _i64, _u64, _vp,
                                                                        ctypes.POINTER(ctypes.c_double)])
 
@@ -78,7 +79,8 @@ fleche_debug_locations = _sig("fleche_debug_locations", ctypes.c_int, [_vp, _vp,
 EXPORTED = ["fleche_create", "fleche_query", "fleche_query_pooled", "fleche_query_host", "fleche_stats",
             "fleche_reset_stats", "fleche_destroy", "fleche_strerror", "fleche_get_encoding", "fleche_get_geometry",
             "fleche_debug_snapshot", "fleche_debug_locations", "fleche_set_profiling", "fleche_kernel_times",
-            "fleche_probe_host_read", "fleche_route", "fleche_query_keys", "fleche_restore", "fleche_shard_stats"]
+            "fleche_probe_host_read", "fleche_route", "fleche_query_keys", "fleche_restore", "fleche_shard_stats",
+            "fleche_kernel_times_ex"]
 
 
 def probe_host_read(host_ptr: int, nbytes: int, row_bytes: int, rows: int, seed: int = 1, stream=None) -> float:
@@ -228,6 +230,13 @@ class FlatCache:
 
     def set_profiling(self, on: bool):
         _check(fleche_set_profiling(self.h, 1 if on else 0), "fleche_set_profiling")
+
+    def kernel_times_ex(self):
+        """({'kq','km','kd','kp'} ms totals, profiled queries) since the last call."""
+        ms = (ctypes.c_double * 4)()
+        q = _u64()
+        _check(fleche_kernel_times_ex(self.h, ms, ctypes.byref(q)), "fleche_kernel_times_ex")
+        return dict(zip(["kq", "km", "kd", "kp"], [float(x) for x in ms])), int(q.value)
 
     def kernel_times(self):
         """(KQ ms total, KI ms total, profiled queries) since the last call."""

@@ -41,6 +41,7 @@ struct fleche_ctx {
   TableInfo* d_tables = nullptr;
   int km_blocks = 0;
   int km_bps = 4;  // KM CTAs per SM
+  int kd_blocks = 0;
   bool per_table_launch = false;
   size_t km_smem = 0;
   // host-side counters
@@ -206,6 +207,25 @@ fleche_status prof_event(fleche_ctx* c, cudaStream_t s, bool first, int kinds) {
   return FLECHE_OK;
 }
 
+// Launch with programmatic stream serialization (PDL): the kernel's launch and prologue
+// overlap its predecessor's tail; the kernel's pdl_wait() orders its dependent work.
+bool g_pdl = getenv("FLECHE_NO_PDL") == nullptr;
+template <typename... KArgs, typename... Args>
+cudaError_t launch_k(void (*kern)(KArgs...), unsigned grid, unsigned block, size_t smem, cudaStream_t s,
+                     Args&&... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(block);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = g_pdl ? 1 : 0;
+  return cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
+}
+
 // KQ + KM for one batch of one-hot lookups into `out` (table-major rows).
 template <int MAXT>
 fleche_status launch_query(fleche_ctx* c, const int64_t* const* ids, const int64_t* lengths, float* out,
@@ -239,7 +259,7 @@ fleche_status launch_query(fleche_ctx* c, const int64_t* const* ids, const int64
   if (st != FLECHE_OK) return st;
   if (total > 0 && !c->per_table_launch) {
     const int64_t blocks = (total + 127) / 128;
-    kq_kernel<MAXT><<<(unsigned)blocks, 128, 0, s>>>(qa, c->dv);
+    launch_k(kq_kernel<MAXT>, (unsigned)blocks, 128, 0, s, qa, c->dv);
     c->kernels++;
   } else if (total > 0) {  // ablation: one query launch per table (n launches)
     QArgs<32> q1;
@@ -255,14 +275,15 @@ fleche_status launch_query(fleche_ctx* c, const int64_t* const* ids, const int64
       q1.scan[0] = 0;
       q1.scan[1] = lengths[t];
       q1.out_off[0] = qa.out_off[t];
-      kq_kernel<32><<<(unsigned)((lengths[t] + 127) / 128), 128, 0, s>>>(q1, c->dv);
+      launch_k(kq_kernel<32>, (unsigned)((lengths[t] + 127) / 128), 128, 0, s, q1, c->dv);
       c->kernels++;
     }
   }
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
-  if (c->dv.bytes) km_kernel<true><<<c->km_blocks, 128, c->km_smem, s>>>(c->dv, ka);
-  else km_kernel<false><<<c->km_blocks, 128, 0, s>>>(c->dv, ka);
-  kd_kernel<<<c->km_blocks, 128, 0, s>>>(c->dv, out);
+  if (c->dv.bytes) launch_k(km_kernel<true>, c->km_blocks, 128, c->km_smem, s, c->dv, ka);
+  else launch_k(km_kernel<false>, c->km_blocks, 128, 0, s, c->dv, ka);
+  if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
+  launch_k(kd_kernel, c->kd_blocks, 128, 0, s, c->dv, out);
   c->kernels += 2;
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
   cudaError_t e = cudaGetLastError();
@@ -271,7 +292,7 @@ fleche_status launch_query(fleche_ctx* c, const int64_t* const* ids, const int64
 }
 
 fleche_status query_impl(fleche_ctx* c, const int64_t* const* ids, const int64_t* lengths, float* out,
-                         cudaStream_t s, int nev = 3) {
+                         cudaStream_t s, int nev = 4) {
   int64_t total = 0;
   for (int t = 0; t < c->n; ++t) {
     if (lengths[t] < 0) return FLECHE_EINVAL;
@@ -314,7 +335,7 @@ fleche_status launch_pool(fleche_ctx* c, const int64_t* const* offsets, const in
   }
   pa.cscan[c->n] = cs;
   if (cs > 0) {
-    kp_kernel<MAXT><<<(unsigned)((cs + 255) / 256), 256, 0, s>>>(pa, c->d_tables);
+    launch_k(kp_kernel<MAXT>, (unsigned)((cs + 255) / 256), 256, 0, s, pa, (const TableInfo*)c->d_tables);
     c->kernels++;
   }
   fleche_status st = prof_event(c, s, false, 0);
@@ -496,6 +517,7 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   c->km_blocks = (int)std::min<int64_t>((int64_t)c->km_bps * c->sm_count,
                                         std::max<int64_t>(1, (cfg->max_lookups + 255) / 256));
   c->km_smem = bytes ? (size_t)kKmWarps * kKmSmemF4 * sizeof(float4) : 0;
+  c->kd_blocks = std::max(1, std::min(c->km_blocks, c->sm_count));  // one wave: duplicates are few
   if (cudaDeviceSynchronize() != cudaSuccess) return fail(FLECHE_ECUDA);
   *out = c;
   return FLECHE_OK;
@@ -523,7 +545,7 @@ fleche_status fleche_query_pooled(fleche_ctx* c, const int64_t* const* ids, cons
   if (!c->d_pool_stage) FL_CUDA(c, cudaMalloc((void**)&c->d_pool_stage, (size_t)c->max_lookups * c->max_dim * 4));
   cudaStream_t s = (cudaStream_t)stream;
   // one-hot lookups of every ID into the staging rows (A1-A8), then bag sums (KP)
-  st = query_impl(c, ids, nnz, c->d_pool_stage, s, 4);
+  st = query_impl(c, ids, nnz, c->d_pool_stage, s, 5);
   if (st != FLECHE_OK) return st;
   if (c->n <= 32) return launch_pool<32>(c, offsets, bags, nnz, out, s);
   if (c->n <= 128) return launch_pool<128>(c, offsets, bags, nnz, out, s);
@@ -683,25 +705,34 @@ fleche_status fleche_set_profiling(fleche_ctx* c, int enable) {
   return FLECHE_OK;
 }
 
-fleche_status fleche_kernel_times(fleche_ctx* c, double* kq_ms, double* ki_ms, uint64_t* queries) {
+fleche_status fleche_kernel_times_ex(fleche_ctx* c, double* ms4, uint64_t* queries) {
   if (!c) return FLECHE_EINVAL;
   if (c->poisoned) return FLECHE_ESTATE;
-  double a = 0, b = 0;
+  double acc[4] = {0, 0, 0, 0};
   size_t i = 0;
-  for (int k : c->ev_kinds) {  // events: [start, after KQ, after KM (, after KP)]
-    float x = 0, y = 0;
+  for (int k : c->ev_kinds) {  // events: [start, after KQ, after KM, after KD (, after KP)]
     FL_CUDA(c, cudaEventSynchronize(c->ev_pool[i + k - 1]));
-    FL_CUDA(c, cudaEventElapsedTime(&x, c->ev_pool[i], c->ev_pool[i + 1]));
-    FL_CUDA(c, cudaEventElapsedTime(&y, c->ev_pool[i + 1], c->ev_pool[i + k - 1]));
-    a += x;
-    b += y;
+    for (int j = 0; j + 1 < k; ++j) {
+      float x = 0;
+      FL_CUDA(c, cudaEventElapsedTime(&x, c->ev_pool[i + j], c->ev_pool[i + j + 1]));
+      acc[j] += x;
+    }
     i += k;
   }
-  if (kq_ms) *kq_ms = a;
-  if (ki_ms) *ki_ms = b;
+  if (ms4)
+    for (int j = 0; j < 4; ++j) ms4[j] = acc[j];
   if (queries) *queries = c->ev_kinds.size();
   c->ev_used = 0;
   c->ev_kinds.clear();
+  return FLECHE_OK;
+}
+
+fleche_status fleche_kernel_times(fleche_ctx* c, double* kq_ms, double* ki_ms, uint64_t* queries) {
+  double ms4[4];
+  fleche_status st = fleche_kernel_times_ex(c, ms4, queries);
+  if (st != FLECHE_OK) return st;
+  if (kq_ms) *kq_ms = ms4[0];
+  if (ki_ms) *ki_ms = ms4[1] + ms4[2] + ms4[3];
   return FLECHE_OK;
 }
 
@@ -762,15 +793,16 @@ fleche_status launch_keys(fleche_ctx* c, const uint32_t* keys, int64_t count, fl
   ka.out = rows;
   ka.ncls = 1;
   ka.cls_dim[0] = c->max_dim;
-  fleche_status st = prof_event(c, s, true, 3);
+  fleche_status st = prof_event(c, s, true, 4);
   if (st != FLECHE_OK) return st;
   if (count > 0) {
-    kq_kernel<MAXT><<<(unsigned)((count + 127) / 128), 128, 0, s>>>(qa, c->dv);
+    launch_k(kq_kernel<MAXT>, (unsigned)((count + 127) / 128), 128, 0, s, qa, c->dv);
     c->kernels++;
   }
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
-  km_kernel<false><<<c->km_blocks, 128, 0, s>>>(c->dv, ka);
-  kd_kernel<<<c->km_blocks, 128, 0, s>>>(c->dv, rows);
+  launch_k(km_kernel<false>, c->km_blocks, 128, 0, s, c->dv, ka);
+  if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
+  launch_k(kd_kernel, c->kd_blocks, 128, 0, s, c->dv, rows);
   c->kernels += 2;
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
   cudaError_t e = cudaGetLastError();

@@ -233,6 +233,13 @@ __device__ __forceinline__ unsigned long long ld_cg_u64(const unsigned long long
 __device__ __forceinline__ void st_v4(float* p, float4 v) {
   asm volatile("st.global.v4.f32 [%0], {%1,%2,%3,%4};" ::"l"(p), "f"(v.x), "f"(v.y), "f"(v.z), "f"(v.w) : "memory");
 }
+// Programmatic dependent launch (sm_90+): the batch's kernels are launched with
+// programmatic stream serialization, so a kernel's launch and prologue overlap the tail
+// of its predecessor; pdl_wait() (griddepcontrol.wait) then blocks until the
+// predecessor grid has completed and its writes are visible.  No-ops otherwise.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
 __device__ __forceinline__ unsigned long long warp_min_u64(unsigned long long x) {
 #pragma unroll
   for (int o = 16; o; o >>= 1) {
@@ -344,6 +351,7 @@ __global__ void __launch_bounds__(128) kq_kernel(const __grid_constant__ QArgs<M
   __shared__ unsigned long long s_ctr[kNumCtr];
   for (int i = threadIdx.x; i <= qa.n; i += blockDim.x) s_scan[i] = qa.scan[i];
   if (threadIdx.x < kNumCtr) s_ctr[threadIdx.x] = 0;
+  pdl_wait();  // the previous batch (or the caller's producer of ids) has completed
   __syncthreads();
 
   const int lane = threadIdx.x & 31;
@@ -503,6 +511,7 @@ __global__ void __launch_bounds__(128) kq_kernel(const __grid_constant__ QArgs<M
       if (dup_m) atomicAdd(&s_ctr[C_DUPS], (unsigned long long)__popc(dup_m));
     }
   }
+  pdl_trigger();  // KM may be scheduled now; its pdl_wait still waits for this grid
   __syncthreads();
   if (threadIdx.x < kNumCtr && s_ctr[threadIdx.x])
     atomicAdd(dv.stats + (blockIdx.x % kStripes) * kNumCtr + threadIdx.x, s_ctr[threadIdx.x]);
@@ -758,6 +767,7 @@ __global__ void __launch_bounds__(128, 4) km_kernel(const __grid_constant__ Dev 
   extern __shared__ float4 s_dyn[];
   if (threadIdx.x < kNumCtr) s_ctr[threadIdx.x] = 0;
   __syncthreads();
+  pdl_wait();  // KQ has completed: miss lists and owner rows are final
   const uint32_t epoch = *(volatile uint32_t*)&dv.ctl->epoch;
   const int par = epoch & 1u;
   const int lane = threadIdx.x & 31;
@@ -811,13 +821,26 @@ __global__ void __launch_bounds__(128, 4) km_kernel(const __grid_constant__ Dev 
   __syncthreads();
   if (threadIdx.x < kNumCtr && s_ctr[threadIdx.x])
     atomicAdd(dv.stats + (blockIdx.x % kStripes) * kNumCtr + threadIdx.x, s_ctr[threadIdx.x]);
+  pdl_trigger();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    const uint32_t prev = atomicAdd(&dv.ctl->done, 1u);
+    if (prev == gridDim.x - 1) {  // last CTA closes the batch: next batch's counters, epoch + 1
+#pragma unroll
+      for (int c = 0; c < 8; ++c) dv.ctl->counts[par ^ 1][c] = 0;
+      dv.ctl->done = 0;
+      __threadfence();
+      *(volatile uint32_t*)&dv.ctl->epoch = epoch + 1u;
+    }
+  }
 }
 
 // KD restore: every duplicate occurrence of a missed key copies its owner's
-// row (written by KM) in parallel; then the last CTA closes the batch: resets the next
-// batch's counters and advances the device-resident epoch (graph-replay safe).
+// row (written by KM) in parallel.
 __global__ void __launch_bounds__(128) kd_kernel(const __grid_constant__ Dev dv, float* __restrict__ out) {
-  const uint32_t epoch = *(volatile uint32_t*)&dv.ctl->epoch;
+  pdl_wait();
+  // KM's last CTA already advanced the epoch: this batch is epoch - 1
+  const uint32_t epoch = *(volatile uint32_t*)&dv.ctl->epoch - 1u;
   const int par = epoch & 1u;
   const uint32_t ndup = *(volatile uint32_t*)&dv.ctl->counts[par][kDupSlot];
   const int lane = threadIdx.x & 31;
@@ -828,18 +851,7 @@ __global__ void __launch_bounds__(128) kd_kernel(const __grid_constant__ Dev dv,
     const float* src = out + dv.owner_off[r.scr];
     for (int c = lane; c < r.dim / 4; c += 32) st_v4(out + r.off + 4 * c, ld_cg_v4(src + 4 * c));
   }
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    __threadfence();
-    const uint32_t prev = atomicAdd(&dv.ctl->done, 1u);
-    if (prev == gridDim.x - 1) {  // last CTA: reset next batch's counters, advance the epoch
-#pragma unroll
-      for (int c = 0; c < 8; ++c) dv.ctl->counts[par ^ 1][c] = 0;
-      dv.ctl->done = 0;
-      __threadfence();
-      *(volatile uint32_t*)&dv.ctl->epoch = epoch + 1u;
-    }
-  }
+  pdl_trigger();
 }
 
 // Pooling: one thread per (bag, 4-float column); sums the bag's staged
@@ -850,6 +862,8 @@ __global__ void __launch_bounds__(256) kp_kernel(const __grid_constant__ PArgs<M
   __shared__ int64_t s_scan[MAXT + 1];
   for (int i = threadIdx.x; i <= pa.n; i += blockDim.x) s_scan[i] = pa.cscan[i];
   __syncthreads();
+  pdl_wait();
+  pdl_trigger();
   const int64_t g = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (g >= s_scan[pa.n]) return;
   int lo = 0, hi = pa.n;

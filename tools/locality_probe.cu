@@ -1,7 +1,7 @@
-// tools/locality_probe.cu — is the large-span zero-copy read rate limited per 2 MiB
-// page translation?  Random 256 B rows from a mapped pinned host buffer, where each
-// group of k consecutive lanes draws rows from the SAME 2 MiB page (k = 1: uniform).
-// If the rate in rows/s scales with k at large spans, grouping misses by page pays.
+// tools/locality_probe.cu — what limits random-row zero-copy reads at large spans?
+// Random 256 B rows from a mapped pinned host buffer, where each group of k consecutive
+// lanes draws rows from the SAME page of 2^shift bytes (k = 1: uniform).  If the rows/s
+// rate scales with k for some page size, one translation per such page is the limiter.
 #include <cuda_runtime.h>
 
 #include <cstdio>
@@ -27,27 +27,28 @@ int main() {
   float* sink;
   cudaMalloc(&sink, 4096 * 512);
   printf("{");
-  for (size_t span : {1ull << 30, 8ull << 30, 32ull << 30}) {
+  for (size_t span : {1ull << 30, 8ull << 30}) {
     void* h;
     if (cudaHostAlloc(&h, span, cudaHostAllocMapped) != cudaSuccess) continue;
     cudaMemset(h, 1, span);
     void* d;
     cudaHostGetDevicePointer(&d, h, 0);
-    const uint64_t rpp = (2u << 20) / 256, pages = span >> 21;
-    for (int k : {1, 2, 4, 8, 32}) {
-      const int64_t rows = 1 << 20;
-      cudaEvent_t a, b;
-      cudaEventCreate(&a);
-      cudaEventCreate(&b);
-      grouped_probe<64><<<(rows + 127) / 128, 128>>>((const float*)d, pages, rpp, rows, k, 3, sink);
-      cudaEventRecord(a);
-      grouped_probe<64><<<(rows + 127) / 128, 128>>>((const float*)d, pages, rpp, rows, k, 5, sink);
-      cudaEventRecord(b);
-      cudaEventSynchronize(b);
-      float ms;
-      cudaEventElapsedTime(&ms, a, b);
-      printf("\"span%zuG_k%d_gbs\": %.2f, \"span%zuG_k%d_Mrows\": %.1f, ", span >> 30, k, rows * 256.0 / (ms * 1e6),
-             span >> 30, k, rows / (ms * 1e3));
+    for (int shift : {21, 16, 12}) {
+      const uint64_t rpp = (1ull << shift) / 256, pages = span >> shift;
+      for (int k : {1, 4, 16}) {
+        const int64_t rows = 1 << 20;
+        cudaEvent_t a, b;
+        cudaEventCreate(&a);
+        cudaEventCreate(&b);
+        grouped_probe<64><<<(rows + 127) / 128, 128>>>((const float*)d, pages, rpp, rows, k, 3, sink);
+        cudaEventRecord(a);
+        grouped_probe<64><<<(rows + 127) / 128, 128>>>((const float*)d, pages, rpp, rows, k, 5, sink);
+        cudaEventRecord(b);
+        cudaEventSynchronize(b);
+        float ms;
+        cudaEventElapsedTime(&ms, a, b);
+        printf("\"span%zuG_page2^%d_k%d_Mrows\": %.1f, ", span >> 30, shift, k, rows / (ms * 1e3));
+      }
     }
     cudaFreeHost(h);
     fflush(stdout);
