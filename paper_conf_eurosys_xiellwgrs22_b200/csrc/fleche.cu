@@ -518,6 +518,10 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
                                         std::max<int64_t>(1, (cfg->max_lookups + 255) / 256));
   c->km_smem = bytes ? (size_t)kKmWarps * kKmSmemF4 * sizeof(float4) : 0;
   c->kd_blocks = std::max(1, std::min(c->km_blocks, c->sm_count));  // one wave: duplicates are few
+#ifdef FLECHE_EXPERIMENTS
+  if (cudaMalloc((void**)&dv.exp_buf, (size_t)c->km_blocks * 4 * 4 * 8) != cudaSuccess) return fail(FLECHE_ENOMEM);
+  cudaMemset(dv.exp_buf, 0, (size_t)c->km_blocks * 4 * 4 * 8);
+#endif
   if (cudaDeviceSynchronize() != cudaSuccess) return fail(FLECHE_ECUDA);
   *out = c;
   return FLECHE_OK;
@@ -982,3 +986,14 @@ fleche_status fleche_shard_stats(fleche_ctx* c, uint64_t* lookups, uint64_t* hit
 }
 
 }  // extern "C"
+
+#ifdef FLECHE_EXPERIMENTS
+// timing experiments only: per-KM-warp globaltimer stamps of the last query
+extern "C" __attribute__((visibility("default"))) fleche_status fleche_exp_timeline(fleche_ctx* c, uint64_t* host,
+                                                                                    size_t n) {
+  if (!c || !host) return FLECHE_EINVAL;
+  if (c->have_last) cudaStreamSynchronize(c->last_stream);
+  const size_t m = std::min(n, (size_t)c->km_blocks * 16);
+  return cudaMemcpy(host, c->dv.exp_buf, m * 8, cudaMemcpyDeviceToHost) == cudaSuccess ? FLECHE_OK : FLECHE_ECUDA;
+}
+#endif

@@ -121,6 +121,7 @@ struct Dev {
 #ifdef FLECHE_EXPERIMENTS
   int32_t exp_mode;  // timing experiments only (libfleche_exp.so); breaks semantics
   int32_t exp_pad;
+  unsigned long long* exp_buf;  // per KM warp: globaltimer at start / rows landed / end
 #endif
 };
 
@@ -681,6 +682,14 @@ __device__ __forceinline__ void km_rows(const Dev& dv, float* __restrict__ out, 
                                         uint32_t epoch, uint32_t nmiss, int lane, uint32_t gw, uint32_t nw,
                                         unsigned& ins, unsigned& ev, unsigned& byp, long long& docc,
                                         unsigned long long& hostb, float4* wsm) {
+#ifdef FLECHE_EXPERIMENTS
+  if (dv.exp_buf && lane == 0) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    dv.exp_buf[gw * 4 + 0] = t;
+    dv.exp_buf[gw * 4 + 1] = 0;
+  }
+#endif
   for (uint32_t base = gw * M; base < nmiss; base += nw * M) {
     const uint32_t k = base + lane;
     bool has = lane < M && k < nmiss;
@@ -705,8 +714,8 @@ __device__ __forceinline__ void km_rows(const Dev& dv, float* __restrict__ out, 
       hostb += 4ull * D;
     }
     if constexpr (!BYTES) {
-      // A7 while the loads are in flight: victim claim (L2 round trips only)
-      rb.store(has ? out + m.off : nullptr, lane);
+      // A7 while the loads are in flight: victim claim (L2 round trips only); the first
+      // use of the loaded rows (the slab store) comes after this round's claims
       bool pending = has && admit;
       if (has && !admit) ++byp;
       const TableInfo* ti = dv.tables + (has ? m.t : 0);
@@ -741,6 +750,15 @@ __device__ __forceinline__ void km_rows(const Dev& dv, float* __restrict__ out, 
         }
         if (slot == kClaimRetry && pending) __nanosleep(100);
       }
+      rb.store(has ? out + m.off : nullptr, lane);  // the owner's output row
+#ifdef FLECHE_EXPERIMENTS
+      if (dv.exp_buf && lane == 0 && base == gw * M) {
+        unsigned long long t;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+        dv.exp_buf[gw * 4 + 1] = t;
+        dv.exp_buf[gw * 4 + 3] = (unsigned long long)__popc(__activemask());
+      }
+#endif
     } else {
       rb.store(has ? out + m.off : nullptr, lane);
       rb.to_smem(wsm, lane);
@@ -758,8 +776,14 @@ __device__ __forceinline__ void km_rows(const Dev& dv, float* __restrict__ out, 
     }
     __syncwarp();
   }
+#ifdef FLECHE_EXPERIMENTS
+  if (dv.exp_buf && lane == 0) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    dv.exp_buf[gw * 4 + 2] = t;
+  }
+#endif
 }
-
 
 template <bool BYTES>
 __global__ void __launch_bounds__(128, 4) km_kernel(const __grid_constant__ Dev dv, const __grid_constant__ KMArgs ka) {
