@@ -209,10 +209,18 @@ fleche_status prof_event(fleche_ctx* c, cudaStream_t s, bool first, int kinds) {
 
 // Launch with programmatic stream serialization (PDL): the kernel's launch and prologue
 // overlap its predecessor's tail; the kernel's pdl_wait() orders its dependent work.
-bool g_pdl = getenv("FLECHE_NO_PDL") == nullptr;
+// Per-kernel PDL mask (bit 0 KQ, 1 KM, 2 KD, 3 KP).  KM is launched without it by default:
+// its blocks would be placed early, during KQ's tail, which measured slower for the
+// address-ordered miss fetch (profiles/README.md).
+enum { kPdlKQ = 0, kPdlKM = 1, kPdlKD = 2, kPdlKP = 3 };
+int pdl_mask() {
+  static const int m = getenv("FLECHE_NO_PDL") ? 0 : (getenv("FLECHE_PDL_MASK") ? atoi(getenv("FLECHE_PDL_MASK")) : 0xD);
+  return m;
+}
 template <typename... KArgs, typename... Args>
-cudaError_t launch_k(void (*kern)(KArgs...), unsigned grid, unsigned block, size_t smem, cudaStream_t s,
+cudaError_t launch_k(int which, void (*kern)(KArgs...), unsigned grid, unsigned block, size_t smem, cudaStream_t s,
                      Args&&... args) {
+  const bool g_pdl = (pdl_mask() >> which) & 1;
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(grid);
   cfg.blockDim = dim3(block);
@@ -259,7 +267,7 @@ fleche_status launch_query(fleche_ctx* c, const int64_t* const* ids, const int64
   if (st != FLECHE_OK) return st;
   if (total > 0 && !c->per_table_launch) {
     const int64_t blocks = (total + 127) / 128;
-    launch_k(kq_kernel<MAXT>, (unsigned)blocks, 128, 0, s, qa, c->dv);
+    launch_k(kPdlKQ, kq_kernel<MAXT>, (unsigned)blocks, 128, 0, s, qa, c->dv);
     c->kernels++;
   } else if (total > 0) {  // ablation: one query launch per table (n launches)
     QArgs<32> q1;
@@ -275,15 +283,15 @@ fleche_status launch_query(fleche_ctx* c, const int64_t* const* ids, const int64
       q1.scan[0] = 0;
       q1.scan[1] = lengths[t];
       q1.out_off[0] = qa.out_off[t];
-      launch_k(kq_kernel<32>, (unsigned)((lengths[t] + 127) / 128), 128, 0, s, q1, c->dv);
+      launch_k(kPdlKQ, kq_kernel<32>, (unsigned)((lengths[t] + 127) / 128), 128, 0, s, q1, c->dv);
       c->kernels++;
     }
   }
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
-  if (c->dv.bytes) launch_k(km_kernel<true>, c->km_blocks, 128, c->km_smem, s, c->dv, ka);
-  else launch_k(km_kernel<false>, c->km_blocks, 128, 0, s, c->dv, ka);
+  if (c->dv.bytes) launch_k(kPdlKM, km_kernel<true>, c->km_blocks, 128, c->km_smem, s, c->dv, ka);
+  else launch_k(kPdlKM, km_kernel<false>, c->km_blocks, 128, 0, s, c->dv, ka);
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
-  launch_k(kd_kernel, c->kd_blocks, 128, 0, s, c->dv, out);
+  launch_k(kPdlKD, kd_kernel, c->kd_blocks, 128, 0, s, c->dv, out);
   c->kernels += 2;
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
   cudaError_t e = cudaGetLastError();
@@ -335,7 +343,7 @@ fleche_status launch_pool(fleche_ctx* c, const int64_t* const* offsets, const in
   }
   pa.cscan[c->n] = cs;
   if (cs > 0) {
-    launch_k(kp_kernel<MAXT>, (unsigned)((cs + 255) / 256), 256, 0, s, pa, (const TableInfo*)c->d_tables);
+    launch_k(kPdlKP, kp_kernel<MAXT>, (unsigned)((cs + 255) / 256), 256, 0, s, pa, (const TableInfo*)c->d_tables);
     c->kernels++;
   }
   fleche_status st = prof_event(c, s, false, 0);
@@ -512,6 +520,22 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
                       p_rows[t], p_slab[t]};
   if (cudaMemcpy(c->d_tables, ti.data(), sizeof(TableInfo) * n, cudaMemcpyHostToDevice) != cudaSuccess)
     return fail(FLECHE_ECUDA);
+  {  // address-ordered miss scratch (uniform layout): slot0 monotone in the host-row address
+    uint64_t lo = ~0ull, hi = 0;
+    for (int t = 0; t < n; ++t) {
+      lo = std::min<uint64_t>(lo, (uint64_t)dptr[t]);
+      hi = std::max<uint64_t>(hi, (uint64_t)dptr[t] + (uint64_t)c->card[t] * (uint64_t)c->dims[t] * 4u);
+    }
+    const uint64_t span = hi - lo;
+    // only worth it when the host tier outgrows the host link's translation reach (~1 GiB
+    // measured, profiles/hostlink_locality_r01.json); below that the scan costs more than it saves
+    uint64_t min_span = 1ull << 30;
+    if (const char* e = getenv("FLECHE_ORDER_MIN_SPAN")) min_span = strtoull(e, nullptr, 10);
+    dv.ordered = (!bytes && !part && span > (uint64_t)scr_n && span >= min_span && getenv("FLECHE_NO_ORDER") == nullptr)
+                     ? 1 : 0;
+    dv.host_lo = lo;
+    dv.host_mul = dv.ordered ? (uint64_t)(((unsigned __int128)scr_n << 64) / span) : 0;
+  }
   if (cudaEventCreateWithFlags(&c->chain_ev, cudaEventDisableTiming) != cudaSuccess) return fail(FLECHE_ECUDA);
   // KM: enough warps for the expected unique misses, km_bps CTAs of 4 warps per SM
   c->km_blocks = (int)std::min<int64_t>((int64_t)c->km_bps * c->sm_count,
@@ -800,13 +824,13 @@ fleche_status launch_keys(fleche_ctx* c, const uint32_t* keys, int64_t count, fl
   fleche_status st = prof_event(c, s, true, 4);
   if (st != FLECHE_OK) return st;
   if (count > 0) {
-    launch_k(kq_kernel<MAXT>, (unsigned)((count + 127) / 128), 128, 0, s, qa, c->dv);
+    launch_k(kPdlKQ, kq_kernel<MAXT>, (unsigned)((count + 127) / 128), 128, 0, s, qa, c->dv);
     c->kernels++;
   }
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
-  launch_k(km_kernel<false>, c->km_blocks, 128, 0, s, c->dv, ka);
+  launch_k(kPdlKM, km_kernel<false>, c->km_blocks, 128, 0, s, c->dv, ka);
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
-  launch_k(kd_kernel, c->kd_blocks, 128, 0, s, c->dv, rows);
+  launch_k(kPdlKD, kd_kernel, c->kd_blocks, 128, 0, s, c->dv, rows);
   c->kernels += 2;
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
   cudaError_t e = cudaGetLastError();

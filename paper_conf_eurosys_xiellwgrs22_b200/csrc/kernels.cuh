@@ -118,6 +118,12 @@ struct Dev {
   int32_t part;      // static per-table partitions (HugeCTR-like baseline, NEXT-1)
   int32_t ntables;
   const uint64_t* kdec;  // [ntables] (base_t << 16 | t) sorted by base: flat key -> table
+  // address-ordered miss scratch (uniform layout): a missed key's first scratch slot is
+  // monotone in its host-row address, slot0 = ((addr - host_lo) * host_mul) >> 64, so KM
+  // can hand each warp a contiguous address window (host-link reads in address order)
+  int32_t ordered;
+  int32_t pad2;
+  uint64_t host_lo, host_mul;
 #ifdef FLECHE_EXPERIMENTS
   int32_t exp_mode;  // timing experiments only (libfleche_exp.so); breaks semantics
   int32_t exp_pad;
@@ -450,7 +456,9 @@ __global__ void __launch_bounds__(128) kq_kernel(const __grid_constant__ QArgs<M
     uint32_t scr = 0;
     if (miss) {
       const unsigned long long tag = ((unsigned long long)epoch << 32) | fk;
-      uint32_t h = scr_hash(fk) & dv.scr_mask;
+      uint32_t h = dv.ordered ? (uint32_t)__umul64hi((uint64_t)(ti->host + (size_t)id * (size_t)d) - dv.host_lo,
+                                                     dv.host_mul) & dv.scr_mask
+                              : scr_hash(fk) & dv.scr_mask;
       unsigned long long cur = ld_cg_u64(dv.scratch + h);
       while (true) {
         if (cur == tag) { kind = 2; break; }
@@ -690,13 +698,11 @@ __device__ __forceinline__ void km_rows(const Dev& dv, float* __restrict__ out, 
     dv.exp_buf[gw * 4 + 1] = 0;
   }
 #endif
-  for (uint32_t base = gw * M; base < nmiss; base += nw * M) {
-    const uint32_t k = base + lane;
-    bool has = lane < M && k < nmiss;
-    MissRec m{};
+  bool first_chunk = true;
+  // one chunk of up to M unique misses (lane r < M holds miss r)
+  auto chunk = [&](bool has, MissRec m) {
     const float* src = nullptr;
     if (has) {
-      m = mlist[k];
       const TableInfo* ti = dv.tables + m.t;
       src = ti->host + (size_t)(m.fk - ti->base) * D;  // unified index: computed host address
     }
@@ -752,7 +758,7 @@ __device__ __forceinline__ void km_rows(const Dev& dv, float* __restrict__ out, 
       }
       rb.store(has ? out + m.off : nullptr, lane);  // the owner's output row
 #ifdef FLECHE_EXPERIMENTS
-      if (dv.exp_buf && lane == 0 && base == gw * M) {
+      if (dv.exp_buf && lane == 0 && first_chunk) {
         unsigned long long t;
         asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
         dv.exp_buf[gw * 4 + 1] = t;
@@ -775,6 +781,64 @@ __device__ __forceinline__ void km_rows(const Dev& dv, float* __restrict__ out, 
       }
     }
     __syncwarp();
+    first_chunk = false;
+  };
+
+  if (BYTES || !dv.ordered) {  // misses from this width's region of the miss list
+    for (uint32_t base = gw * M; base < nmiss; base += nw * M) {
+      const uint32_t k = base + lane;
+      const bool has = lane < M && k < nmiss;
+      MissRec m{};
+      if (has) m = mlist[k];
+      chunk(has, m);
+    }
+  } else {
+    // address-ordered scratch: warp gw owns a contiguous slot window = a contiguous window
+    // of host addresses, so the GPU's host-link reads go out in (near) address order
+    const uint32_t nslots = dv.scr_mask + 1u;
+    const uint32_t per = (nslots + nw - 1) / nw;
+    const uint32_t lo = min(nslots, gw * per), hi = min(nslots, lo + per);
+    uint32_t my_slot = 0;
+    int P = 0;  // misses collected so far (lanes 0..P-1 hold their slots)
+    auto flush = [&]() {
+      MissRec m{};
+      const bool has = lane < P;
+      if (has) {
+        const unsigned long long tag = ld_cg_u64(dv.scratch + my_slot);
+        m.fk = (uint32_t)tag;
+        m.scr = my_slot;
+        m.off = dv.owner_off[my_slot];
+        int a = 0, b = dv.ntables;  // decode the table from the flat key (prefix match)
+        while (b - a > 1) {
+          const int mid = (a + b) >> 1;
+          if ((uint32_t)(dv.kdec[mid] >> 16) <= m.fk) a = mid; else b = mid;
+        }
+        m.t = (int32_t)(dv.kdec[a] & 0xFFFFu);
+      }
+      chunk(has, m);
+      P = 0;
+    };
+    for (uint32_t s1 = lo; s1 < hi; s1 += 256) {  // 8 tag loads per lane in flight, then in order
+      unsigned long long tags[8];
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        const uint32_t slot = s1 + 32 * i + lane;
+        tags[i] = slot < hi ? ld_cg_u64(dv.scratch + slot) : 0ull;
+      }
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        const uint32_t slot = s1 + 32 * i + lane;
+        unsigned found = __ballot_sync(kFull, slot < hi && (uint32_t)(tags[i] >> 32) == epoch);
+        while (found) {
+          const int f = __ffs(found) - 1;
+          found &= found - 1;
+          const uint32_t fs = __shfl_sync(kFull, slot, f);
+          if (lane == P) my_slot = fs;
+          if (++P == M) flush();
+        }
+      }
+    }
+    if (__any_sync(kFull, P > 0)) flush();
   }
 #ifdef FLECHE_EXPERIMENTS
   if (dv.exp_buf && lane == 0) {
