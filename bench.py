@@ -30,6 +30,8 @@ import numpy as np  # noqa: E402
 from workload import configs  # noqa: E402
 
 PREFILL = {"cfg0": 20, "cfg1": 150, "cfg2": 300, "cfg4": 30, "cfg5": 60}  # >= 2x the Che fill time
+# cfg3 (TB shape, batch 32768): Che fill time 177 / 437 / 1,492 / 3,898 batches at 1 / 2 / 5 / 10 %
+PREFILL_CFG3 = {0.01: 360, 0.02: 880, 0.05: 3000, 0.10: 7800}
 HASH_SEED = 0x9E3779B9
 
 
@@ -45,6 +47,7 @@ def parse():
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=15.0, help="oracle sample budget")
     p.add_argument("--flags", type=int, default=0, help="fleche_config.flags (ablations)")
+    p.add_argument("--cache-frac", type=float, default=None, help="override the config's cache fraction (sweeps)")
     p.add_argument("--mode", default="replicated", choices=["replicated", "sharded"],
                    help="multi-GPU partitioning: per-GPU replicated caches, or one key-sharded cache (NCCL all-to-all)")
     return p.parse_args()
@@ -217,7 +220,11 @@ def main():
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     w = configs.get(args.config)
+    if args.cache_frac is not None:
+        w = w.with_(cache_frac=args.cache_frac)
     P = PREFILL.get(args.config, 300) if args.prefill is None else args.prefill
+    if args.prefill is None and args.config.startswith("cfg3"):
+        P = PREFILL_CFG3.get(round(w.cache_frac, 2), 360)
     W, K = max(args.warmup, 0), max(args.steps, 1)
     if args.impl == "reference":
         return run_reference(args, w, P, W, K)

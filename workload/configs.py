@@ -114,6 +114,8 @@ def get(name: str) -> Workload:
         return Workload("cfg2", 2, list(KAGGLE), [64] * 26, [1.05] * 26, 8192, 0.05)
     if name == "cfg3":
         return Workload("cfg3", 3, list(TERABYTE), [64] * 26, [1.05] * 26, 32768, 0.01)
+    if name == "cfg3h":  # cfg3 at d = 32 (113 GB host tier): the GPU box has 196 GB of RAM
+        return Workload("cfg3h", 3, list(TERABYTE), [32] * 26, [1.05] * 26, 32768, 0.01)
     if name == "cfg4":
         c, d, s, h = _cfg4_tables()
         return Workload("cfg4", 4, c, d, s, 16384, 0.05, hotness=h)

@@ -178,7 +178,7 @@ EXPORT void flg_gen_ids(uint64_t s_id, uint64_t s_perm, int64_t b, int64_t t, in
   perm_init(&p, s_perm, t, c);
 #ifdef _OPENMP
   if (nthreads <= 0) nthreads = omp_get_max_threads();
-#pragma omp parallel for schedule(static, 2048) num_threads(nthreads) if (n > 65536)
+#pragma omp parallel for schedule(static, 1024) num_threads(nthreads) if (n >= 16384)
 #endif
   for (int64_t i = 0; i < n; ++i) {
     uint64_t q = id_stream(s_id, b, t, j0 + i);
