@@ -434,6 +434,17 @@ __global__ void __launch_bounds__(128) kq_kernel(const __grid_constant__ QArgs<M
       }
     }
     float* dst = (active && !miss) ? qa.out + off : nullptr;
+    // issue the timestamp read (hits) and the first scratch read (misses) now, so their
+    // L2 round trips overlap the row gather; they are consumed after it
+    uint32_t old_ts = 0, h = 0;
+    unsigned long long cur = 0;
+    if (hit) old_ts = ld_cg_u32(dv.ts + slot);
+    if (miss) {
+      h = dv.ordered ? (uint32_t)__umul64hi((uint64_t)(ti->host + (size_t)id * (size_t)d) - dv.host_lo, dv.host_mul) &
+                           dv.scr_mask
+                     : scr_hash(fk) & dv.scr_mask;
+      cur = ld_cg_u64(dv.scratch + h);
+    }
     const int d0 = __shfl_sync(kFull, d, 0);
     const bool uni = __all_sync(kFull, !active || d == d0);
     if (uni && d0 == 32) gather_rows<32>(src, dst, lane);
@@ -446,20 +457,13 @@ __global__ void __launch_bounds__(128) kq_kernel(const __grid_constant__ QArgs<M
 
     // hit: refresh the way's timestamp once per batch (approximate LRU)
     bool uhit = false;
-    if (hit) {
-      const uint32_t old = ld_cg_u32(dv.ts + slot);
-      if (old != epoch) uhit = atomicExch(dv.ts + slot, epoch) != epoch;
-    }
+    if (hit && old_ts != epoch) uhit = atomicExch(dv.ts + slot, epoch) != epoch;
 
     // A5 miss dedup: the lane whose CAS installs (epoch, fk) owns the miss
     int kind = 0;  // 1 = owner, 2 = duplicate
     uint32_t scr = 0;
     if (miss) {
       const unsigned long long tag = ((unsigned long long)epoch << 32) | fk;
-      uint32_t h = dv.ordered ? (uint32_t)__umul64hi((uint64_t)(ti->host + (size_t)id * (size_t)d) - dv.host_lo,
-                                                     dv.host_mul) & dv.scr_mask
-                              : scr_hash(fk) & dv.scr_mask;
-      unsigned long long cur = ld_cg_u64(dv.scratch + h);
       while (true) {
         if (cur == tag) { kind = 2; break; }
         if ((uint32_t)(cur >> 32) != epoch) {

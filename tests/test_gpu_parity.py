@@ -225,3 +225,24 @@ def test_cfg2_full_size_parity():
     assert abs(hg - ho) < 0.01, (hg, ho)
     st = gpu.stats()
     assert st["occupancy_bytes"] <= st["capacity_bytes"]
+
+
+@pytest.mark.parametrize("ordered", ["0", "1"])
+def test_address_ordered_scratch_exact(monkeypatch, ordered):
+    # the address-ordered miss scratch (KM hands each warp a contiguous host-address
+    # window) must leave results and stats unchanged: force it on / off for a small tier
+    if ordered == "1":
+        monkeypatch.setenv("FLECHE_ORDER_MIN_SPAN", "0")
+    else:
+        monkeypatch.setenv("FLECHE_NO_ORDER", "1")
+    w = configs.get("cfg0").with_(cache_frac=0.02, invalid_ppm=3000, skews=[0.7] * 7)
+    gpu, orc = _run(w, _tables(w), 25)
+    keys, _, slab = gpu.snapshot()
+    _, base, fb = gpu.encoding()
+    tabs = _tables(w)
+    live = np.nonzero(keys != 0xFFFFFFFF)[0]
+    assert {(int(np.nonzero((base <= k) & (k < base + (1 << fb.astype(np.int64))))[0][0]), 0) for k in keys[live]}
+    for way in live:
+        k = int(keys[way])
+        t = int(np.nonzero((base <= k) & (k < base + (1 << fb.astype(np.int64))))[0][0])
+        assert H.bits_equal(slab[way], tabs[t][k - int(base[t])])
