@@ -33,6 +33,13 @@
 #pragma once
 #include <cstdint>
 
+#ifndef FL_GATHER_F4
+#define FL_GATHER_F4 8  // float4 loads per lane in flight in a row gather (A/B builds vary it)
+#endif
+#ifndef FL_KQ_MIN_BLOCKS
+#define FL_KQ_MIN_BLOCKS 1  // KQ CTAs per SM the register budget must allow (A/B builds vary it)
+#endif
+
 namespace fl {
 
 constexpr uint32_t kEmpty = 0xFFFFFFFFu;
@@ -266,7 +273,7 @@ __device__ __forceinline__ void gather_rows(const float* src, float* dst, int la
   constexpr int RPP = 32 / LPR;             // rows per pass
   constexpr int VPL = VEC / LPR;            // float4 per lane per row
   constexpr int PASSES = 32 / RPP;
-  constexpr int CH0 = (8 / VPL) > 0 ? (8 / VPL) : 1;
+  constexpr int CH0 = (FL_GATHER_F4 / VPL) > 0 ? (FL_GATHER_F4 / VPL) : 1;
   constexpr int CH = CH0 < PASSES ? CH0 : PASSES;
   const int sub = lane % LPR, rs = lane / LPR;
 #pragma unroll 1
@@ -353,7 +360,8 @@ struct RowBuf {
 };
 
 template <int MAXT>
-__global__ void __launch_bounds__(128) kq_kernel(const __grid_constant__ QArgs<MAXT> qa, const __grid_constant__ Dev dv) {
+__global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_constant__ QArgs<MAXT> qa,
+                                                                   const __grid_constant__ Dev dv) {
   __shared__ int64_t s_scan[MAXT + 1];
   __shared__ unsigned long long s_ctr[kNumCtr];
   for (int i = threadIdx.x; i <= qa.n; i += blockDim.x) s_scan[i] = qa.scan[i];
