@@ -43,6 +43,12 @@ struct fleche_ctx {
   int km_bps = 4;  // KM CTAs per SM
   int kd_blocks = 0;
   bool per_table_launch = false;
+  // decoupled hit copy (uniform layout): KG on a side stream, forked after KQ, joined after KD
+  bool decoupled = false;
+  cudaStream_t side = nullptr;
+  cudaEvent_t fork_ev = nullptr, join_ev = nullptr;
+  uint32_t* d_slots = nullptr;
+  int64_t decouple_min = 65536;  // lookups per batch from which the hit copy is decoupled
   size_t km_smem = 0;
   // host-side counters
   uint64_t batches = 0, lookups = 0, kernels = 0;
@@ -168,12 +174,15 @@ void free_all(fleche_ctx* c) {
                   c->dv.firstpos, c->dv.ipos,
                   c->dv.miss, c->dv.dup, c->dv.ctl, c->dv.stats, c->d_tables, c->d_ids_stage, c->d_out_stage,
                   c->d_pool_stage, c->d_kdec, c->rd.scratch, c->rd.slotval, c->rd.inv, c->rd.region, c->rd.cnt,
-                  c->rd.prefix, c->rd.done, c->rd.stats};
+                  c->rd.prefix, c->rd.done, c->rd.stats, c->d_slots};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   for (auto& r : c->registered) cudaHostUnregister(r.first);
   c->registered.clear();
   if (c->chain_ev) cudaEventDestroy(c->chain_ev);
+  if (c->fork_ev) cudaEventDestroy(c->fork_ev);
+  if (c->join_ev) cudaEventDestroy(c->join_ev);
+  if (c->side) cudaStreamDestroy(c->side);
   for (cudaEvent_t e : c->ev_pool) cudaEventDestroy(e);
   c->ev_pool.clear();
 }
@@ -265,10 +274,20 @@ fleche_status launch_query(fleche_ctx* c, const int64_t* const* ids, const int64
   }
   fleche_status st = prof_event(c, s, true, nev);
   if (st != FLECHE_OK) return st;
+  // small batches: the fork/join costs more than the overlap saves (cfg1 measured +5 %)
+  const bool decouple = c->decoupled && total >= c->decouple_min && !c->per_table_launch;
+  if (decouple) qa.slots = c->d_slots;
   if (total > 0 && !c->per_table_launch) {
     const int64_t blocks = (total + 127) / 128;
     launch_k(kPdlKQ, kq_kernel<MAXT>, (unsigned)blocks, 128, 0, s, qa, c->dv);
     c->kernels++;
+    if (decouple) {  // fork: the hit copy runs on the side stream, concurrently with KM
+      FL_CUDA(c, cudaEventRecord(c->fork_ev, s));
+      FL_CUDA(c, cudaStreamWaitEvent(c->side, c->fork_ev, 0));
+      kg_kernel<MAXT><<<(unsigned)blocks, 128, 0, c->side>>>(qa, c->dv);
+      c->kernels++;
+      FL_CUDA(c, cudaEventRecord(c->join_ev, c->side));
+    }
   } else if (total > 0) {  // ablation: one query launch per table (n launches)
     QArgs<32> q1;
     memset(&q1, 0, sizeof(q1));
@@ -293,6 +312,7 @@ fleche_status launch_query(fleche_ctx* c, const int64_t* const* ids, const int64
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
   launch_k(kPdlKD, kd_kernel, c->kd_blocks, 128, 0, s, c->dv, out);
   c->kernels += 2;
+  if (decouple) FL_CUDA(c, cudaStreamWaitEvent(s, c->join_ev, 0));  // join: out complete on s
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return poison(c, e, "kernel launch");
@@ -542,6 +562,17 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
                                         std::max<int64_t>(1, (cfg->max_lookups + 255) / 256));
   c->km_smem = bytes ? (size_t)kKmWarps * kKmSmemF4 * sizeof(float4) : 0;
   c->kd_blocks = std::max(1, std::min(c->km_blocks, c->sm_count));  // one wave: duplicates are few
+  // decoupled hit copy: uniform layout only (the bytes layout compacts set regions in KM,
+  // which may move rows a concurrent copy reads; epoch protection covers the uniform slots)
+  c->decoupled = !bytes && getenv("FLECHE_FUSED_GATHER") == nullptr;
+  if (const char* e = getenv("FLECHE_DECOUPLE_MIN")) c->decouple_min = strtoll(e, nullptr, 10);
+  if (c->decoupled) {
+    if (cudaStreamCreateWithFlags(&c->side, cudaStreamNonBlocking) != cudaSuccess ||
+        cudaEventCreateWithFlags(&c->fork_ev, cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&c->join_ev, cudaEventDisableTiming) != cudaSuccess ||
+        cudaMalloc((void**)&c->d_slots, (size_t)cfg->max_lookups * 4) != cudaSuccess)
+      return fail(FLECHE_ENOMEM);
+  }
 #ifdef FLECHE_EXPERIMENTS
   if (cudaMalloc((void**)&dv.exp_buf, (size_t)c->km_blocks * 4 * 4 * 8) != cudaSuccess) return fail(FLECHE_ENOMEM);
   cudaMemset(dv.exp_buf, 0, (size_t)c->km_blocks * 4 * 4 * 8);

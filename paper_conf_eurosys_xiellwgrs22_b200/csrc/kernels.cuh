@@ -47,6 +47,7 @@ constexpr unsigned kFull = 0xFFFFFFFFu;
 constexpr int kStripes = 64;  // stats counters are striped to spread L2 atomics
 constexpr int kMaxCls = 6;    // row widths 8, 16, 32, 64, 128, 256 floats
 constexpr int kDupSlot = 7;   // Ctl::counts column of duplicate misses
+constexpr uint32_t kSlotMiss = 0xFFFFFFFFu, kSlotZero = 0xFFFFFFFEu;  // KQ -> KG codes
 constexpr int kKmWarps = 4;     // KM CTA = 4 warps
 constexpr int kKmStageF4 = 256; // bytes layout, per warp: staged rows of a chunk (<= 4 KB) ...
 constexpr int kKmSmemF4 = 512;  // ... + the compaction buffer of one set region (<= 4 KB)
@@ -148,6 +149,7 @@ struct QArgs {
   int64_t g0;                // batch position of this launch's first lookup (per-table launches)
   const uint32_t* fkeys;     // key-sharded owner side: flat keys instead of per-table IDs
   uint8_t* hit_flags;        // optional per-lookup hit flags (key-sharded)
+  uint32_t* slots;           // decoupled copy: per-lookup hit slot / kSlotMiss / kSlotZero for KG
   int32_t n;
   int32_t t0;                // first table of this launch (per-table launches: t0 = t, n = 1)
 };
@@ -311,6 +313,19 @@ __device__ __forceinline__ void gather_rows_any(const float* src, float* dst, in
   }
 }
 
+// Row gather for the warp's 32 lanes, specialised when every active lane has the same width.
+__device__ __forceinline__ void gather_dispatch(const float* src, float* dst, int d, bool active, int lane) {
+  const int d0 = __shfl_sync(kFull, d, 0);
+  const bool uni = __all_sync(kFull, !active || d == d0);
+  if (uni && d0 == 32) gather_rows<32>(src, dst, lane);
+  else if (uni && d0 == 64) gather_rows<64>(src, dst, lane);
+  else if (uni && d0 == 128) gather_rows<128>(src, dst, lane);
+  else if (uni && d0 == 16) gather_rows<16>(src, dst, lane);
+  else if (uni && d0 == 8) gather_rows<8>(src, dst, lane);
+  else if (uni && d0 == 256) gather_rows<256>(src, dst, lane);
+  else gather_rows_any(src, dst, d, lane);
+}
+
 // Rows of M misses held in registers across the warp (row r on lanes r*LPR..).
 template <int D, int M>
 struct RowBuf {
@@ -453,15 +468,11 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
                      : scr_hash(fk) & dv.scr_mask;
       cur = ld_cg_u64(dv.scratch + h);
     }
-    const int d0 = __shfl_sync(kFull, d, 0);
-    const bool uni = __all_sync(kFull, !active || d == d0);
-    if (uni && d0 == 32) gather_rows<32>(src, dst, lane);
-    else if (uni && d0 == 64) gather_rows<64>(src, dst, lane);
-    else if (uni && d0 == 128) gather_rows<128>(src, dst, lane);
-    else if (uni && d0 == 16) gather_rows<16>(src, dst, lane);
-    else if (uni && d0 == 8) gather_rows<8>(src, dst, lane);
-    else if (uni && d0 == 256) gather_rows<256>(src, dst, lane);
-    else gather_rows_any(src, dst, d, lane);
+    if (!qa.slots) {
+      gather_dispatch(src, dst, d, active, lane);
+    } else if (active) {  // decoupled: KG copies the hits on a side stream while KM fetches misses
+      qa.slots[g] = hit ? slot : (miss ? kSlotMiss : kSlotZero);
+    }
 
     // hit: refresh the way's timestamp once per batch (approximate LRU)
     bool uhit = false;
@@ -536,6 +547,47 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
   __syncthreads();
   if (threadIdx.x < kNumCtr && s_ctr[threadIdx.x])
     atomicAdd(dv.stats + (blockIdx.x % kStripes) * kNumCtr + threadIdx.x, s_ctr[threadIdx.x]);
+}
+
+// KG decoupled hit copy (Fig 8b): KQ only indexes (slot per lookup); KG copies
+// the hit rows from the slab on a side stream WHILE KM fetches the misses over the host
+// link -- the copy leaves the critical path of the miss handling.
+template <int MAXT>
+__global__ void __launch_bounds__(128) kg_kernel(const __grid_constant__ QArgs<MAXT> qa, const __grid_constant__ Dev dv) {
+  __shared__ int64_t s_scan[MAXT + 1];
+  for (int i = threadIdx.x; i <= qa.n; i += blockDim.x) s_scan[i] = qa.scan[i];
+  __syncthreads();
+  const int lane = threadIdx.x & 31;
+  const int64_t N = s_scan[qa.n];
+  const int64_t g = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (g - lane >= N) return;
+  const bool active = g < N;
+  int t = 0;
+  if (active) {
+    int lo = 0, hi = qa.n;
+    while (hi - lo > 1) {
+      const int mid = (lo + hi) >> 1;
+      if (s_scan[mid] <= g) lo = mid; else hi = mid;
+    }
+    t = lo;
+  }
+  const TableInfo* ti = dv.tables + t;
+  const int d = ti->dim;
+  const uint32_t code = active ? qa.slots[g] : kSlotMiss;
+  const float* src = nullptr;
+  float* dst = nullptr;
+  if (code != kSlotMiss) {
+    dst = qa.out + qa.out_off[t] + (g - s_scan[t]) * (int64_t)d;
+    if (code != kSlotZero) {
+      if (!dv.bytes) {
+        src = slot_row(dv, ti, code, d);
+      } else {
+        const uint32_t l = ld_nc_u32((const uint32_t*)(dv.loc + (code & ~1u))) >> ((code & 1u) * 16);
+        src = dv.slab + ((size_t)(code >> 5) * dv.set_units + (l & 0xFFu)) * 8u;
+      }
+    }
+  }
+  gather_dispatch(src, dst, d, active, lane);
 }
 
 // Uniform layout: claim a way for fk (first occurrence `pos` in the batch).

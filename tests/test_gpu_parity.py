@@ -121,6 +121,20 @@ def test_zero_capacity_and_empty_and_ragged():
         assert sg[k] == so[k], k
 
 
+@pytest.mark.parametrize("mode", ["decoupled", "fused"])
+def test_decoupled_hit_copy_exact(monkeypatch, mode):
+    # the hit copy on a side stream (KG, concurrent with the miss kernel) relies on epoch
+    # protection: this batch's hit ways are never victims, so their slab rows stay valid
+    if mode == "decoupled":
+        monkeypatch.setenv("FLECHE_DECOUPLE_MIN", "0")
+    else:
+        monkeypatch.setenv("FLECHE_FUSED_GATHER", "1")
+    w = configs.get("cfg0").with_(cache_frac=0.01, invalid_ppm=3000, skews=[0.6] * 7, batch_size=400)
+    gpu, _ = _run(w, _tables(w), 30)
+    per_batch = gpu.stats()["kernels_launched"] / 30
+    assert per_batch == (4 if mode == "decoupled" else 3)
+
+
 def test_admission_probability_exact():
     w = configs.get("cfg0").with_(cache_frac=0.25)
     _run(w, _tables(w), 20, admit_p=0.3, admit_seed=gen.seeds()["admit"])
