@@ -48,6 +48,7 @@ def parse():
     p.add_argument("--cpu-seconds", type=float, default=15.0, help="oracle sample budget")
     p.add_argument("--flags", type=int, default=0, help="fleche_config.flags (ablations)")
     p.add_argument("--cache-frac", type=float, default=None, help="override the config's cache fraction (sweeps)")
+    p.add_argument("--admit-prob", type=float, default=1.0, help="admission probability p (P:L655-659); 1 = canonical")
     p.add_argument("--mode", default="replicated", choices=["replicated", "sharded"],
                    help="multi-GPU partitioning: per-GPU replicated caches, or one key-sharded cache (NCCL all-to-all)")
     return p.parse_args()
@@ -258,8 +259,9 @@ def main():
     sharded = args.mode == "sharded"
     if sharded and (w.pooled or not uniform):
         raise SystemExit("--mode sharded supports one-hot, uniform-width configs (cfg1, cfg2, cfg5)")
-    cache = fl.FlatCache(w.cards, w.dims, tabs, w.cache_bytes, N * (world if sharded else 1), local, 1.0, 0,
-                         HASH_SEED, args.flags)
+    from workload import gen as _gen
+    cache = fl.FlatCache(w.cards, w.dims, tabs, w.cache_bytes, N * (world if sharded else 1), local,
+                         args.admit_prob, _gen.seeds()["admit"], HASH_SEED, args.flags)
     shard = None
     if sharded:
         if dist is None:
@@ -489,7 +491,7 @@ def main():
                        "cache_bytes": w.cache_bytes, "host_table_bytes": w.table_bytes,
                        "parallelism": (f"key-sharded x{world} (NCCL all-to-all)" if sharded else
                                        (f"replicated x{world}" if world > 1 else "single GPU")),
-                       "prefill_batches": P, "distinct_timed_batches": min(R, K),
+                       "prefill_batches": P, "distinct_timed_batches": min(R, K), "admit_prob": args.admit_prob,
                        "l2": "inputs larger than L2: fresh ID batch per step, 4 rotating output buffers "
                              f"({4 * out_max * 4 / 1e6:.0f} MB), {w.cache_bytes / 1e6:.0f} MB slab"},
             "hit_ratio": hit, "hit_ratio_unique": uhit,
