@@ -1,9 +1,17 @@
 # Build every native artefact in-tree (they travel to the GPU box with gpurun).
+# libfleche.so is linked from four translation units compiled in parallel (make -j):
+# the host side and three kernel groups (fns.h).
 NVCC    ?= /usr/local/cuda/bin/nvcc
 ARCH    := -gencode arch=compute_100a,code=sm_100a
 PKG     := paper_conf_eurosys_xiellwgrs22_b200
+CSRC    := $(PKG)/csrc
+BUILD   := build
 CFLAGS  := -O2 -fPIC -shared -fopenmp -Wall -Wextra
-NVFLAGS := $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC,-Wall -shared -cudart static -Iinclude
+NVFLAGS := $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC,-Wall -Iinclude
+HDRS    := $(wildcard $(CSRC)/*.cuh $(CSRC)/*.h) include/fleche.h
+UNITS   := fleche k_query k_miss k_misc
+OBJS    := $(UNITS:%=$(BUILD)/%.o)
+MAKEFLAGS += -j4
 
 all: workload/libflgen.so oracle/libfleche_oracle.so $(PKG)/libfleche.so
 
@@ -13,14 +21,21 @@ workload/libflgen.so: workload/gen.c
 oracle/libfleche_oracle.so: oracle/oracle.cpp
 	g++ -std=c++17 -O2 -fPIC -shared -Wall -Wextra -o $@ $<
 
-$(PKG)/libfleche.so: $(wildcard $(PKG)/csrc/*.cu $(PKG)/csrc/*.cuh $(PKG)/csrc/*.cpp) include/fleche.h
-	$(NVCC) $(NVFLAGS) -Xptxas -v -o $@ $(PKG)/csrc/fleche.cu 2> $(PKG)/ptxas.log || (cat $(PKG)/ptxas.log; exit 1)
+$(BUILD)/%.o: $(CSRC)/%.cu $(HDRS)
+	@mkdir -p $(BUILD)
+	$(NVCC) $(NVFLAGS) $(EXTRA) -Xptxas -v -c -o $@ $< 2> $(BUILD)/$*.ptxas.log || (cat $(BUILD)/$*.ptxas.log; exit 1)
+
+$(PKG)/libfleche.so: $(OBJS)
+	$(NVCC) $(ARCH) -shared -cudart static -o $@ $(OBJS)
+	cat $(UNITS:%=$(BUILD)/%.ptxas.log) > $(PKG)/ptxas.log
 
 clean:
-	rm -f workload/libflgen.so oracle/libfleche_oracle.so $(PKG)/libfleche.so
+	rm -rf $(BUILD) workload/libflgen.so oracle/libfleche_oracle.so $(PKG)/libfleche.so $(PKG)/libfleche_exp.so
 
 .PHONY: all clean
 
-# timing-experiment build (tools only; semantics-breaking knobs behind FLECHE_EXP_MODE)
-$(PKG)/libfleche_exp.so: $(wildcard $(PKG)/csrc/*.cu $(PKG)/csrc/*.cuh) include/fleche.h
-	$(NVCC) $(NVFLAGS) -DFLECHE_EXPERIMENTS -o $@ $(PKG)/csrc/fleche.cu
+# timing-experiment build (tools only; semantics-breaking knobs behind FLECHE_EXPERIMENTS)
+$(PKG)/libfleche_exp.so: $(wildcard $(CSRC)/*.cu) $(HDRS)
+	@mkdir -p $(BUILD)/exp
+	for u in $(UNITS); do $(NVCC) $(NVFLAGS) -DFLECHE_EXPERIMENTS -c -o $(BUILD)/exp/$$u.o $(CSRC)/$$u.cu || exit 1; done
+	$(NVCC) $(ARCH) -shared -cudart static -o $@ $(UNITS:%=$(BUILD)/exp/%.o)

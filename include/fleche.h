@@ -96,6 +96,22 @@ typedef struct {
  *   self-identified launch; the kernel-maintenance cost of P:L479-497). */
 #define FLECHE_FLAG_STATIC_PER_TABLE 0x2u
 #define FLECHE_FLAG_PER_TABLE_LAUNCH 0x4u
+/* HOST_ASSIST: host-assisted miss fetch -- the paper's decoupled workflow with the
+ * CPU-DRAM layer queried "ahead", as soon as the indexing kernel knows which keys miss,
+ * in parallel with the GPU's hit copy (Fig 8b; CPU-DRAM layer P:L177-178).
+ * The default path is the unified index (Fig 8c): the GPU reads each missed
+ * row where it lies in the host tables.  On a host whose IOMMU translation caps scattered
+ * zero-copy reads (measured on the graft B200 pool: ~80 M rows/s beyond a ~1 GiB span,
+ * DESIGN.md §6) the ctx can instead run host threads that gather the batch's unique
+ * missed rows into a contiguous pinned staging buffer, which the miss kernel then reads
+ * over the link at its full rate.  Requests travel GPU -> host through pinned memory (no
+ * host sync, no extra launch: the query path stays asynchronous and graph-capturable);
+ * a block the threads have not staged within FLECHE_HA_TIMEOUT_US (default 2000) is read
+ * zero-copy from the tables instead, so correctness never depends on the threads.  Env:
+ * FLECHE_HA_THREADS (default 12), FLECHE_HA_STAGE_KB (staging per epoch parity, default
+ * 131072; rows beyond it are read zero-copy).  Not with PER_TABLE_LAUNCH (FLECHE_EINVAL).  `out`, hits and every cache decision are identical with and without
+ * it; only where the missed rows are read from changes. */
+#define FLECHE_FLAG_HOST_ASSIST 0x8u
 
 typedef struct {
   uint64_t batches;            /* query calls                                                       */
@@ -115,6 +131,8 @@ typedef struct {
   uint64_t index_bytes;        /* HBM used by index + scratch (not counted in cache_bytes)          */
   uint64_t host_bytes_fetched; /* bytes read from the host tier over the host link                  */
   uint64_t kernels_launched;   /* kernels this ctx launched                                         */
+  uint64_t assisted_rows;      /* HOST_ASSIST: unique misses read from the host threads' staging    */
+  uint64_t assist_timeouts;    /* HOST_ASSIST: staging blocks fetched zero-copy after the timeout   */
 } fleche_stats_t;
 
 /* Create a cache for the tables in *cfg on cfg->device.  Allocates every device

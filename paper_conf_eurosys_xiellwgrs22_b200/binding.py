@@ -20,6 +20,7 @@ _lib = ctypes.CDLL(LIB_PATH)
 
 OK, EINVAL, ENOMEM, ECUDA, ENCCL, ERANGE, ESTATE = 0, -1, -2, -3, -4, -5, -6
 FLAG_L2_PREFETCH = 0x1
+FLAG_STATIC_PER_TABLE, FLAG_PER_TABLE_LAUNCH, FLAG_HOST_ASSIST = 0x2, 0x4, 0x8
 MAX_TABLES = 512
 
 _vp, _i64, _i32, _u64, _u32 = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32, ctypes.c_uint64, ctypes.c_uint32
@@ -33,7 +34,7 @@ class fleche_config(ctypes.Structure):
 
 STAT_FIELDS = ["batches", "lookups", "hits", "misses", "invalid", "unique_keys", "unique_hits", "unique_misses",
                "inserted", "evicted", "bypassed", "occupancy_bytes", "capacity_bytes", "index_bytes",
-               "host_bytes_fetched", "kernels_launched"]
+               "host_bytes_fetched", "kernels_launched", "assisted_rows", "assist_timeouts"]
 
 
 class fleche_stats_t(ctypes.Structure):

@@ -7,18 +7,54 @@
 // query path), cross-stream ordering, and the stats read-back.
 #include <cuda_runtime.h>
 
+#include <immintrin.h>
+#include <time.h>
+
 #include <algorithm>
+#include <atomic>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
 #include <new>
+#include <thread>
 #include <vector>
 
 #include "fleche.h"
-#include "kernels.cuh"
-#include "shard.cuh"
+#include "fns.h"
 
 using namespace fl;
+
+// Host-assisted miss fetch (FLECHE_FLAG_HOST_ASSIST; device side in kernels.cuh): the
+// CPU-DRAM layer's threads gather the rows KQ requests into the pinned
+// staging buffer.  Thread i owns every staging block k with k % nthreads == i, in every
+// batch, so a block is only ever written by one thread, batch after batch in order: a
+// thread that fell behind (its blocks timed out on the GPU, which fetched them itself)
+// can never overwrite a newer batch's rows after their ready flag.
+struct HostAssist {
+  int nthreads = 0;
+  std::vector<std::thread> th;
+  std::atomic<bool> stop{false};
+  // mapped pinned host memory (cudaHostAlloc): host pointers (the device sees the same
+  // allocations through Dev::ha_*)
+  void* mem = nullptr;
+  HaReq* req = nullptr;                // [2][req_cap] (indexed like the miss list)
+  HaDesc* desc = nullptr;              // [2]
+  unsigned long long* bell = nullptr;  // doorbell (epoch)
+  uint32_t* ready = nullptr;           // [2][blk_cap]
+  float* stage = nullptr;              // [2][stage_floats]
+  uint32_t req_cap = 0, blk_cap = 0;
+  bool nt_stores = true;  // FLECHE_HA_NT=0: plain memcpy into the staging buffer (A/B)
+  uint64_t stage_floats = 0;
+  // the tables as the host threads see them
+  std::vector<const float*> host;
+  std::vector<int64_t> card;
+  std::vector<int32_t> dims;
+#ifdef FLECHE_EXPERIMENTS
+  uint64_t exp_t[64 * 2 * 64] = {};
+  uint64_t* exp_pub = nullptr;  // CLOCK_REALTIME when each block's ready flag was published
+  bool exp_nogather = getenv("FLECHE_HA_EXP_NOGATHER") != nullptr;
+#endif
+};
 
 struct fleche_ctx {
   int device = 0;
@@ -72,6 +108,7 @@ struct fleche_ctx {
   bool rd_ready = false;
   uint32_t repoch = 0;
   std::vector<int64_t> route_len;
+  HostAssist* ha = nullptr;
 };
 
 namespace {
@@ -169,6 +206,128 @@ fleche_status register_host(fleche_ctx* c, const float* const* host, std::vector
   return FLECHE_OK;
 }
 
+// Row copy into the staging buffer with non-temporal stores: the rows go to DRAM, not
+// into this core's cache, so the GPU's link reads of them are not stalled snooping
+// modified lines out of the writer's cache (dst 32 B aligned, bytes a multiple of 32).
+__attribute__((target("avx2"))) void stage_row(float* dst, const float* src, size_t bytes) {
+  for (size_t b = 0; b < bytes; b += 32)
+    _mm256_stream_si256((__m256i*)((char*)dst + b), _mm256_loadu_si256((const __m256i*)((const char*)src + b)));
+}
+
+// One host-assist thread: wait for a doorbell, gather this thread's blocks of the
+// batch's requests (block k = miss-list indices [64k, 64k + 64), rows of every width class
+// in it), publish each block's ready flag.  Spins while batches keep coming; after ~2 ms
+// without one it polls every 50 us (an idle ctx burns no core).  No `pause` in the spin:
+// on a KVM guest it can trigger pause-loop exits that deschedule the vCPU.
+void ha_worker(HostAssist* h, int me) {
+  uint32_t last = 0;
+  uint64_t spins = 0;
+  auto now_ns = []() {
+    struct timespec ts;
+    clock_gettime(CLOCK_MONOTONIC, &ts);
+    return (uint64_t)ts.tv_sec * 1000000000ull + (uint64_t)ts.tv_nsec;
+  };
+  uint64_t t_last = now_ns();
+  const int nt = (int)h->host.size();
+  while (!h->stop.load(std::memory_order_relaxed)) {
+    const uint32_t e = (uint32_t)__atomic_load_n(h->bell, __ATOMIC_ACQUIRE);
+    if (e == last) {
+      if ((++spins & 1023) == 0 && now_ns() - t_last > 2000000ull) {
+        struct timespec ts = {0, 50000};
+        nanosleep(&ts, nullptr);
+      }
+      continue;
+    }
+    last = e;
+    t_last = now_ns();
+#ifdef FLECHE_EXPERIMENTS
+    auto rt = []() {
+      struct timespec ts;
+      clock_gettime(CLOCK_REALTIME, &ts);
+      return (uint64_t)ts.tv_sec * 1000000000ull + (uint64_t)ts.tv_nsec;
+    };
+    if (me < 64) h->exp_t[(e % 64) * 128 + me] = rt();
+#endif
+    const int par = e & 1u;
+    const HaDesc d = h->desc[par];
+    if (d.epoch != e) continue;  // the GPU is a full parity cycle ahead: this batch timed out anyway
+    const HaReq* rq = h->req + (size_t)par * h->req_cap;
+    float* st = h->stage + (size_t)par * h->stage_floats;
+    uint64_t lo_all = ~0ull, hi_all = 0;
+    for (int c = 0; c < 8; ++c)
+      if (d.cnt[c]) {
+        lo_all = std::min<uint64_t>(lo_all, d.off[c]);
+        hi_all = std::max<uint64_t>(hi_all, (uint64_t)d.off[c] + d.cnt[c]);
+      }
+    if (hi_all == 0 || hi_all > h->req_cap) continue;
+    auto src_of = [&](const HaReq& r, int32_t* dim) -> const float* {
+      const int t = (int)(r.tid >> 48);
+      const int64_t id = (int64_t)(r.tid & 0xFFFFFFFFFFFFull);
+      if (r.stage == kNoStage || t >= nt || id >= h->card[t]) return nullptr;  // no room / defensive
+      *dim = h->dims[t];
+      if (r.stage + (uint64_t)*dim > h->stage_floats) return nullptr;
+      return h->host[t] + (size_t)id * (size_t)*dim;
+    };
+    auto prefetch = [&](uint64_t i) {
+      int32_t dd = 0;
+      if (const float* p = src_of(rq[i], &dd))
+        for (int b = 0; b < dd * 4; b += 64) __builtin_prefetch((const char*)p + b, 0, 0);
+    };
+    const uint64_t kb0 = lo_all / kHaBlock, kb1 = (hi_all - 1) / kHaBlock;
+    for (uint64_t kb = kb0; kb <= kb1; ++kb) {
+      if (kb % (uint64_t)h->nthreads != (uint64_t)me) continue;
+      bool any = false;
+      for (int c = 0; c < 8; ++c) {  // the rows of every class region that overlaps block kb
+        if (!d.cnt[c]) continue;
+        const uint64_t lo = std::max<uint64_t>(kb * kHaBlock, d.off[c]);
+        const uint64_t hi = std::min<uint64_t>(kb * kHaBlock + kHaBlock, (uint64_t)d.off[c] + d.cnt[c]);
+        if (lo >= hi) continue;
+        any = true;
+        constexpr uint64_t PF = 8;  // rows prefetched ahead
+        for (uint64_t i = lo; i < std::min(hi, lo + PF); ++i) prefetch(i);
+        for (uint64_t i = lo; i < hi; ++i) {
+          if (i + PF < hi) prefetch(i + PF);
+          const HaReq r = rq[i];
+          int32_t dd = 0;
+          if (const float* p = src_of(r, &dd)) {
+#ifdef FLECHE_EXPERIMENTS
+            if (h->exp_nogather) continue;  // timing experiment: publish without gathering (wrong rows)
+#endif
+            if (h->nt_stores) stage_row(st + r.stage, p, (size_t)dd * 4u);
+            else memcpy(st + r.stage, p, (size_t)dd * 4u);
+          }
+        }
+      }
+      if (h->nt_stores) _mm_sfence();  // streaming stores are weakly ordered: drain them before the flag
+      if (any) __atomic_store_n(h->ready + (size_t)par * h->blk_cap + kb, e, __ATOMIC_RELEASE);
+#ifdef FLECHE_EXPERIMENTS
+      if (any && h->exp_pub) {
+        struct timespec ts;
+        clock_gettime(CLOCK_REALTIME, &ts);
+        h->exp_pub[kb] = (uint64_t)ts.tv_sec * 1000000000ull + (uint64_t)ts.tv_nsec;
+      }
+#endif
+    }
+#ifdef FLECHE_EXPERIMENTS
+    if (me < 64) {
+      struct timespec ts;
+      clock_gettime(CLOCK_REALTIME, &ts);
+      h->exp_t[(e % 64) * 128 + 64 + me] = (uint64_t)ts.tv_sec * 1000000000ull + (uint64_t)ts.tv_nsec;
+    }
+#endif
+  }
+}
+
+void ha_stop(HostAssist* h) {
+  if (!h) return;
+  h->stop.store(true);
+  for (auto& t : h->th)
+    if (t.joinable()) t.join();
+  h->th.clear();
+  if (h->mem) cudaFreeHost(h->mem);
+  h->mem = nullptr;
+}
+
 void free_all(fleche_ctx* c) {
   void* ptrs[] = {c->dv.keys, c->dv.ts, c->dv.loc, c->dv.lock, c->dv.slab, c->dv.scratch, c->dv.owner_off,
                   c->dv.firstpos, c->dv.ipos,
@@ -185,6 +344,11 @@ void free_all(fleche_ctx* c) {
   if (c->side) cudaStreamDestroy(c->side);
   for (cudaEvent_t e : c->ev_pool) cudaEventDestroy(e);
   c->ev_pool.clear();
+  if (c->ha) {
+    ha_stop(c->ha);
+    delete c->ha;
+    c->ha = nullptr;
+  }
 }
 
 fleche_status ensure_device(fleche_ctx* c) {
@@ -221,7 +385,7 @@ fleche_status prof_event(fleche_ctx* c, cudaStream_t s, bool first, int kinds) {
 // Per-kernel PDL mask (bit 0 KQ, 1 KM, 2 KD, 3 KP).  KM is launched without it by default:
 // its blocks would be placed early, during KQ's tail, which measured slower for the
 // address-ordered miss fetch (profiles/README.md).
-enum { kPdlKQ = 0, kPdlKM = 1, kPdlKD = 2, kPdlKP = 3 };
+enum { kPdlKQ = 0, kPdlKM = 1, kPdlKD = 2, kPdlKP = 3, kPdlNone = 30 };
 int pdl_mask() {
   static const int m = getenv("FLECHE_NO_PDL") ? 0 : (getenv("FLECHE_PDL_MASK") ? atoi(getenv("FLECHE_PDL_MASK")) : 0xD);
   return m;
@@ -279,12 +443,12 @@ fleche_status launch_query(fleche_ctx* c, const int64_t* const* ids, const int64
   if (decouple) qa.slots = c->d_slots;
   if (total > 0 && !c->per_table_launch) {
     const int64_t blocks = (total + 127) / 128;
-    launch_k(kPdlKQ, kq_kernel<MAXT>, (unsigned)blocks, 128, 0, s, qa, c->dv);
+    launch_k(kPdlKQ, kq_fn<MAXT>(), (unsigned)blocks, 128, 0, s, qa, c->dv);
     c->kernels++;
     if (decouple) {  // fork: the hit copy runs on the side stream, concurrently with KM
       FL_CUDA(c, cudaEventRecord(c->fork_ev, s));
       FL_CUDA(c, cudaStreamWaitEvent(c->side, c->fork_ev, 0));
-      kg_kernel<MAXT><<<(unsigned)blocks, 128, 0, c->side>>>(qa, c->dv);
+      launch_k(kPdlNone, kg_fn<MAXT>(), (unsigned)blocks, 128, 0, c->side, qa, c->dv);
       c->kernels++;
       FL_CUDA(c, cudaEventRecord(c->join_ev, c->side));
     }
@@ -302,15 +466,14 @@ fleche_status launch_query(fleche_ctx* c, const int64_t* const* ids, const int64
       q1.scan[0] = 0;
       q1.scan[1] = lengths[t];
       q1.out_off[0] = qa.out_off[t];
-      launch_k(kPdlKQ, kq_kernel<32>, (unsigned)((lengths[t] + 127) / 128), 128, 0, s, q1, c->dv);
+      launch_k(kPdlKQ, kq_fn<32>(), (unsigned)((lengths[t] + 127) / 128), 128, 0, s, q1, c->dv);
       c->kernels++;
     }
   }
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
-  if (c->dv.bytes) launch_k(kPdlKM, km_kernel<true>, c->km_blocks, 128, c->km_smem, s, c->dv, ka);
-  else launch_k(kPdlKM, km_kernel<false>, c->km_blocks, 128, 0, s, c->dv, ka);
+  launch_k(kPdlKM, km_fn(c->dv.bytes != 0, c->cls_dim.size() == 1 ? c->max_dim : 0), c->km_blocks, 128, c->km_smem, s, c->dv, ka);
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
-  launch_k(kPdlKD, kd_kernel, c->kd_blocks, 128, 0, s, c->dv, out);
+  launch_k(kPdlKD, kd_fn(), c->kd_blocks, 128, 0, s, c->dv, out);
   c->kernels += 2;
   if (decouple) FL_CUDA(c, cudaStreamWaitEvent(s, c->join_ev, 0));  // join: out complete on s
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
@@ -363,7 +526,7 @@ fleche_status launch_pool(fleche_ctx* c, const int64_t* const* offsets, const in
   }
   pa.cscan[c->n] = cs;
   if (cs > 0) {
-    launch_k(kPdlKP, kp_kernel<MAXT>, (unsigned)((cs + 255) / 256), 256, 0, s, pa, (const TableInfo*)c->d_tables);
+    launch_k(kPdlKP, kp_fn<MAXT>(), (unsigned)((cs + 255) / 256), 256, 0, s, pa, (const TableInfo*)c->d_tables);
     c->kernels++;
   }
   fleche_status st = prof_event(c, s, false, 0);
@@ -395,8 +558,10 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   *out = nullptr;
   const int n = cfg->num_tables;
   if (n < 1 || n > FLECHE_MAX_TABLES || !cfg->cardinalities || !cfg->dims || !cfg->host_tables) return FLECHE_EINVAL;
-  const uint32_t known = FLECHE_FLAG_L2_PREFETCH | FLECHE_FLAG_STATIC_PER_TABLE | FLECHE_FLAG_PER_TABLE_LAUNCH;
+  const uint32_t known = FLECHE_FLAG_L2_PREFETCH | FLECHE_FLAG_STATIC_PER_TABLE | FLECHE_FLAG_PER_TABLE_LAUNCH |
+                         FLECHE_FLAG_HOST_ASSIST;
   if (cfg->max_lookups < 1 || cfg->max_lookups > (int64_t(1) << 31) || (cfg->flags & ~known)) return FLECHE_EINVAL;
+  if ((cfg->flags & FLECHE_FLAG_HOST_ASSIST) && (cfg->flags & FLECHE_FLAG_PER_TABLE_LAUNCH)) return FLECHE_EINVAL;
   for (int t = 0; t < n; ++t) {
     if (cfg->cardinalities[t] < 1 || !valid_dim(cfg->dims[t])) return FLECHE_EINVAL;
     if (!cfg->host_tables[t] || ((uintptr_t)cfg->host_tables[t] & 15u)) return FLECHE_EINVAL;
@@ -485,9 +650,6 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   dv.admit_thr = dv.admit_all ? ~0ull : (uint64_t)ldexp(p, 64);
   dv.admit_seed = cfg->admit_seed;
   dv.prefetch = (cfg->flags & FLECHE_FLAG_L2_PREFETCH) ? 1 : 0;
-  dv.km_m = c->max_dim <= 32 ? 16 : 8;
-  if (const char* e = getenv("FLECHE_KM_M")) dv.km_m = atoi(e);  // tuning knob (bench sweeps)
-  if (bytes) dv.km_m = std::min(dv.km_m, 8);                     // smem staging holds <= 4 KB of rows
   if (const char* e = getenv("FLECHE_KM_BLOCKS_PER_SM")) c->km_bps = std::max(1, atoi(e));
 #ifdef FLECHE_EXPERIMENTS
   if (const char* e = getenv("FLECHE_EXP_MODE")) dv.exp_mode = atoi(e);
@@ -560,7 +722,12 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   // KM: enough warps for the expected unique misses, km_bps CTAs of 4 warps per SM
   c->km_blocks = (int)std::min<int64_t>((int64_t)c->km_bps * c->sm_count,
                                         std::max<int64_t>(1, (cfg->max_lookups + 255) / 256));
-  c->km_smem = bytes ? (size_t)kKmWarps * kKmSmemF4 * sizeof(float4) : 0;
+  c->km_smem = (size_t)kKmWarps * ((bytes ? kKmSmemF4 : 0) + ((cfg->flags & FLECHE_FLAG_HOST_ASSIST) ? kHaSmemF4 : 0)) *
+               sizeof(float4);
+  if (c->km_smem > 48 * 1024 &&
+      cudaFuncSetAttribute((const void*)km_fn(bytes, c->cls_dim.size() == 1 ? c->max_dim : 0),
+                           cudaFuncAttributeMaxDynamicSharedMemorySize, (int)c->km_smem) != cudaSuccess)
+    return fail(FLECHE_ECUDA);
   c->kd_blocks = std::max(1, std::min(c->km_blocks, c->sm_count));  // one wave: duplicates are few
   // decoupled hit copy: uniform layout only (the bytes layout compacts set regions in KM,
   // which may move rows a concurrent copy reads; epoch protection covers the uniform slots)
@@ -573,9 +740,60 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
         cudaMalloc((void**)&c->d_slots, (size_t)cfg->max_lookups * 4) != cudaSuccess)
       return fail(FLECHE_ENOMEM);
   }
+  if (cfg->flags & FLECHE_FLAG_HOST_ASSIST) {
+    HostAssist* h = c->ha = new (std::nothrow) HostAssist();
+    if (!h) return fail(FLECHE_ENOMEM);
+    auto env_u = [](const char* k, uint64_t dflt) {
+      const char* e = getenv(k);
+      return e ? strtoull(e, nullptr, 10) : dflt;
+    };
+    h->nthreads = (int)std::max<uint64_t>(1, std::min<uint64_t>(64, env_u("FLECHE_HA_THREADS", 12)));
+    h->req_cap = (uint32_t)cfg->max_lookups;  // requests are indexed like the miss list
+    h->blk_cap = h->req_cap / kHaBlock + 2;
+    h->stage_floats = std::max<uint64_t>(1024, env_u("FLECHE_HA_STAGE_KB", 131072) << 8);
+    const size_t o_req = 0, o_desc = o_req + 2 * sizeof(HaReq) * (size_t)h->req_cap, o_bell = o_desc + 2 * sizeof(HaDesc),
+                 o_ready = (o_bell + 8 + 63) & ~size_t(63), o_stage = (o_ready + 8ull * h->blk_cap + 255) & ~size_t(255),
+                 total = o_stage + 2 * 4 * h->stage_floats;
+    if (cudaHostAlloc(&h->mem, total, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess) {
+      cudaGetLastError();
+      h->mem = nullptr;
+      return fail(FLECHE_ENOMEM);
+    }
+    memset(h->mem, 0, o_stage);
+    char* b = (char*)h->mem;
+    h->req = (HaReq*)(b + o_req);
+    h->desc = (HaDesc*)(b + o_desc);
+    h->bell = (unsigned long long*)(b + o_bell);
+    h->ready = (uint32_t*)(b + o_ready);
+    h->stage = (float*)(b + o_stage);
+    void* dmem = nullptr;
+    if (cudaHostGetDevicePointer(&dmem, h->mem, 0) != cudaSuccess) return fail(FLECHE_ECUDA);
+    char* db = (char*)dmem;
+    dv.ha = 1;
+    dv.ha_req = (HaReq*)(db + o_req);
+    dv.ha_desc = (HaDesc*)(db + o_desc);
+    dv.ha_bell = (unsigned long long*)(db + o_bell);
+    dv.ha_ready = (uint32_t*)(db + o_ready);
+    dv.ha_stage = (float*)(db + o_stage);
+    dv.ha_req_cap = h->req_cap;
+    dv.ha_blk_cap = h->blk_cap;
+    dv.ha_stage_floats = h->stage_floats;
+    dv.ha_timeout_ns = env_u("FLECHE_HA_TIMEOUT_US", 2000) * 1000ull;
+    h->nt_stores = env_u("FLECHE_HA_NT", 1) != 0 && __builtin_cpu_supports("avx2");
+    h->host.assign(cfg->host_tables, cfg->host_tables + n);
+    h->card = c->card;
+    h->dims = c->dims;
+    for (int i = 0; i < h->nthreads; ++i) h->th.emplace_back(ha_worker, h, i);
+  }
 #ifdef FLECHE_EXPERIMENTS
-  if (cudaMalloc((void**)&dv.exp_buf, (size_t)c->km_blocks * 4 * 4 * 8) != cudaSuccess) return fail(FLECHE_ENOMEM);
-  cudaMemset(dv.exp_buf, 0, (size_t)c->km_blocks * 4 * 4 * 8);
+  if (cudaMalloc((void**)&dv.exp_buf, ((size_t)c->km_blocks * 4 * 4 + 8) * 8) != cudaSuccess) return fail(FLECHE_ENOMEM);
+  cudaMemset(dv.exp_buf, 0, ((size_t)c->km_blocks * 4 * 4 + 8) * 8);
+  dv.exp_slots = (uint32_t)c->km_blocks * 16;
+  if (c->ha) {
+    if (cudaMalloc((void**)&dv.exp_blk, ((size_t)c->ha->blk_cap * 4) * 8) != cudaSuccess) return fail(FLECHE_ENOMEM);
+    cudaMemset(dv.exp_blk, 0, ((size_t)c->ha->blk_cap * 4) * 8);
+    c->ha->exp_pub = new uint64_t[c->ha->blk_cap]();
+  }
 #endif
   if (cudaDeviceSynchronize() != cudaSuccess) return fail(FLECHE_ECUDA);
   *out = c;
@@ -684,6 +902,8 @@ fleche_status fleche_stats(fleche_ctx* c, fleche_stats_t* out) {
   out->index_bytes = c->index_bytes;
   out->host_bytes_fetched = v[C_HOSTBYTES];
   out->kernels_launched = c->kernels;
+  out->assisted_rows = v[C_HAROWS];
+  out->assist_timeouts = v[C_HATIMEOUT];
   return ctl.err_invalid ? FLECHE_ERANGE : FLECHE_OK;
 }
 
@@ -812,10 +1032,7 @@ fleche_status fleche_probe_host_read(const void* host, uint64_t bytes, int32_t r
   const uint64_t span = bytes / (uint64_t)row_bytes;
   const unsigned blocks = (unsigned)((rows + 127) / 128);
   auto launch = [&](uint64_t sd) {
-    if (D == 32) probe_host_kernel<32><<<blocks, 128, 0, s>>>((const float*)dev, span, rows, sd, sink);
-    else if (D == 64) probe_host_kernel<64><<<blocks, 128, 0, s>>>((const float*)dev, span, rows, sd, sink);
-    else if (D == 128) probe_host_kernel<128><<<blocks, 128, 0, s>>>((const float*)dev, span, rows, sd, sink);
-    else probe_host_kernel<256><<<blocks, 128, 0, s>>>((const float*)dev, span, rows, sd, sink);
+    launch_k(kPdlNone, probe_fn(D), blocks, 128, 0, s, (const float*)dev, span, rows, sd, sink);
   };
   launch(seed ^ 0x5555);  // warm-up (clocks)
   cudaEventRecord(e0, s);
@@ -855,13 +1072,13 @@ fleche_status launch_keys(fleche_ctx* c, const uint32_t* keys, int64_t count, fl
   fleche_status st = prof_event(c, s, true, 4);
   if (st != FLECHE_OK) return st;
   if (count > 0) {
-    launch_k(kPdlKQ, kq_kernel<MAXT>, (unsigned)((count + 127) / 128), 128, 0, s, qa, c->dv);
+    launch_k(kPdlKQ, kq_fn<MAXT>(), (unsigned)((count + 127) / 128), 128, 0, s, qa, c->dv);
     c->kernels++;
   }
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
-  launch_k(kPdlKM, km_kernel<false>, c->km_blocks, 128, 0, s, c->dv, ka);
+  launch_k(kPdlKM, km_fn(false, c->cls_dim.size() == 1 ? c->max_dim : 0), c->km_blocks, 128, c->km_smem, s, c->dv, ka);
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
-  launch_k(kPdlKD, kd_kernel, c->kd_blocks, 128, 0, s, c->dv, rows);
+  launch_k(kPdlKD, kd_fn(), c->kd_blocks, 128, 0, s, c->dv, rows);
   c->kernels += 2;
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
   cudaError_t e = cudaGetLastError();
@@ -891,11 +1108,12 @@ fleche_status launch_route(fleche_ctx* c, const int64_t* const* ids, const int64
   RArgs<MAXT> ra;
   fill_rargs<MAXT>(c, ra, ids, lengths);
   if (total > 0) {
-    kr_kernel<MAXT><<<(unsigned)((total + 127) / 128), 128, 0, s>>>(ra, c->rd, c->d_tables);
+    launch_k(kPdlNone, kr_fn<MAXT>(), (unsigned)((total + 127) / 128), 128, 0, s, ra, c->rd,
+             (const TableInfo*)c->d_tables);
     c->kernels++;
   }
-  kpk_kernel<<<std::max(1, std::min(2 * c->sm_count, (int)((total + 255) / 256))), 256, 0, s>>>(c->rd, send_keys,
-                                                                                              send_counts);
+  launch_k(kPdlNone, kpk_fn(), (unsigned)std::max(1, std::min(2 * c->sm_count, (int)((total + 255) / 256))), 256, 0, s,
+           c->rd, send_keys, send_counts);
   c->kernels++;
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return poison(c, e, "kernel launch");
@@ -908,7 +1126,7 @@ fleche_status launch_restore_d(fleche_ctx* c, const float* rows, const uint8_t* 
   fill_rargs<MAXT>(c, ra, nullptr, c->route_len.data());
   const int64_t total = ra.scan[c->n];
   if (total > 0) {
-    krs_kernel<MAXT, D><<<(unsigned)((total + 127) / 128), 128, 0, s>>>(ra, c->rd, rows, flags, out);
+    launch_k(kPdlNone, krs_fn<MAXT>(D), (unsigned)((total + 127) / 128), 128, 0, s, ra, c->rd, rows, flags, out);
     c->kernels++;
   }
   cudaError_t e = cudaGetLastError();
@@ -1048,7 +1266,30 @@ extern "C" __attribute__((visibility("default"))) fleche_status fleche_exp_timel
                                                                                     size_t n) {
   if (!c || !host) return FLECHE_EINVAL;
   if (c->have_last) cudaStreamSynchronize(c->last_stream);
-  const size_t m = std::min(n, (size_t)c->km_blocks * 16);
+  const size_t m = std::min(n, (size_t)c->km_blocks * 16 + 8);
   return cudaMemcpy(host, c->dv.exp_buf, m * 8, cudaMemcpyDeviceToHost) == cudaSuccess ? FLECHE_OK : FLECHE_ECUDA;
+}
+// host-assist threads: CLOCK_REALTIME (ns) when each thread saw the doorbell of epoch e
+// and when it finished its blocks, out[(e % 64) * 2 * 64 + {0,1} * 64 + thread]
+extern "C" __attribute__((visibility("default"))) fleche_status fleche_exp_ha_times(fleche_ctx* c, uint64_t* host,
+                                                                                    size_t n) {
+  if (!c || !host || !c->ha) return FLECHE_EINVAL;
+  if (c->have_last) cudaStreamSynchronize(c->last_stream);
+  memcpy(host, c->ha->exp_t, std::min(n, (size_t)64 * 2 * 64) * 8);
+  return FLECHE_OK;
+}
+// per staging block: [GPU wait start, GPU flag seen, GPU rows landed, GPU done, CPU published (REALTIME)]
+extern "C" __attribute__((visibility("default"))) fleche_status fleche_exp_ha_blocks(fleche_ctx* c, uint64_t* host,
+                                                                                     size_t nblk) {
+  if (!c || !host || !c->ha) return FLECHE_EINVAL;
+  if (c->have_last) cudaStreamSynchronize(c->last_stream);
+  const size_t m = std::min(nblk, (size_t)c->ha->blk_cap);
+  std::vector<uint64_t> g(m * 4);
+  if (cudaMemcpy(g.data(), c->dv.exp_blk, m * 4 * 8, cudaMemcpyDeviceToHost) != cudaSuccess) return FLECHE_ECUDA;
+  for (size_t k = 0; k < m; ++k) {
+    for (int j = 0; j < 4; ++j) host[k * 5 + j] = g[k * 4 + j];
+    host[k * 5 + 4] = c->ha->exp_pub[k];
+  }
+  return FLECHE_OK;
 }
 #endif

@@ -51,6 +51,8 @@ constexpr uint32_t kSlotMiss = 0xFFFFFFFFu, kSlotZero = 0xFFFFFFFEu;  // KQ -> K
 constexpr int kKmWarps = 4;     // KM CTA = 4 warps
 constexpr int kKmStageF4 = 256; // bytes layout, per warp: staged rows of a chunk (<= 4 KB) ...
 constexpr int kKmSmemF4 = 512;  // ... + the compaction buffer of one set region (<= 4 KB)
+constexpr int kHaBlock = 64;    // host-assisted miss fetch: rows per staging block (one ready flag)
+constexpr int kHaSmemF4 = 1024; // host-assisted KM, per warp: 16 KB of rows landed from the host
 
 enum Ctr : int {
   C_HITS = 0,
@@ -63,6 +65,8 @@ enum Ctr : int {
   C_BYPASSED,
   C_HOSTBYTES,
   C_DUPS,
+  C_HAROWS,     // host-assisted: unique misses read from the staging buffer
+  C_HATIMEOUT,  // host-assisted: staging blocks not ready in time (fetched zero-copy instead)
   kNumCtr = 16
 };
 
@@ -84,7 +88,9 @@ struct MissRec {  // one unique missed key (its owner lookup)
   uint32_t scr;   // scratch slot of the key (head of its duplicate chain)
   int32_t t;      // table
   int32_t pad;
+  uint64_t hst;   // host-assisted: float offset of the row's staging slot (kNoStage: read the table)
 };
+constexpr unsigned long long kNoStage = ~0ull;
 
 struct DupRec {  // a later occurrence of a missed key in the same batch
   int64_t off;   // float offset of the duplicate's row in `out`
@@ -96,9 +102,31 @@ struct Ctl {
   uint32_t epoch;  // current batch epoch (1-based); advanced by the last KM CTA
   uint32_t done;   // KM CTA arrival counter
   uint32_t err_invalid;
-  uint32_t pad;
+  uint32_t ha_rung;  // host-assisted: epoch whose doorbell KM has rung (warps poll host flags after it)
   uint32_t counts[2][8];  // [epoch & 1][class 0..5: unique misses; 7: duplicate misses]
+  unsigned long long ha_f[2];  // [epoch & 1] host-assisted staging floats allocated
   long long occ_bytes;    // row bytes currently cached
+};
+
+// Host-assisted miss fetch (FLECHE_FLAG_HOST_ASSIST).  The owner lane of each unique
+// miss in KQ writes (table, row, staging slot) to the request list in pinned host memory
+// at the miss's own miss-list index; KM's first thread rings a doorbell with the batch's
+// per-width miss counts (KQ's writes are complete by then: stream order).  Host threads gather the
+// requested rows into the contiguous pinned staging buffer, kHaBlock list indices at a
+// time, and publish a ready flag (= epoch) per block.  KM then takes whole blocks, waits
+// for each block's flag once and reads its staged rows (contiguous zero-copy: no per-row
+// address translation on the host link, the limit of the plain unified index on this
+// platform) instead of the scattered table rows.  A block not ready within the timeout
+// is fetched zero-copy from the tables as in the plain path, so a missing or slow host
+// thread costs time, never correctness.  Every area is double-buffered by epoch parity.
+struct HaReq {             // one request: (table << 48 | row), float offset of its staging slot
+  unsigned long long tid;
+  unsigned long long stage;  // kNoStage: no staging room this batch (KM reads the table row)
+};
+struct HaDesc {            // written by KM's first thread, read by the host threads
+  uint32_t epoch;
+  uint32_t cnt[8];         // unique misses of width class c (list indices off[c] .. off[c] + cnt[c])
+  uint32_t off[8];
 };
 
 struct Dev {
@@ -120,7 +148,7 @@ struct Dev {
   int32_t dim, admit_all;     // dim: row width of the uniform layout
   uint64_t admit_thr, admit_seed;
   int32_t prefetch;  // KQ starts each unique miss's host-row transfer into L2
-  int32_t km_m;      // unique misses per KM warp iteration (4, 8, 16, 32)
+  int32_t km_pad;
   int32_t bytes;     // 0 = uniform layout, 1 = bytes layout
   uint32_t set_units;  // bytes layout: region of a set in 32 B units (<= 256)
   int32_t part;      // static per-table partitions (HugeCTR-like baseline, NEXT-1)
@@ -132,10 +160,24 @@ struct Dev {
   int32_t ordered;
   int32_t pad2;
   uint64_t host_lo, host_mul;
+  // host-assisted miss fetch (mapped pinned host memory; see HaReq)
+  int32_t ha;                  // 1 = host-assisted miss fetch on
+  int32_t ha_pad;
+  HaReq* ha_req;               // [2][ha_req_cap]: indexed like the miss list
+  HaDesc* ha_desc;             // [2]
+  unsigned long long* ha_bell; // doorbell: epoch of the latest published descriptor
+  uint32_t* ha_ready;          // [2][ha_blk_cap] epoch of the block's staged rows
+  float* ha_stage;             // [2][ha_stage_floats]
+  uint32_t ha_req_cap, ha_blk_cap;
+  uint64_t ha_stage_floats;
+  uint64_t ha_timeout_ns;
 #ifdef FLECHE_EXPERIMENTS
   int32_t exp_mode;  // timing experiments only (libfleche_exp.so); breaks semantics
   int32_t exp_pad;
   unsigned long long* exp_buf;  // per KM warp: globaltimer at start / rows landed / end
+  uint32_t exp_slots;           // exp_buf[exp_slots]: KQ's doorbell time (host-assisted)
+  uint32_t exp_pad2;
+  unsigned long long* exp_blk;  // host-assisted KM, per staging block: wait start / flag seen / rows landed / done
 #endif
 };
 
@@ -249,6 +291,54 @@ __device__ __forceinline__ unsigned long long ld_cg_u64(const unsigned long long
 __device__ __forceinline__ void st_v4(float* p, float4 v) {
   asm volatile("st.global.v4.f32 [%0], {%1,%2,%3,%4};" ::"l"(p), "f"(v.x), "f"(v.y), "f"(v.z), "f"(v.w) : "memory");
 }
+// System-scope accesses to the host-assisted areas (written by host threads while the
+// kernel runs: strong loads, never a stale L1/L2 copy; the ready flag is an acquire).
+__device__ __forceinline__ uint32_t ld_acquire_sys_u32(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+// Staging rows: weak loads that coalesce into full-line link reads, but never hit a
+// stale L2 copy of system memory (.cv: discard a matching L2 line, fetch again); their
+// freshness w.r.t. the host's writes comes from the block's acquire of the ready flag.
+__device__ __forceinline__ float4 ld_cv_v4(const float* p) {
+  float4 v;
+  asm volatile("ld.global.cv.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_sys_u64(unsigned long long* p, unsigned long long v) {
+  asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ unsigned long long globaltimer_ns() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+// Poll of a host-written flag: .cv discards a matching (possibly stale) L2 copy of the
+// system-memory line and fetches it again over the link.
+__device__ __forceinline__ uint32_t ld_cv_u32(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.global.cv.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+// Wait (one lane) until a staging block carries this batch's epoch; false after timeout_ns.
+// First waits (in device memory) for KM's doorbell, so no host poll is in flight while the
+// doorbell's system fence drains; then polls the host flag (.cv loads) and takes one
+// acquire load once it matches.
+__device__ __forceinline__ bool ha_wait_block(const uint32_t* flag, const uint32_t* rung, uint32_t epoch,
+                                              unsigned long long timeout_ns) {
+  const unsigned long long t0 = globaltimer_ns();
+  while (*(const volatile uint32_t*)rung != epoch) {
+    __nanosleep(200);
+    if (globaltimer_ns() - t0 > timeout_ns) return false;
+  }
+  while (ld_cv_u32(flag) != epoch) {
+    __nanosleep(500);  // each poll is a host-link round trip: one poller per block
+    if (globaltimer_ns() - t0 > timeout_ns) return false;
+  }
+  return ld_acquire_sys_u32(flag) == epoch;
+}
+
 // Programmatic dependent launch (sm_90+): the batch's kernels are launched with
 // programmatic stream serialization, so a kernel's launch and prologue overlap the tail
 // of its predecessor; pdl_wait() (griddepcontrol.wait) then blocks until the
@@ -297,6 +387,28 @@ __device__ __forceinline__ void gather_rows(const float* src, float* dst, int la
 #pragma unroll
         for (int k = 0; k < VPL; ++k) st_v4(o[q] + 4 * (sub + k * LPR), v[q][k]);
       }
+  }
+}
+
+// Same copy with rows in shared memory (generic loads): row r of the warp at src[lane r].
+template <int D>
+__device__ __forceinline__ void copy_rows_generic(const float* src, float* dst, int lane) {
+  constexpr int VEC = D / 4;
+  constexpr int LPR = VEC < 32 ? VEC : 32;
+  constexpr int RPP = 32 / LPR;
+  constexpr int VPL = VEC / LPR;
+  constexpr int PASSES = 32 / RPP;
+  const int sub = lane % LPR, rs = lane / LPR;
+#pragma unroll 4
+  for (int p = 0; p < PASSES; ++p) {
+    const int r = p * RPP + rs;
+    const float* s = (const float*)__shfl_sync(kFull, (unsigned long long)src, r);
+    float* o = (float*)__shfl_sync(kFull, (unsigned long long)dst, r);
+    if (o) {
+#pragma unroll
+      for (int k = 0; k < VPL; ++k)
+        st_v4(o + 4 * (sub + k * LPR), *reinterpret_cast<const float4*>(s + 4 * (sub + k * LPR)));
+    }
   }
 }
 
@@ -510,9 +622,36 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
       uint32_t b = 0;
       if (kind == 1 && lane == leader) b = atomicAdd(&dv.ctl->counts[par][cls], (uint32_t)__popc(grp));
       b = __shfl_sync(kFull, b, leader);
+      uint64_t hst = kNoStage;
+      if (dv.ha && dv.bytes) {  // host-assisted, mixed widths: a staging slot (warp-aggregated)
+        const int myd = kind == 1 ? d : 0;
+        int incl = myd;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          const int y = __shfl_up_sync(kFull, incl, o);
+          if (lane >= o) incl += y;
+        }
+        const int tot = __shfl_sync(kFull, incl, 31);
+        unsigned long long f0 = 0;
+        if (lane == 0) f0 = atomicAdd(&dv.ctl->ha_f[par], (unsigned long long)tot);
+        f0 = __shfl_sync(kFull, f0, 0);
+        const uint64_t so = f0 + (uint64_t)(incl - myd);
+        if (kind == 1 && so + (uint64_t)d <= dv.ha_stage_floats) hst = so;
+      }
       if (kind == 1) {
-        dv.miss[qa.cls_off[cls] + b + __popc(grp & lt)] = MissRec{off, fk, scr, qa.t0 + t, 0};
+        const uint32_t r = b + __popc(grp & lt);
+        const int64_t li = qa.cls_off[cls] + r;  // miss-list index = request index
+        // uniform rows: the slot follows the list index (class regions are disjoint at
+        // ascending widths), so a block's staged rows are contiguous
+        if (dv.ha && !dv.bytes && (uint64_t)(li + 1) * (uint64_t)d <= dv.ha_stage_floats) hst = (uint64_t)li * d;
+        dv.miss[li] = MissRec{off, fk, scr, qa.t0 + t, 0, hst};
         dv.owner_off[scr] = off;
+#ifdef FLECHE_EXPERIMENTS
+        if (dv.exp_mode != 4)
+#endif
+        if (dv.ha)  // published by KM's doorbell (after this grid completes)
+          dv.ha_req[(size_t)par * dv.ha_req_cap + li] =
+              HaReq{((unsigned long long)(qa.t0 + t) << 48) | (unsigned long long)id, hst};
         if (dv.prefetch) {  // experimental: start the host-link transfer now
           const float* hrow = ti->host + (size_t)id * (size_t)d;
           asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(hrow), "r"(4u * (unsigned)d) : "memory");
@@ -657,7 +796,7 @@ __device__ __forceinline__ int64_t claim_victim(const Dev& dv, const TableInfo* 
 // first-fit, compacting the set's region through `cbuf` (set_units * 2 float4 of
 // smem) when free space is fragmented.  Returns false (bypass) if no candidate is
 // left; evictions already made stay made (as in the oracle's MODE_SETBYTES).
-__device__ bool bytes_insert(const Dev& dv, uint32_t fk, int units, const float4* row, uint32_t epoch, int lane,
+static __device__ bool bytes_insert(const Dev& dv, uint32_t fk, int units, const float4* row, uint32_t epoch, int lane,
                              unsigned& ev, long long& docc, float4* cbuf) {
   const uint32_t s = set_of(dv, fk);
   const int SU = (int)dv.set_units;
@@ -746,6 +885,146 @@ __device__ bool bytes_insert(const Dev& dv, uint32_t fk, int units, const float4
   if (lane == 0) atomicExch(lk, 0u);
   __syncwarp();
   return ok;
+}
+
+// Host-assisted KM for row width D (FLECHE_FLAG_HOST_ASSIST): warp gw takes whole
+// staging blocks (kHaBlock miss-list indices); lane 0 waits once for the block's ready
+// flag, then the warp pulls all of the block's rows over the host link at once
+// (ld.cv 16 B loads, 16 in flight per lane, into shared memory: two link round
+// trips per block instead of one per chunk) -- staged rows from the contiguous staging
+// buffer, rows without a staging slot (or after a timeout) from the tables -- and
+// places them 32 at a time (one row per lane: admission, victim claim, slab + out).
+template <bool BYTES, int D>
+__device__ __forceinline__ void km_ha(const Dev& dv, float* __restrict__ out, const MissRec* __restrict__ mlist,
+                                      uint32_t epoch, uint32_t nmiss, int lane, uint32_t gw, uint32_t nw, unsigned& ins,
+                                      unsigned& ev, unsigned& byp, long long& docc, unsigned long long& hostb,
+                                      float4* hsm, float4* cbuf, unsigned& harows, unsigned& hato) {
+  constexpr int VEC = D / 4;
+  constexpr int ROWS = (kHaSmemF4 / VEC) < kHaBlock ? (kHaSmemF4 / VEC) : kHaBlock;  // rows per piece
+  constexpr int PER_LANE = ROWS * VEC / 32;  // float4 per lane per piece
+  constexpr int INFL = PER_LANE < 16 ? PER_LANE : 16;
+  const uint32_t off = (uint32_t)(mlist - dv.miss);
+  const uint32_t kb0 = off / kHaBlock, kb1 = (off + nmiss - 1) / kHaBlock;
+  const uint32_t* flags = dv.ha_ready + (size_t)(epoch & 1u) * dv.ha_blk_cap;
+  const float* stage = dv.ha_stage + (size_t)(epoch & 1u) * dv.ha_stage_floats;
+  for (uint32_t kb = kb0 + gw; kb <= kb1; kb += nw) {
+    int ok = 0;
+#ifdef FLECHE_EXPERIMENTS
+    if (dv.exp_blk && lane == 0) dv.exp_blk[kb * 4 + 0] = globaltimer_ns();
+#endif
+    if (lane == 0) {
+      ok = ha_wait_block(flags + kb, &dv.ctl->ha_rung, epoch, dv.ha_timeout_ns);
+      if (!ok) ++hato;
+    }
+#ifdef FLECHE_EXPERIMENTS
+    if (dv.exp_blk && lane == 0) dv.exp_blk[kb * 4 + 1] = globaltimer_ns();
+#endif
+    ok = __shfl_sync(kFull, ok, 0);
+    const uint32_t blo = max(kb * kHaBlock, off) - off, bhi = min(kb * kHaBlock + kHaBlock, off + nmiss) - off;
+    for (uint32_t plo = blo; plo < bhi; plo += ROWS) {
+      const uint32_t n = min((uint32_t)ROWS, bhi - plo);
+      // the piece's miss records (row r on lane r % 32) and row sources
+      MissRec m[(ROWS + 31) / 32];
+      const float* src[(ROWS + 31) / 32];
+#pragma unroll
+      for (int h = 0; h < (ROWS + 31) / 32; ++h) {
+        const uint32_t r = h * 32 + lane;
+        src[h] = nullptr;
+        if (r < n) {
+          m[h] = mlist[plo + r];
+          const TableInfo* ti = dv.tables + m[h].t;
+          const bool st = ok && m[h].hst != kNoStage;
+          src[h] = st ? stage + m[h].hst : ti->host + (size_t)(m[h].fk - ti->base) * D;
+          if (st) ++harows;
+          hostb += 4ull * D;
+        }
+      }
+      // all rows of the piece over the link into shared memory
+#pragma unroll 1
+      for (int q0 = 0; q0 < PER_LANE; q0 += INFL) {
+        float4 v[INFL];
+#pragma unroll
+        for (int i = 0; i < INFL; ++i) {
+          const int q = (q0 + i) * 32 + lane, r = q / VEC, c = q % VEC;
+          const float* s0 = (const float*)__shfl_sync(kFull, (unsigned long long)src[0], r & 31);
+          const float* s1 = (ROWS > 32) ? (const float*)__shfl_sync(kFull, (unsigned long long)src[(ROWS + 31) / 32 - 1], r & 31)
+                                        : s0;
+          const float* sp = r < 32 ? s0 : s1;
+          v[i] = (r < (int)n && sp) ? ld_cv_v4(sp + 4 * c) : make_float4(0.f, 0.f, 0.f, 0.f);
+        }
+#pragma unroll
+        for (int i = 0; i < INFL; ++i) hsm[(q0 + i) * 32 + lane] = v[i];
+      }
+      __syncwarp();
+#ifdef FLECHE_EXPERIMENTS
+      if (dv.exp_blk && lane == 0 && plo == blo) dv.exp_blk[kb * 4 + 2] = globaltimer_ns();
+#endif
+      // place the rows, 32 at a time (lane = row)
+#pragma unroll
+      for (int h = 0; h < (ROWS + 31) / 32; ++h) {
+        const uint32_t r = h * 32 + lane;
+        const bool has = r < n;
+        const MissRec mm = has ? m[h] : MissRec{};
+        const float* row = (const float*)(hsm + (size_t)r * VEC);
+        bool admit = false;
+        if (has)
+          admit = dv.admit_all ||
+                  splitmix64(dv.admit_seed ^ (uint64_t)mm.fk ^ ((uint64_t)(epoch - 1u) << 32)) < dv.admit_thr;
+        if constexpr (!BYTES) {
+          bool pending = has && admit;
+          if (has && !admit) ++byp;
+          const TableInfo* ti = dv.tables + (has ? mm.t : 0);
+          const uint32_t pos = pending ? (uint32_t)ld_cg_u64(dv.firstpos + mm.scr) : 0u;
+          while (__any_sync(kFull, pending)) {
+            float* slab_dst = nullptr;
+            int64_t slot = kClaimRetry;
+            if (pending) {
+              uint32_t old_key = kEmpty;
+              bool took = false;
+              slot = claim_victim(dv, ti, mm.fk, epoch, pos, &old_key, &took);
+              if (slot >= 0) {
+                pending = false;
+                if (took) {
+                  ++byp;
+                } else {
+                  ++ins;
+                  docc += 4ll * D;
+                  if (old_key != kEmpty) { ++ev; docc -= 4ll * D; }
+                }
+                slab_dst = slot_row(dv, ti, (uint32_t)slot, D);
+              } else if (slot == kClaimBypass) {
+                pending = false;
+                ++byp;
+              }
+            }
+            copy_rows_generic<D>(row, slab_dst, lane);
+            if (slab_dst) {
+              dv.keys[slot] = mm.fk;
+              __threadfence();
+              *(volatile unsigned long long*)(dv.ipos + slot) = ((unsigned long long)epoch << 32) | ((unsigned long long)pos << 1);
+            }
+            if (slot == kClaimRetry && pending) __nanosleep(100);
+          }
+        } else {
+          for (int q = 0; q < 32; ++q) {  // inserts, one set lock at a time
+            if (!__shfl_sync(kFull, (int)has, q)) continue;
+            const uint32_t fk = __shfl_sync(kFull, mm.fk, q);
+            if (!__shfl_sync(kFull, (int)admit, q)) {
+              if (lane == 0) ++byp;
+              continue;
+            }
+            const bool okk = bytes_insert(dv, fk, D / 8, hsm + (size_t)(h * 32 + q) * VEC, epoch, lane, ev, docc, cbuf);
+            if (lane == 0) { if (okk) ++ins; else ++byp; }
+          }
+        }
+        copy_rows_generic<D>(row, has ? out + mm.off : nullptr, lane);  // the owner's output row
+      }
+      __syncwarp();
+    }
+#ifdef FLECHE_EXPERIMENTS
+    if (dv.exp_blk && lane == 0) dv.exp_blk[kb * 4 + 3] = globaltimer_ns();
+#endif
+  }
 }
 
 // KM for row width D: each warp iteration handles M unique misses of this class.
@@ -913,7 +1192,15 @@ __device__ __forceinline__ void km_rows(const Dev& dv, float* __restrict__ out, 
 #endif
 }
 
-template <bool BYTES>
+// Misses per KM warp iteration for a row width (the KM shape sweep was flat within
+// noise, profiles/README.md; these keep the rows of one iteration in registers)
+template <bool BYTES, int D>
+struct KmM {
+  static constexpr int value = D >= 256 ? 4 : (BYTES || D >= 64 ? 8 : 16);
+};
+
+// DU > 0: uniform layout of width DU (one class); DU = 0: every width class in turn.
+template <bool BYTES, int DU>
 __global__ void __launch_bounds__(128, 4) km_kernel(const __grid_constant__ Dev dv, const __grid_constant__ KMArgs ka) {
   __shared__ unsigned long long s_ctr[kNumCtr];
   extern __shared__ float4 s_dyn[];
@@ -923,41 +1210,64 @@ __global__ void __launch_bounds__(128, 4) km_kernel(const __grid_constant__ Dev 
   const uint32_t epoch = *(volatile uint32_t*)&dv.ctl->epoch;
   const int par = epoch & 1u;
   const int lane = threadIdx.x & 31;
+  if (dv.ha && blockIdx.x == 0 && threadIdx.x == 0) {
+    // host-assisted: ring the doorbell.  KQ (the previous grid in stream order) wrote the
+    // requests; this fence orders them before the doorbell for the host threads.
+    HaDesc hd;
+    hd.epoch = epoch;
+#pragma unroll
+    for (int c = 0; c < 8; ++c) {
+      hd.cnt[c] = c < ka.ncls ? *(volatile uint32_t*)&dv.ctl->counts[par][c] : 0u;
+      hd.off[c] = c < ka.ncls ? (uint32_t)ka.cls_off[c] : 0u;
+    }
+    dv.ha_desc[par] = hd;
+    __threadfence_system();  // before any warp polls the host (a system fence drains link traffic)
+    st_release_sys_u64(dv.ha_bell, (unsigned long long)epoch);
+    *(volatile uint32_t*)&dv.ctl->ha_rung = epoch;
+#ifdef FLECHE_EXPERIMENTS
+    if (dv.exp_buf) dv.exp_buf[dv.exp_slots] = globaltimer_ns();
+#endif
+  }
   // block-interleaved warp numbering: consecutive miss chunks land on different SMs,
   // so the host-link loads of a batch are spread over the whole GPU
   const uint32_t gw = (threadIdx.x >> 5) * gridDim.x + blockIdx.x;
   const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
-  float4* wsm = BYTES ? s_dyn + (threadIdx.x >> 5) * kKmSmemF4 : nullptr;
-  unsigned ins = 0, ev = 0, byp = 0;
+  // per warp: [kHaSmemF4 host-assisted rows][kKmSmemF4 bytes-layout staging + compaction]
+  const int wsm_f4 = (dv.ha ? kHaSmemF4 : 0) + (BYTES ? kKmSmemF4 : 0);
+  float4* hsm = s_dyn + (threadIdx.x >> 5) * wsm_f4;
+  float4* wsm = hsm + (dv.ha ? kHaSmemF4 : 0);
+  unsigned ins = 0, ev = 0, byp = 0, harows = 0, hato = 0;
   long long docc = 0;
   unsigned long long hostb = 0;
   for (int c = 0; c < ka.ncls; ++c) {
     const uint32_t nmiss = *(volatile uint32_t*)&dv.ctl->counts[par][c];
     if (!nmiss) continue;
     const MissRec* ml = dv.miss + ka.cls_off[c];
-#define FL_KM(D, M) km_rows<BYTES, D, M>(dv, ka.out, ml, epoch, nmiss, lane, gw, nw, ins, ev, byp, docc, hostb, wsm)
-#define FL_KM_MS(D)                    \
-  switch (dv.km_m) {                   \
-    case 4: FL_KM(D, 4); break;        \
-    case 16: FL_KM(D, 16); break;      \
-    case 32: FL_KM(D, 32); break;      \
-    default: FL_KM(D, 8); break;       \
-  }
-    switch (ka.cls_dim[c]) {  // fleche_create only admits these widths
-      case 8: FL_KM_MS(8); break;
-      case 16: FL_KM_MS(16); break;
-      case 32: FL_KM_MS(32); break;
-      case 64: FL_KM_MS(64); break;
-      case 128: if (dv.km_m <= 4) FL_KM(128, 4); else FL_KM(128, 8); break;
-      case 256: FL_KM(256, 4); break;
-      default: break;
+#define FL_KM(D)                                                                                              \
+  if (dv.ha)                                                                                                  \
+    km_ha<BYTES, D>(dv, ka.out, ml, epoch, nmiss, lane, gw, nw, ins, ev, byp, docc, hostb, hsm, wsm, harows, hato); \
+  else                                                                                                        \
+    km_rows<BYTES, D, KmM<BYTES, D>::value>(dv, ka.out, ml, epoch, nmiss, lane, gw, nw, ins, ev, byp, docc, hostb, wsm)
+    if constexpr (DU > 0) {
+      FL_KM(DU);
+    } else {
+      switch (ka.cls_dim[c]) {  // fleche_create only admits these widths
+        case 8: FL_KM(8); break;
+        case 16: FL_KM(16); break;
+        case 32: FL_KM(32); break;
+        case 64: FL_KM(64); break;
+        case 128: FL_KM(128); break;
+        case 256: FL_KM(256); break;
+        default: break;
+      }
     }
-#undef FL_KM_MS
 #undef FL_KM
   }
   ins = __reduce_add_sync(kFull, ins);
   ev = __reduce_add_sync(kFull, ev);
   byp = __reduce_add_sync(kFull, byp);
+  harows = __reduce_add_sync(kFull, harows);
+  hato = __reduce_add_sync(kFull, hato);
 #pragma unroll
   for (int o = 16; o; o >>= 1) {
     hostb += __shfl_xor_sync(kFull, hostb, o);
@@ -967,6 +1277,8 @@ __global__ void __launch_bounds__(128, 4) km_kernel(const __grid_constant__ Dev 
     if (ins) atomicAdd(&s_ctr[C_INSERTED], (unsigned long long)ins);
     if (ev) atomicAdd(&s_ctr[C_EVICTED], (unsigned long long)ev);
     if (byp) atomicAdd(&s_ctr[C_BYPASSED], (unsigned long long)byp);
+    if (harows) atomicAdd(&s_ctr[C_HAROWS], (unsigned long long)harows);
+    if (hato) atomicAdd(&s_ctr[C_HATIMEOUT], (unsigned long long)hato);
     if (hostb) atomicAdd(&s_ctr[C_HOSTBYTES], hostb);
     if (docc) atomicAdd((unsigned long long*)&dv.ctl->occ_bytes, (unsigned long long)docc);
   }
@@ -980,6 +1292,7 @@ __global__ void __launch_bounds__(128, 4) km_kernel(const __grid_constant__ Dev 
     if (prev == gridDim.x - 1) {  // last CTA closes the batch: next batch's counters, epoch + 1
 #pragma unroll
       for (int c = 0; c < 8; ++c) dv.ctl->counts[par ^ 1][c] = 0;
+      dv.ctl->ha_f[par ^ 1] = 0;
       dv.ctl->done = 0;
       __threadfence();
       *(volatile uint32_t*)&dv.ctl->epoch = epoch + 1u;
@@ -989,6 +1302,7 @@ __global__ void __launch_bounds__(128, 4) km_kernel(const __grid_constant__ Dev 
 
 // KD restore: every duplicate occurrence of a missed key copies its owner's
 // row (written by KM) in parallel.
+template <int = 0>
 __global__ void __launch_bounds__(128) kd_kernel(const __grid_constant__ Dev dv, float* __restrict__ out) {
   pdl_wait();
   // KM's last CTA already advanced the epoch: this batch is epoch - 1

@@ -125,6 +125,7 @@ __global__ void __launch_bounds__(128) kr_kernel(const __grid_constant__ RArgs<M
 
 // KPK: owner groups -> contiguous send buffer; counts out; the last CTA clears the
 // per-owner counters for the next batch.
+template <int = 0>
 __global__ void __launch_bounds__(256) kpk_kernel(const __grid_constant__ RouteDev rd, uint32_t* __restrict__ send_keys,
                                                   int64_t* __restrict__ send_counts) {
   __shared__ int64_t s_pre[kMaxWorld + 1];

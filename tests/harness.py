@@ -10,12 +10,12 @@ HASH_SEED = 0x9E3779B9
 
 
 def make_pair(w, tabs, mode=O.MODE_SETASSOC, max_lookups=None, admit_p=1.0, admit_seed=0, hash_seed=HASH_SEED,
-              cache_bytes=None):
+              cache_bytes=None, flags=0):
     import paper_conf_eurosys_xiellwgrs22_b200 as fl
     cb = w.cache_bytes if cache_bytes is None else cache_bytes
     if max_lookups is None:
         max_lookups = w.batch_size * w.n
-    gpu = fl.FlatCache(w.cards, w.dims, tabs, cb, max_lookups, 0, admit_p, admit_seed, hash_seed)
+    gpu = fl.FlatCache(w.cards, w.dims, tabs, cb, max_lookups, 0, admit_p, admit_seed, hash_seed, flags)
     orc = O.Oracle(w.cards, w.dims, tabs, cb, mode, admit_p, admit_seed, hash_seed)
     return gpu, orc
 

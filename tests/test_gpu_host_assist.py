@@ -1,0 +1,147 @@
+"""Host-assisted miss fetch (FLECHE_FLAG_HOST_ASSIST) vs the CPU oracle (needs a B200).
+
+The flag only changes WHERE a missed row is read from (a contiguous staging buffer the
+ctx's host threads fill, instead of the scattered table row): `out` must stay bit-exact
+and every counter of the cache policy exactly the set-associative oracle's, also when
+the staging/request capacity overflows (those rows go zero-copy) and when every block
+times out (the GPU fetches them itself).
+"""
+import numpy as np
+import pytest
+
+from oracle import oracle as O
+from tests import harness as H
+from workload import configs
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+
+import paper_conf_eurosys_xiellwgrs22_b200 as fl  # noqa: E402
+
+HA = fl.binding.FLAG_HOST_ASSIST
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _need_gpu():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+
+
+def _tables(w):
+    return [np.ascontiguousarray(t) for t in w.make_tables()[1]]
+
+
+def _run(w, tabs, batches, mode=O.MODE_SETASSOC, exact=True, **kw):
+    gpu, orc = H.make_pair(w, tabs, mode, flags=HA, **kw)
+    for b in range(batches):
+        bt = w.batch(b)
+        g0, o0 = gpu.stats(), orc.stats()
+        got = H.run_batch_gpu(gpu, bt.ids, torch)
+        ref = orc.query(bt.ids)
+        assert H.bits_equal(got, ref), (b, H.first_mismatch(got, ref, w.dims, [x.size for x in bt.ids]))
+        if exact:
+            dg, do = H.delta(g0, gpu.stats()), H.delta(o0, orc.stats())
+            for k in H.STAT_KEYS_EXACT:
+                assert dg[k] == do[k], (b, k, dg[k], do[k])
+    return gpu, orc
+
+
+@pytest.mark.parametrize("value_mode", [0, 1])
+def test_assisted_bit_exact_and_exact_stats(value_mode):
+    w = configs.get("cfg0").with_(value_mode=value_mode, invalid_ppm=5000, cache_frac=0.05)
+    gpu, _ = _run(w, _tables(w), 30)
+    st = gpu.stats()
+    # no timeouts at a 2 ms budget: every unique miss came through the staging buffer
+    assert st["assist_timeouts"] == 0, st
+    assert st["assisted_rows"] == st["unique_misses"] > 0
+
+
+def test_assisted_churn_no_stale_rows():
+    w = configs.get("cfg0").with_(skews=[0.5] * 7, cache_frac=0.002, batch_size=500)
+    tabs = _tables(w)
+    gpu, orc = _run(w, tabs, 60)
+    keys, _, slab = gpu.snapshot()
+    _, base, fb = gpu.encoding()
+    for way in np.nonzero(keys != 0xFFFFFFFF)[0]:
+        k = int(keys[way])
+        t = int(np.nonzero((base <= k) & (k < base + (1 << fb.astype(np.int64))))[0][0])
+        assert H.bits_equal(slab[way], tabs[t][k - int(base[t])])
+
+
+def test_assisted_overflow_goes_zero_copy(monkeypatch):
+    # 16 KB of staging per batch: most misses find no slot and are fetched zero-copy by
+    # KM (within the same blocks as staged ones); results and stats unchanged
+    monkeypatch.setenv("FLECHE_HA_STAGE_KB", "16")
+    w = configs.get("cfg0").with_(cache_frac=0.02, invalid_ppm=3000, skews=[0.7] * 7)
+    gpu, _ = _run(w, _tables(w), 20)
+    st = gpu.stats()
+    assert 0 < st["assisted_rows"] < st["unique_misses"]
+
+
+def test_assisted_timeouts_fall_back(monkeypatch):
+    # zero timeout: KM gives up on blocks that are not already staged and reads the
+    # table rows itself; the host threads keep writing (stale) blocks meanwhile
+    monkeypatch.setenv("FLECHE_HA_TIMEOUT_US", "0")
+    w = configs.get("cfg0").with_(cache_frac=0.02, skews=[0.7] * 7)
+    gpu, _ = _run(w, _tables(w), 25)
+    st = gpu.stats()
+    assert st["assisted_rows"] + st["assist_timeouts"] > 0
+
+
+def test_assisted_mixed_widths_pooled():
+    w = configs.get("cfg4")
+    w = w.with_(cards=[max(3, c // 64) for c in w.cards], batch_size=128, invalid_ppm=2000)
+    tabs = _tables(w)
+    gpu, glob = H.make_pair(w, tabs, O.MODE_GLOBAL, max_lookups=w.batch(0).lookups * 2, flags=HA)
+    for b in range(12):
+        bt = w.batch(b)
+        ids = [torch.from_numpy(x).cuda() for x in bt.ids]
+        offs = [torch.from_numpy(o).cuda() for o in bt.offsets]
+        n_out = gpu.pooled_floats([o.size - 1 for o in bt.offsets])
+        out = torch.full((max(n_out, 1),), float("nan"), device="cuda")
+        gpu.query_pooled(ids, offs, out)
+        torch.cuda.synchronize()
+        assert H.bits_equal(out[:n_out].cpu().numpy(), glob.query_pooled(bt.ids, bt.offsets)), b
+    st = gpu.stats()
+    assert st["assist_timeouts"] == 0 and st["assisted_rows"] == st["unique_misses"]
+
+
+def test_assisted_cuda_graph_replay():
+    # requests, doorbell and ready flags are epoch-tagged on the device: graph replays work
+    w = configs.get("cfg0")
+    tabs = _tables(w)
+    gpu, orc = H.make_pair(w, tabs, flags=HA)
+    lens = [w.batch_size] * w.n
+    ids_dev = [torch.zeros(L, dtype=torch.int64, device="cuda") for L in lens]
+    out = torch.zeros(gpu.out_floats(lens), device="cuda")
+    s = torch.cuda.Stream()
+    g = torch.cuda.CUDAGraph()
+    torch.cuda.synchronize()
+    with torch.cuda.graph(g, stream=s):
+        gpu.query(ids_dev, out, stream=s)
+    for b in range(8):
+        bt = w.batch(b)
+        for d, x in zip(ids_dev, bt.ids):
+            d.copy_(torch.from_numpy(x))
+        torch.cuda.synchronize()
+        g.replay()
+        torch.cuda.synchronize()
+        assert H.bits_equal(out.cpu().numpy(), orc.query(bt.ids)), b
+    assert gpu.stats()["assisted_rows"] == orc.stats()["unique_misses"]
+
+
+def test_assisted_cfg2_full_size():
+    # the bench's workload and launch configuration: 8.64 GB host tier, 212,992 lookups
+    # per batch; bit-exact, no timeouts, every unique miss staged by the host threads
+    w = configs.get("cfg2")
+    tabs = _tables(w)
+    gpu, glob = H.make_pair(w, tabs, O.MODE_GLOBAL, flags=HA)
+    for b in range(40):
+        bt = w.batch(b)
+        got = H.run_batch_gpu(gpu, bt.ids, torch)
+        ref = glob.query(bt.ids)
+        if b % 5 == 0 or b >= 35:
+            assert H.bits_equal(got, ref), b
+    st = gpu.stats()
+    assert st["assist_timeouts"] == 0 and st["assisted_rows"] == st["unique_misses"]
