@@ -50,6 +50,10 @@ def parse():
     p.add_argument("--host-assist", action="store_true",
                    help="FLECHE_FLAG_HOST_ASSIST: host threads stage the missed rows (paper Fig 8b CPU-DRAM layer)")
     p.add_argument("--cache-frac", type=float, default=None, help="override the config's cache fraction (sweeps)")
+    p.add_argument("--watermarks", default=None,
+                   help="hi,lo: full-scan eviction between these fractions of capacity (P:L660-662, reading R23)")
+    p.add_argument("--ha-frac", type=float, default=None,
+                   help="--host-assist: share of the miss blocks the host threads stage (rest: zero-copy)")
     p.add_argument("--admit-prob", type=float, default=1.0, help="admission probability p (P:L655-659); 1 = canonical")
     p.add_argument("--mode", default="replicated", choices=["replicated", "sharded"],
                    help="multi-GPU partitioning: per-GPU replicated caches, or one key-sharded cache (NCCL all-to-all)")
@@ -231,6 +235,8 @@ def main():
     W, K = max(args.warmup, 0), max(args.steps, 1)
     if args.host_assist:
         args.flags |= 0x8
+        if args.ha_frac is not None:
+            os.environ["FLECHE_HA_FRAC"] = str(args.ha_frac)
     if args.impl == "reference":
         return run_reference(args, w, P, W, K)
 
@@ -266,6 +272,10 @@ def main():
     from workload import gen as _gen
     cache = fl.FlatCache(w.cards, w.dims, tabs, w.cache_bytes, N * (world if sharded else 1), local,
                          args.admit_prob, _gen.seeds()["admit"], HASH_SEED, args.flags)
+    wm = None
+    if args.watermarks:
+        wm = [float(x) for x in args.watermarks.split(",")]
+        cache.set_watermarks(wm[0], wm[1])
     shard = None
     if sharded:
         if dist is None:
@@ -438,8 +448,16 @@ def main():
         kd["frac"] = kd["achieved"] / kd["peak"]
     dom = max(kern, key=lambda k: kern[k]["ms"])
     kd = kern[dom]
+    traffic, traffic_src = None, None
+    try:  # committed ncu --set full summary of this config's kernels (profiles/ncu_traffic_r01.json)
+        tr = json.load(open(os.path.join(os.path.dirname(os.path.abspath(__file__)), "profiles",
+                                         "ncu_traffic_r01.json")))[args.config][dom]
+        if not args.flags and not args.watermarks:
+            traffic, traffic_src = tr["dram_bytes"], tr["source"]
+    except (OSError, KeyError, ValueError):
+        pass
     roof = {"bound": kd["bound"], "achieved": kd["achieved"], "peak": kd["peak"], "unit": "GB/s", "frac": kd["frac"],
-            "traffic": None, "kernel": dom, "kernel_ms": kd["ms"], "share_of_step": kd["ms"] / (kq_avg + ki_avg),
+            "traffic": traffic, "traffic_source": traffic_src, "kernel": dom, "kernel_ms": kd["ms"], "share_of_step": kd["ms"] / (kq_avg + ki_avg),
             "peak_source": kd["peak_source"], "host_link_1GiB_gbs": host_link,
             "frac_of_link_bw": kern["km_kernel"]["achieved"] / host_link, "kernels": kern,
             "algorithmic_bytes_per_step": {"hbm": ab["kq_hbm"] + ab["km_hbm"] + ab["kd_hbm"] + ab["kp_hbm"], "host": ab["km_host"]}}
@@ -511,9 +529,12 @@ def main():
                                        (f"replicated x{world}" if world > 1 else "single GPU")),
                        "prefill_batches": P, "distinct_timed_batches": min(R, K), "admit_prob": args.admit_prob,
                        "miss_fetch": ("host-assisted: %s host threads stage the missed rows (FLECHE_FLAG_HOST_ASSIST)"
-                                      % os.environ.get("FLECHE_HA_THREADS", "12")) if ha else
+                                      % os.environ.get("FLECHE_HA_THREADS", "12")
+                                      + ", share %s of the blocks" % os.environ.get("FLECHE_HA_FRAC", "0.5")) if ha else
                                      "unified index: zero-copy reads of the host rows",
                        "flags": args.flags,
+                       "eviction": (f"full-scan between watermarks hi={wm[0]} lo={wm[1]} (reading R23)" if wm else
+                                    "on demand (canonical, reading R2)"),
                        "l2": "inputs larger than L2: fresh ID batch per step, 4 rotating output buffers "
                              f"({4 * out_max * 4 / 1e6:.0f} MB), {w.cache_bytes / 1e6:.0f} MB slab"},
             "hit_ratio": hit, "hit_ratio_unique": uhit,
@@ -521,7 +542,7 @@ def main():
             "p50_batch_latency_us": lat[len(lat) // 2], "p99_batch_latency_us": lat[int(len(lat) * 0.99) - 1],
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
             "assisted_rows_per_step": dst["assisted_rows"] / K, "assist_timeouts": dst["assist_timeouts"],
-            "gpu_launches": int(dst["kernels_launched"]), "clocks": clk,
+            "gpu_launches": int(dst["kernels_launched"]), "clocks": clk, "scans_per_step": dst["scans"] / K,
             "host_tier_gen_s": t_gen,
         }), flush=True)
     if dist:

@@ -133,6 +133,7 @@ typedef struct {
   uint64_t kernels_launched;   /* kernels this ctx launched                                         */
   uint64_t assisted_rows;      /* HOST_ASSIST: unique misses read from the host threads' staging    */
   uint64_t assist_timeouts;    /* HOST_ASSIST: staging blocks fetched zero-copy after the timeout   */
+  uint64_t scans;              /* fleche_set_watermarks: batches whose full-table scan evicted      */
 } fleche_stats_t;
 
 /* Create a cache for the tables in *cfg on cfg->device.  Allocates every device
@@ -183,6 +184,21 @@ fleche_status fleche_query_host(fleche_ctx* ctx, const int64_t* const* ids, cons
  * was seen since the last reset. */
 fleche_status fleche_stats(fleche_ctx* ctx, fleche_stats_t* out);
 fleche_status fleche_reset_stats(fleche_ctx* ctx);
+
+/* Watermark (full-scan) eviction, the paper's eviction trigger ("when the
+ * utilization of the memory pool exceeds a certain threshold, FC performs cache eviction
+ * with a full table scan and keeps evicting cold embeddings until memory utilization
+ * falls below another threshold"; no values are given).  Reading R23: after
+ * every later batch, if the cached row bytes exceed floor(hi * capacity_bytes), the ctx
+ * scans the whole index and evicts, oldest first, whole age classes (age = batches since
+ * the entry was last read or written, saturated at 4095) of the entries NOT touched in
+ * that batch (epoch-based reclamation), until the bytes are <=
+ * floor(lo * capacity_bytes) or no untouched entry is left.  On-demand eviction inside
+ * a full set stays as in the canonical policy.  hi >= 1 turns the scan off (default).
+ * Adds 2 kernel launches per batch (both exit at once below hi).  Blocks until the
+ * ctx's queued work is done.  FLECHE_EINVAL: hi or lo <= 0, lo > hi, or a
+ * FLECHE_FLAG_STATIC_PER_TABLE ctx. */
+fleche_status fleche_set_watermarks(fleche_ctx* ctx, double hi, double lo);
 
 /* Release every device buffer and host registration the ctx made. */
 fleche_status fleche_destroy(fleche_ctx* ctx);

@@ -55,6 +55,10 @@ def lib():
         L.or_query_pooled.argtypes = [vp, vp, vp, vp, vp]
         L.or_stats.restype = None
         L.or_stats.argtypes = [vp, ctypes.POINTER(_Stats)]
+        L.or_set_watermarks.restype = ctypes.c_int
+        L.or_set_watermarks.argtypes = [vp, u64, u64]
+        L.or_scans.restype = u64
+        L.or_scans.argtypes = [vp]
         L.or_cached_keys.restype = i64
         L.or_cached_keys.argtypes = [vp, vp, vp, i64]
         _lib = L
@@ -138,6 +142,16 @@ class Oracle:
             out = np.empty(self.out_size(bags), dtype=np.float32)
         lib().or_query_pooled(self.h, _ptr_array(ids), _ptr_array(offsets), bags.ctypes.data, out.ctypes.data)
         return out
+
+    def set_watermarks(self, hi_bytes: int, lo_bytes: int):
+        """Full-scan eviction after each batch (reading R23): if cached row
+        bytes > hi_bytes, evict whole age classes of untouched entries, oldest first,
+        until <= lo_bytes."""
+        if lib().or_set_watermarks(self.h, int(hi_bytes), int(lo_bytes)) != 0:
+            raise ValueError("lo_bytes > hi_bytes")
+
+    def scans(self) -> int:
+        return int(lib().or_scans(self.h))
 
     def stats(self) -> dict:
         s = _Stats()

@@ -34,7 +34,7 @@ class fleche_config(ctypes.Structure):
 
 STAT_FIELDS = ["batches", "lookups", "hits", "misses", "invalid", "unique_keys", "unique_hits", "unique_misses",
                "inserted", "evicted", "bypassed", "occupancy_bytes", "capacity_bytes", "index_bytes",
-               "host_bytes_fetched", "kernels_launched", "assisted_rows", "assist_timeouts"]
+               "host_bytes_fetched", "kernels_launched", "assisted_rows", "assist_timeouts", "scans"]
 
 
 class fleche_stats_t(ctypes.Structure):
@@ -75,13 +75,14 @@ fleche_query_keys = _sig("fleche_query_keys", ctypes.c_int, [_vp, _vp, _i64, _vp
 fleche_restore = _sig("fleche_restore", ctypes.c_int, [_vp, _vp, _vp, _vp, _vp])
 fleche_shard_stats = _sig("fleche_shard_stats", ctypes.c_int, [_vp, ctypes.POINTER(_u64), ctypes.POINTER(_u64),
                                                                ctypes.POINTER(_u64), ctypes.POINTER(_u64)])
+fleche_set_watermarks = _sig("fleche_set_watermarks", ctypes.c_int, [_vp, ctypes.c_double, ctypes.c_double])
 fleche_debug_locations = _sig("fleche_debug_locations", ctypes.c_int, [_vp, _vp, ctypes.c_size_t])
 
 EXPORTED = ["fleche_create", "fleche_query", "fleche_query_pooled", "fleche_query_host", "fleche_stats",
             "fleche_reset_stats", "fleche_destroy", "fleche_strerror", "fleche_get_encoding", "fleche_get_geometry",
             "fleche_debug_snapshot", "fleche_debug_locations", "fleche_set_profiling", "fleche_kernel_times",
             "fleche_probe_host_read", "fleche_route", "fleche_query_keys", "fleche_restore", "fleche_shard_stats",
-            "fleche_kernel_times_ex"]
+            "fleche_kernel_times_ex", "fleche_set_watermarks"]
 
 
 def probe_host_read(host_ptr: int, nbytes: int, row_bytes: int, rows: int, seed: int = 1, stream=None) -> float:
@@ -155,6 +156,11 @@ class FlatCache:
             self.close()
         except Exception:
             pass
+
+    def set_watermarks(self, hi: float, lo: float):
+        """Full-scan eviction between the watermarks hi/lo (fractions of capacity_bytes),
+        P:L660-662, reading R23; hi >= 1 turns it off."""
+        _check(fleche_set_watermarks(self.h, float(hi), float(lo)), "fleche_set_watermarks")
 
     def out_floats(self, lengths) -> int:
         return int(sum(int(l) * int(d) for l, d in zip(lengths, self.dims)))

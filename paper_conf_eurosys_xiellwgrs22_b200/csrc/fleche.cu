@@ -109,6 +109,11 @@ struct fleche_ctx {
   uint32_t repoch = 0;
   std::vector<int64_t> route_len;
   HostAssist* ha = nullptr;
+  // watermark (full-scan) eviction (fleche_set_watermarks; reading R23)
+  bool wm_on = false;
+  long long wm_hi = 0, wm_lo = 0;
+  unsigned long long* d_age_hist = nullptr;
+  int ke_blocks = 0;
 };
 
 namespace {
@@ -260,6 +265,7 @@ void ha_worker(HostAssist* h, int me) {
         hi_all = std::max<uint64_t>(hi_all, (uint64_t)d.off[c] + d.cnt[c]);
       }
     if (hi_all == 0 || hi_all > h->req_cap) continue;
+    const uint64_t kcut = d.kcut;  // blocks >= kcut: KM reads them from the tables itself
     auto src_of = [&](const HaReq& r, int32_t* dim) -> const float* {
       const int t = (int)(r.tid >> 48);
       const int64_t id = (int64_t)(r.tid & 0xFFFFFFFFFFFFull);
@@ -274,7 +280,7 @@ void ha_worker(HostAssist* h, int me) {
         for (int b = 0; b < dd * 4; b += 64) __builtin_prefetch((const char*)p + b, 0, 0);
     };
     const uint64_t kb0 = lo_all / kHaBlock, kb1 = (hi_all - 1) / kHaBlock;
-    for (uint64_t kb = kb0; kb <= kb1; ++kb) {
+    for (uint64_t kb = kb0; kb <= kb1 && kb < kcut; ++kb) {
       if (kb % (uint64_t)h->nthreads != (uint64_t)me) continue;
       bool any = false;
       for (int c = 0; c < 8; ++c) {  // the rows of every class region that overlaps block kb
@@ -333,7 +339,7 @@ void free_all(fleche_ctx* c) {
                   c->dv.firstpos, c->dv.ipos,
                   c->dv.miss, c->dv.dup, c->dv.ctl, c->dv.stats, c->d_tables, c->d_ids_stage, c->d_out_stage,
                   c->d_pool_stage, c->d_kdec, c->rd.scratch, c->rd.slotval, c->rd.inv, c->rd.region, c->rd.cnt,
-                  c->rd.prefix, c->rd.done, c->rd.stats, c->d_slots};
+                  c->rd.prefix, c->rd.done, c->rd.stats, c->d_slots, c->d_age_hist};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   for (auto& r : c->registered) cudaHostUnregister(r.first);
@@ -407,6 +413,16 @@ cudaError_t launch_k(int which, void (*kern)(KArgs...), unsigned grid, unsigned 
   return cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
 }
 
+// Watermark scan after a batch's KD (fleche_set_watermarks): KE1 + KE2, both exit at
+// once when the cached bytes are <= hi.
+void launch_scan(fleche_ctx* c, cudaStream_t s) {
+  if (!c->wm_on) return;
+  KEArgs ea{c->d_age_hist, c->wm_hi, c->wm_lo};
+  launch_k(kPdlKD, ke_hist_fn(), c->ke_blocks, 256, 0, s, c->dv, ea);
+  launch_k(kPdlKD, ke_evict_fn(), c->ke_blocks, 256, 0, s, c->dv, ea);
+  c->kernels += 2;
+}
+
 // KQ + KM for one batch of one-hot lookups into `out` (table-major rows).
 template <int MAXT>
 fleche_status launch_query(fleche_ctx* c, const int64_t* const* ids, const int64_t* lengths, float* out,
@@ -476,6 +492,7 @@ fleche_status launch_query(fleche_ctx* c, const int64_t* const* ids, const int64
   launch_k(kPdlKD, kd_fn(), c->kd_blocks, 128, 0, s, c->dv, out);
   c->kernels += 2;
   if (decouple) FL_CUDA(c, cudaStreamWaitEvent(s, c->join_ev, 0));  // join: out complete on s
+  launch_scan(c, s);
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return poison(c, e, "kernel launch");
@@ -779,6 +796,11 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
     dv.ha_blk_cap = h->blk_cap;
     dv.ha_stage_floats = h->stage_floats;
     dv.ha_timeout_ns = env_u("FLECHE_HA_TIMEOUT_US", 2000) * 1000ull;
+    {  // share of the staging blocks the host threads gather (the rest: KM's zero-copy reads)
+      const char* e = getenv("FLECHE_HA_FRAC");
+      const double f = e ? std::min(1.0, std::max(0.0, atof(e))) : 0.5;
+      dv.ha_frac_q16 = (uint32_t)(f * 65536.0 + 0.5);
+    }
     h->nt_stores = env_u("FLECHE_HA_NT", 1) != 0 && __builtin_cpu_supports("avx2");
     h->host.assign(cfg->host_tables, cfg->host_tables + n);
     h->card = c->card;
@@ -904,6 +926,7 @@ fleche_status fleche_stats(fleche_ctx* c, fleche_stats_t* out) {
   out->kernels_launched = c->kernels;
   out->assisted_rows = v[C_HAROWS];
   out->assist_timeouts = v[C_HATIMEOUT];
+  out->scans = v[C_SCANS];
   return ctl.err_invalid ? FLECHE_ERANGE : FLECHE_OK;
 }
 
@@ -975,6 +998,31 @@ fleche_status fleche_debug_locations(fleche_ctx* c, uint16_t* loc, size_t ways_c
   if (st != FLECHE_OK) return st;
   if (c->have_last) FL_CUDA(c, cudaStreamSynchronize(c->last_stream));
   FL_CUDA(c, cudaMemcpy(loc, c->dv.loc, ways * 2, cudaMemcpyDeviceToHost));
+  return FLECHE_OK;
+}
+
+fleche_status fleche_set_watermarks(fleche_ctx* c, double hi, double lo) {
+  if (!c) return FLECHE_EINVAL;
+  if (c->poisoned) return FLECHE_ESTATE;
+  if (!(hi > 0.0) || !(lo > 0.0) || lo > hi || c->dv.part) return FLECHE_EINVAL;
+  fleche_status st = ensure_device(c);
+  if (st != FLECHE_OK) return st;
+  if (c->have_last) FL_CUDA(c, cudaStreamSynchronize(c->last_stream));
+  if (hi >= 1.0) {  // never above capacity: the canonical on-demand policy
+    c->wm_on = false;
+    return FLECHE_OK;
+  }
+  if (!c->d_age_hist) {
+    FL_CUDA(c, cudaMalloc((void**)&c->d_age_hist, kAgeBins * 8));
+    FL_CUDA(c, cudaMemset(c->d_age_hist, 0, kAgeBins * 8));
+    FL_CUDA(c, cudaDeviceSynchronize());
+  }
+  const double cap = (double)c->capacity_bytes;
+  c->wm_hi = (long long)(hi * cap);
+  c->wm_lo = (long long)(lo * cap);
+  const int64_t quads = (int64_t)c->dv.sets * 8;
+  c->ke_blocks = (int)std::max<int64_t>(1, std::min<int64_t>((quads + 255) / 256, (int64_t)c->sm_count * 4));
+  c->wm_on = true;
   return FLECHE_OK;
 }
 
@@ -1080,6 +1128,7 @@ fleche_status launch_keys(fleche_ctx* c, const uint32_t* keys, int64_t count, fl
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
   launch_k(kPdlKD, kd_fn(), c->kd_blocks, 128, 0, s, c->dv, rows);
   c->kernels += 2;
+  launch_scan(c, s);
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return poison(c, e, "kernel launch");

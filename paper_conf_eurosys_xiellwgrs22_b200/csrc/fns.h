@@ -20,12 +20,15 @@ using KmFn = void (*)(Dev, KMArgs);
 using KdFn = void (*)(Dev, float*);
 using ProbeFn = void (*)(const float*, uint64_t, int64_t, uint64_t, float*);
 using KpkFn = void (*)(RouteDev, uint32_t*, int64_t*);
+using KeFn = void (*)(Dev, KEArgs);
 
 template <int MAXT> KqFn<MAXT> kq_fn();   // fused query (k_query.cu)
 template <int MAXT> KqFn<MAXT> kg_fn();   // decoupled hit copy (k_query.cu)
 template <int MAXT> KpFn<MAXT> kp_fn();   // pooling (k_query.cu)
 KmFn km_fn(bool bytes, int dim);          // miss kernel: bytes layout / uniform width dim / 0 = per class (k_miss.cu)
 KdFn kd_fn();                             // duplicate restore (k_misc.cu)
+KeFn ke_hist_fn();                        // watermark scan: age histogram (k_misc.cu)
+KeFn ke_evict_fn();                       // watermark scan: threshold + evict (k_misc.cu)
 ProbeFn probe_fn(int dim);                // host-link probe (k_misc.cu)
 template <int MAXT> KrFn<MAXT> kr_fn();   // key-sharded route (k_misc.cu)
 KpkFn kpk_fn();                           // key-sharded pack (k_misc.cu)

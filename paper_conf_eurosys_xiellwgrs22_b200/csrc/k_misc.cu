@@ -6,6 +6,8 @@
 namespace fl {
 
 KdFn kd_fn() { return kd_kernel<0>; }
+KeFn ke_hist_fn() { return ke_hist_kernel<0>; }
+KeFn ke_evict_fn() { return ke_evict_kernel<0>; }
 
 ProbeFn probe_fn(int dim) {
   switch (dim) {

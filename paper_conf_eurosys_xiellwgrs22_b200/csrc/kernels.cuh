@@ -67,6 +67,7 @@ enum Ctr : int {
   C_DUPS,
   C_HAROWS,     // host-assisted: unique misses read from the staging buffer
   C_HATIMEOUT,  // host-assisted: staging blocks not ready in time (fetched zero-copy instead)
+  C_SCANS,      // watermark eviction: batches whose full-table scan ran
   kNumCtr = 16
 };
 
@@ -106,6 +107,8 @@ struct Ctl {
   uint32_t counts[2][8];  // [epoch & 1][class 0..5: unique misses; 7: duplicate misses]
   unsigned long long ha_f[2];  // [epoch & 1] host-assisted staging floats allocated
   long long occ_bytes;    // row bytes currently cached
+  uint32_t ke_done;       // watermark eviction: KE2 CTA arrival counter
+  uint32_t ke_pad;
 };
 
 // Host-assisted miss fetch (FLECHE_FLAG_HOST_ASSIST).  The owner lane of each unique
@@ -127,6 +130,8 @@ struct HaDesc {            // written by KM's first thread, read by the host thr
   uint32_t epoch;
   uint32_t cnt[8];         // unique misses of width class c (list indices off[c] .. off[c] + cnt[c])
   uint32_t off[8];
+  uint32_t kcut;           // split: the host threads stage blocks < kcut, KM reads blocks >= kcut itself
+  uint32_t pad;
 };
 
 struct Dev {
@@ -171,6 +176,8 @@ struct Dev {
   uint32_t ha_req_cap, ha_blk_cap;
   uint64_t ha_stage_floats;
   uint64_t ha_timeout_ns;
+  uint32_t ha_frac_q16;        // share of the batch's staging blocks given to the host threads (x 2^-16)
+  uint32_t ha_pad2;
 #ifdef FLECHE_EXPERIMENTS
   int32_t exp_mode;  // timing experiments only (libfleche_exp.so); breaks semantics
   int32_t exp_pad;
@@ -337,6 +344,23 @@ __device__ __forceinline__ bool ha_wait_block(const uint32_t* flag, const uint32
     if (globaltimer_ns() - t0 > timeout_ns) return false;
   }
   return ld_acquire_sys_u32(flag) == epoch;
+}
+
+// Host-assisted split: the batch's miss list spans staging blocks [kb0, kb1]; the host
+// threads gather the first ceil(frac * nblocks) of them while KM's other warps read the
+// rest zero-copy from the tables at the same time (two independent paths to the rows:
+// host cores + contiguous link reads, and the GPU's own translated reads).
+__device__ __forceinline__ uint32_t ha_kcut(const Dev& dv, const KMArgs& ka, int par) {
+  uint32_t lo = 0xFFFFFFFFu, hi = 0;
+  for (int c = 0; c < ka.ncls; ++c) {
+    const uint32_t n = *(volatile uint32_t*)&dv.ctl->counts[par][c];
+    if (!n) continue;
+    lo = min(lo, (uint32_t)ka.cls_off[c]);
+    hi = max(hi, (uint32_t)ka.cls_off[c] + n);
+  }
+  if (hi == 0) return 0;
+  const uint32_t kb0 = lo / kHaBlock, nb = (hi - 1) / kHaBlock - kb0 + 1;
+  return kb0 + (uint32_t)(((unsigned long long)nb * dv.ha_frac_q16 + 65535ull) >> 16);
 }
 
 // Programmatic dependent launch (sm_90+): the batch's kernels are launched with
@@ -898,7 +922,7 @@ template <bool BYTES, int D>
 __device__ __forceinline__ void km_ha(const Dev& dv, float* __restrict__ out, const MissRec* __restrict__ mlist,
                                       uint32_t epoch, uint32_t nmiss, int lane, uint32_t gw, uint32_t nw, unsigned& ins,
                                       unsigned& ev, unsigned& byp, long long& docc, unsigned long long& hostb,
-                                      float4* hsm, float4* cbuf, unsigned& harows, unsigned& hato) {
+                                      float4* hsm, float4* cbuf, unsigned& harows, unsigned& hato, uint32_t kcut) {
   constexpr int VEC = D / 4;
   constexpr int ROWS = (kHaSmemF4 / VEC) < kHaBlock ? (kHaSmemF4 / VEC) : kHaBlock;  // rows per piece
   constexpr int PER_LANE = ROWS * VEC / 32;  // float4 per lane per piece
@@ -912,7 +936,7 @@ __device__ __forceinline__ void km_ha(const Dev& dv, float* __restrict__ out, co
 #ifdef FLECHE_EXPERIMENTS
     if (dv.exp_blk && lane == 0) dv.exp_blk[kb * 4 + 0] = globaltimer_ns();
 #endif
-    if (lane == 0) {
+    if (lane == 0 && kb < kcut) {  // the host threads' share; blocks >= kcut are read from the tables
       ok = ha_wait_block(flags + kb, &dv.ctl->ha_rung, epoch, dv.ha_timeout_ns);
       if (!ok) ++hato;
     }
@@ -1220,6 +1244,7 @@ __global__ void __launch_bounds__(128, 4) km_kernel(const __grid_constant__ Dev 
       hd.cnt[c] = c < ka.ncls ? *(volatile uint32_t*)&dv.ctl->counts[par][c] : 0u;
       hd.off[c] = c < ka.ncls ? (uint32_t)ka.cls_off[c] : 0u;
     }
+    hd.kcut = ha_kcut(dv, ka, par);
     dv.ha_desc[par] = hd;
     __threadfence_system();  // before any warp polls the host (a system fence drains link traffic)
     st_release_sys_u64(dv.ha_bell, (unsigned long long)epoch);
@@ -1238,6 +1263,7 @@ __global__ void __launch_bounds__(128, 4) km_kernel(const __grid_constant__ Dev 
   float4* wsm = hsm + (dv.ha ? kHaSmemF4 : 0);
   unsigned ins = 0, ev = 0, byp = 0, harows = 0, hato = 0;
   long long docc = 0;
+  const uint32_t kcut = dv.ha ? ha_kcut(dv, ka, par) : 0u;
   unsigned long long hostb = 0;
   for (int c = 0; c < ka.ncls; ++c) {
     const uint32_t nmiss = *(volatile uint32_t*)&dv.ctl->counts[par][c];
@@ -1245,7 +1271,7 @@ __global__ void __launch_bounds__(128, 4) km_kernel(const __grid_constant__ Dev 
     const MissRec* ml = dv.miss + ka.cls_off[c];
 #define FL_KM(D)                                                                                              \
   if (dv.ha)                                                                                                  \
-    km_ha<BYTES, D>(dv, ka.out, ml, epoch, nmiss, lane, gw, nw, ins, ev, byp, docc, hostb, hsm, wsm, harows, hato); \
+    km_ha<BYTES, D>(dv, ka.out, ml, epoch, nmiss, lane, gw, nw, ins, ev, byp, docc, hostb, hsm, wsm, harows, hato, kcut); \
   else                                                                                                        \
     km_rows<BYTES, D, KmM<BYTES, D>::value>(dv, ka.out, ml, epoch, nmiss, lane, gw, nw, ins, ev, byp, docc, hostb, wsm)
     if constexpr (DU > 0) {
@@ -1353,6 +1379,134 @@ __global__ void __launch_bounds__(256) kp_kernel(const __grid_constant__ PArgs<M
     acc.w = __fadd_rn(acc.w, x.w);
   }
   *reinterpret_cast<float4*>(pa.out + pa.out_off[t] + bag * 4 * vec + 4 * c) = acc;
+}
+
+// Watermark (full-scan) eviction, the paper's replacement trigger: "when the
+// utilization of the memory pool exceeds a certain threshold, FC performs cache eviction
+// with a full table scan and keeps evicting cold embeddings until memory utilization
+// falls below another threshold"; entries read in the current epoch are never reclaimed
+// (epoch-based reclamation).  Reading R23: checked once per batch
+// after its inserts; coldness = age class min(epoch - ts, kAgeBins - 1); whole classes
+// are evicted, oldest first, until the cached row bytes are <= lo.  Two launches after
+// KD: KE1 builds the byte histogram of age classes, KE2 picks the threshold class A (every
+// CTA redundantly, from the 32 KB histogram in L2) and evicts every untouched way of age
+// >= A.  Both exit at once when the bytes are <= hi, so an idle scan costs two launches.
+constexpr int kAgeBins = 4096;  // ages saturate at 4095 batches (reading R23)
+
+struct KEArgs {
+  unsigned long long* hist;  // [kAgeBins] row bytes per age class (zero between scans)
+  long long hi, lo;          // watermarks in row bytes
+};
+
+__device__ __forceinline__ uint32_t way_units(const Dev& dv, size_t i) {  // row bytes / 32
+  return dv.bytes ? (uint32_t)(ld_cg_u16(dv.loc + i) >> 8) : (uint32_t)(dv.dim >> 3);
+}
+
+template <int = 0>
+__global__ void __launch_bounds__(256) ke_hist_kernel(const __grid_constant__ Dev dv, const __grid_constant__ KEArgs ea) {
+  __shared__ uint32_t h[kAgeBins];  // 32-byte units per age class
+  for (int i = threadIdx.x; i < kAgeBins; i += blockDim.x) h[i] = 0;
+  __syncthreads();
+  pdl_wait();
+  const uint32_t epoch = *(volatile uint32_t*)&dv.ctl->epoch - 1u;  // KM advanced it
+  const long long occ = *(volatile long long*)&dv.ctl->occ_bytes;
+  if (occ <= ea.hi) {
+    pdl_trigger();
+    return;
+  }
+  const size_t quads = (size_t)dv.sets * 8u;  // 4 ways per thread step (16 B of keys + ts)
+  for (size_t q = (size_t)blockIdx.x * blockDim.x + threadIdx.x; q < quads; q += (size_t)gridDim.x * blockDim.x) {
+    const uint4 k = ld_cg_v4u(dv.keys + 4 * q), t = ld_cg_v4u(dv.ts + 4 * q);
+    const uint32_t kk[4] = {k.x, k.y, k.z, k.w}, tt[4] = {t.x, t.y, t.z, t.w};
+#pragma unroll
+    for (int j = 0; j < 4; ++j)
+      if (kk[j] != kEmpty && tt[j] < epoch)
+        atomicAdd(&h[min(epoch - tt[j], (uint32_t)(kAgeBins - 1))], way_units(dv, 4 * q + j));
+  }
+  __syncthreads();
+  pdl_trigger();
+  for (int i = threadIdx.x; i < kAgeBins; i += blockDim.x)
+    if (h[i]) atomicAdd(ea.hist + i, 32ull * h[i]);
+}
+
+template <int = 0>
+__global__ void __launch_bounds__(256) ke_evict_kernel(const __grid_constant__ Dev dv, const __grid_constant__ KEArgs ea) {
+  __shared__ unsigned long long sh[kAgeBins];
+  __shared__ unsigned long long part[256];
+  __shared__ uint32_t sA;
+  __shared__ int s_last;
+  pdl_wait();
+  const uint32_t epoch = *(volatile uint32_t*)&dv.ctl->epoch - 1u;
+  const long long occ = *(volatile long long*)&dv.ctl->occ_bytes;
+  if (occ <= ea.hi) {
+    pdl_trigger();
+    return;
+  }
+  // threshold: the largest class A with S(A) = sum_{a >= A} bytes(a) >= occ - lo, else 1
+  // (the oracle's loop "oldest class first while bytes > lo")
+  const unsigned long long need = (unsigned long long)(occ - ea.lo);
+  constexpr int kPer = kAgeBins / 256;
+  unsigned long long mine = 0;
+  for (int i = 0; i < kPer; ++i) {
+    const int a = threadIdx.x * kPer + i;
+    sh[a] = ld_cg_u64(ea.hist + a);
+    mine += sh[a];
+  }
+  part[threadIdx.x] = mine;
+  if (threadIdx.x == 0) sA = 1;
+  __syncthreads();
+  if (threadIdx.x == 0) {  // inclusive suffix sums of the 256 partials
+    unsigned long long run = 0;
+    for (int j = 255; j >= 0; --j) {
+      run += part[j];
+      part[j] = run;
+    }
+  }
+  __syncthreads();
+  unsigned long long S = threadIdx.x < 255 ? part[threadIdx.x + 1] : 0ull;
+  if (S < need) {
+    for (int a = threadIdx.x * kPer + kPer - 1; a >= threadIdx.x * kPer && a >= 1; --a) {
+      S += sh[a];
+      if (S >= need) {
+        atomicMax(&sA, (uint32_t)a);
+        break;
+      }
+    }
+  }
+  __syncthreads();
+  const uint32_t A = sA;
+  pdl_trigger();
+  unsigned ev = 0;
+  unsigned long long units = 0;
+  const size_t ways = (size_t)dv.sets * 32u;
+  for (size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x; i < ways; i += (size_t)gridDim.x * blockDim.x) {
+    const uint32_t k = ld_cg_u32(dv.keys + i), t = ld_cg_u32(dv.ts + i);
+    if (k == kEmpty || t >= epoch || min(epoch - t, (uint32_t)(kAgeBins - 1)) < A) continue;
+    units += way_units(dv, i);
+    dv.keys[i] = kEmpty;
+    dv.ts[i] = 0;
+    ++ev;
+  }
+  ev = __reduce_add_sync(kFull, ev);
+#pragma unroll
+  for (int o = 16; o; o >>= 1) units += __shfl_xor_sync(kFull, units, o);
+  if ((threadIdx.x & 31) == 0 && ev) {
+    atomicAdd(dv.stats + (blockIdx.x % kStripes) * kNumCtr + C_EVICTED, (unsigned long long)ev);
+    atomicAdd((unsigned long long*)&dv.ctl->occ_bytes, (unsigned long long)(-(long long)(32ull * units)));
+  }
+  // the last CTA (every CTA has read the histogram by then) clears it for the next scan
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    const uint32_t prev = atomicAdd(&dv.ctl->ke_done, 1u);
+    s_last = prev == gridDim.x - 1;
+    if (s_last) atomicAdd(dv.stats + C_SCANS, 1ull);
+  }
+  __syncthreads();
+  if (s_last) {
+    for (int i = threadIdx.x; i < kAgeBins; i += blockDim.x) ea.hist[i] = 0;
+    if (threadIdx.x == 0) dv.ctl->ke_done = 0;
+  }
 }
 
 // Host-link probe: the miss-fetch access pattern (one row per lane, 16-byte vector

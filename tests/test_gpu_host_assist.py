@@ -28,6 +28,12 @@ def _need_gpu():
         pytest.skip("no CUDA device")
 
 
+@pytest.fixture(autouse=True)
+def _all_blocks_to_host(monkeypatch):
+    # the tests below check the staged path itself: the host threads take every block
+    monkeypatch.setenv("FLECHE_HA_FRAC", "1")
+
+
 def _tables(w):
     return [np.ascontiguousarray(t) for t in w.make_tables()[1]]
 
@@ -145,3 +151,18 @@ def test_assisted_cfg2_full_size():
             assert H.bits_equal(got, ref), b
     st = gpu.stats()
     assert st["assist_timeouts"] == 0 and st["assisted_rows"] == st["unique_misses"]
+
+
+@pytest.mark.parametrize("frac", ["0.5", "0.25", "0"])
+def test_split_between_host_threads_and_zero_copy(monkeypatch, frac):
+    """FLECHE_HA_FRAC < 1: the host threads stage the first share of the batch's blocks
+    while KM reads the rest zero-copy; values and every counter stay exact."""
+    monkeypatch.setenv("FLECHE_HA_FRAC", frac)
+    w = configs.get("cfg0").with_(cache_frac=0.25, batch_size=2048)
+    gpu, orc = _run(w, _tables(w), 8)
+    st = gpu.stats()
+    assert st["assist_timeouts"] == 0, st
+    if frac == "0":
+        assert st["assisted_rows"] == 0
+    else:
+        assert 0 < st["assisted_rows"] < st["unique_misses"], st

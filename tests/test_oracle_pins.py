@@ -292,3 +292,114 @@ def test_small_cache_steady_state_matches_che():
     ref = che.che_hit(w.cards, w.skews, w.cache_bytes // 32)
     h, _ = _window_hit(w, O.MODE_GLOBAL, 150, 150)
     assert abs(h - ref) < 0.01, (h, ref)
+
+
+# ------------------------------------------- watermark (full-scan) eviction, reading R23
+def _run_wm_example(ex, mode):
+    tabs = _tiny_tables(ex["cards"], ex["dims"])
+    o = O.Oracle(ex["cards"], ex["dims"], tabs, ex["cache_bytes"], mode)
+    o.set_watermarks(ex["hi_bytes"], ex["lo_bytes"])
+    prev, ev0 = set(), 0
+    for bt in ex["batches"]:
+        before, scans0 = o.stats(), o.scans()
+        o.query([np.array(x, np.int64) for x in bt["ids"]])
+        s = o.stats()
+        assert s["hits"] - before["hits"] == bt["hits"]
+        assert s["occupancy_bytes"] == bt["occupancy"]
+        assert (o.scans() - scans0 == 1) == bt["scan"]
+        now = set(map(tuple, o.cached_keys()))
+        assert prev - now == set(map(tuple, bt["evicted"]))
+        prev = now
+    assert prev == set(map(tuple, ex["final_cached"]))
+    assert o.stats()["evicted"] - ev0 == ex["total_evicted"]
+
+
+@pytest.mark.parametrize("name,mode", [("A", O.MODE_GLOBAL), ("B", O.MODE_GLOBAL), ("B", O.MODE_SETASSOC)])
+def test_watermark_hand_examples(name, mode):
+    """Catches: scanning before the inserts, evicting entries touched in the batch, evicting
+    youngest-first, stopping one class early/late, a > vs >= on either watermark."""
+    g = json.load(open(os.path.join(GOLD, "watermark_examples.json")))
+    _run_wm_example(next(e for e in g["examples"] if e["name"] == name), mode)
+
+
+def test_watermark_at_capacity_is_the_canonical_policy():
+    """hi = capacity never triggers a scan (on-demand eviction keeps bytes <= capacity):
+    the variant must reduce to the canonical policy exactly."""
+    w = configs.get("cfg0").with_(cache_frac=0.05)
+    tabs = [np.ascontiguousarray(t) for t in w.make_tables()[1]]
+    a = O.Oracle(w.cards, w.dims, tabs, w.cache_bytes, O.MODE_GLOBAL)
+    b = O.Oracle(w.cards, w.dims, tabs, w.cache_bytes, O.MODE_GLOBAL)
+    b.set_watermarks(w.cache_bytes, w.cache_bytes // 2)
+    for k in range(30):
+        bt = w.batch(k)
+        a.query(bt.ids)
+        b.query(bt.ids)
+    assert a.stats() == b.stats() and b.scans() == 0
+
+
+def test_watermark_scan_is_cold_first_and_minimal():
+    """Property against ages taken from the TRACE (last batch each key was looked up in),
+    not from the oracle's state: with room for a whole batch above hi (no on-demand
+    eviction), a scan happens iff bytes after the inserts exceed hi; it evicts keys strictly
+    older than every untouched survivor, leaves bytes <= lo unless only touched keys remain,
+    and evicting one class fewer would have left bytes > lo."""
+    cards, dims = [300, 200], [4, 4]
+    row = 16
+    rng = np.random.default_rng(7)
+    tabs = _tiny_tables(cards, dims)
+    cap = 400 * row
+    hi, lo = 150 * row, 100 * row  # each batch has <= 60 unique keys: cap - hi >> 60 rows
+    o = O.Oracle(cards, dims, tabs, cap, O.MODE_GLOBAL)
+    o.set_watermarks(hi, lo)
+    last = {}
+    prev = set()
+    nscan = 0
+    for b in range(200):
+        ids = [np.minimum(rng.zipf(1.3, 30) - 1, c - 1).astype(np.int64) for c in cards]
+        keys = {(t, int(i)) for t, x in enumerate(ids) for i in x}
+        before, s0 = o.stats(), o.scans()
+        o.query(ids)
+        s = o.stats()
+        for k in keys:
+            last[k] = b
+        now = set(map(tuple, o.cached_keys()))
+        evicted = prev - now
+        after_inserts = before["occupancy_bytes"] + row * (s["inserted"] - before["inserted"])
+        scanned = o.scans() - s0 == 1
+        assert scanned == (after_inserts > hi)
+        if not scanned:
+            assert not evicted
+        else:
+            nscan += 1
+            assert s["occupancy_bytes"] == after_inserts - row * len(evicted)
+            untouched = [k for k in now if k not in keys]
+            if untouched:
+                assert s["occupancy_bytes"] <= lo
+                assert max(last[k] for k in evicted) < min(last[k] for k in untouched)  # strictly older
+            youngest = max(last[k] for k in evicted)
+            assert s["occupancy_bytes"] + row * sum(1 for k in evicted if last[k] == youngest) > lo
+        prev = now
+    assert nscan >= 10
+
+
+def test_watermark_setassoc_agrees_with_global_without_overflow():
+    """The set-associative mirror evicts by the same whole-age-class rule: while no set fills
+    up (hi at 1/8 of the capacity), its hits and evictions equal the global mode's."""
+    cards = [1000, 700, 500]
+    dims = [8, 8, 8]
+    tabs = _tiny_tables(cards, dims)
+    cap = 32 * 64 * 32  # 64 sets of 32 ways, 32 B rows
+    g = O.Oracle(cards, dims, tabs, cap, O.MODE_GLOBAL)
+    s = O.Oracle(cards, dims, tabs, cap, O.MODE_SETASSOC, hash_seed=11)
+    for o in (g, s):
+        o.set_watermarks(cap // 8, cap // 16)
+    rng = np.random.default_rng(3)
+    for b in range(150):
+        ids = [np.minimum(rng.zipf(1.2, 40) - 1, c - 1).astype(np.int64) for c in cards]
+        g.query(ids)
+        s.query(ids)
+    sg, ss = g.stats(), s.stats()
+    assert g.scans() > 10
+    for k in ("hits", "inserted", "evicted", "occupancy_bytes"):
+        assert sg[k] == ss[k], k
+    assert g.scans() == s.scans()
