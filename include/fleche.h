@@ -112,6 +112,13 @@ typedef struct {
  * 131072; rows beyond it are read zero-copy).  Not with PER_TABLE_LAUNCH (FLECHE_EINVAL).  `out`, hits and every cache decision are identical with and without
  * it; only where the missed rows are read from changes. */
 #define FLECHE_FLAG_HOST_ASSIST 0x8u
+/* FUSED_HIT_COPY: the query kernel copies each hit row itself (probe and copy in one
+ * kernel, the fused design) instead of the default for uniform layouts with >= 512K
+ * lookups per batch: the decoupled copy (Fig 8b), where the query kernel only
+ * indexes and a copy kernel on a side stream moves the hit rows while the miss kernel
+ * fetches the misses.  The paper's decoupling on/off comparison (Exp #7).
+ * `out` and every counter are identical either way. */
+#define FLECHE_FLAG_FUSED_HIT_COPY 0x10u
 
 typedef struct {
   uint64_t batches;            /* query calls                                                       */
@@ -155,6 +162,13 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out);
  * kernels and never blocks the host. */
 fleche_status fleche_query(fleche_ctx* ctx, const int64_t* const* ids, const int64_t* lengths, float* out,
                            fleche_stream stream);
+
+/* Warm start (the paper warms the cache by first issuing requests): one
+ * batch of one-hot lookups exactly as fleche_query (same policy, same counters: it is a
+ * batch of the cache), whose rows go to a ctx-owned scratch buffer (allocated at the
+ * first call, grown when a larger batch comes) instead of a caller buffer.  ids / lengths
+ * as in fleche_query.  Asynchronous. */
+fleche_status fleche_prefill(fleche_ctx* ctx, const int64_t* const* ids, const int64_t* lengths, fleche_stream stream);
 
 /* One batch of multi-hot lookups with sum pooling per bag (pooling).
  *   ids[t]     : DEVICE pointer to nnz[t] int64 IDs of table t (all bags, concatenated).

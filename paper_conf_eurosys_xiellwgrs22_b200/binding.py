@@ -20,7 +20,7 @@ _lib = ctypes.CDLL(LIB_PATH)
 
 OK, EINVAL, ENOMEM, ECUDA, ENCCL, ERANGE, ESTATE = 0, -1, -2, -3, -4, -5, -6
 FLAG_L2_PREFETCH = 0x1
-FLAG_STATIC_PER_TABLE, FLAG_PER_TABLE_LAUNCH, FLAG_HOST_ASSIST = 0x2, 0x4, 0x8
+FLAG_STATIC_PER_TABLE, FLAG_PER_TABLE_LAUNCH, FLAG_HOST_ASSIST, FLAG_FUSED_HIT_COPY = 0x2, 0x4, 0x8, 0x10
 MAX_TABLES = 512
 
 _vp, _i64, _i32, _u64, _u32 = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32, ctypes.c_uint64, ctypes.c_uint32
@@ -50,6 +50,7 @@ def _sig(name, res, args):
 
 fleche_create = _sig("fleche_create", ctypes.c_int, [ctypes.POINTER(fleche_config), ctypes.POINTER(_vp)])
 fleche_query = _sig("fleche_query", ctypes.c_int, [_vp, _vp, _vp, _vp, _vp])
+fleche_prefill = _sig("fleche_prefill", ctypes.c_int, [_vp, _vp, _vp, _vp])
 fleche_query_host = _sig("fleche_query_host", ctypes.c_int, [_vp, _vp, _vp, _vp, _vp])
 fleche_stats = _sig("fleche_stats", ctypes.c_int, [_vp, ctypes.POINTER(fleche_stats_t)])
 fleche_reset_stats = _sig("fleche_reset_stats", ctypes.c_int, [_vp])
@@ -82,7 +83,7 @@ EXPORTED = ["fleche_create", "fleche_query", "fleche_query_pooled", "fleche_quer
             "fleche_reset_stats", "fleche_destroy", "fleche_strerror", "fleche_get_encoding", "fleche_get_geometry",
             "fleche_debug_snapshot", "fleche_debug_locations", "fleche_set_profiling", "fleche_kernel_times",
             "fleche_probe_host_read", "fleche_route", "fleche_query_keys", "fleche_restore", "fleche_shard_stats",
-            "fleche_kernel_times_ex", "fleche_set_watermarks"]
+            "fleche_kernel_times_ex", "fleche_set_watermarks", "fleche_prefill"]
 
 
 def probe_host_read(host_ptr: int, nbytes: int, row_bytes: int, rows: int, seed: int = 1, stream=None) -> float:
@@ -172,6 +173,14 @@ class FlatCache:
         lp = (_i64 * self.n)(*lengths)
         ip = (_vp * self.n)(*[_ptr(x) for x in ids])
         _check(fleche_query(self.h, ip, lp, _ptr(out), _stream_handle(stream)), "fleche_query")
+
+    def prefill(self, ids, stream=None, lengths=None):
+        """Warm start: one batch of lookups through the cache, rows discarded."""
+        if lengths is None:
+            lengths = [int(x.numel()) for x in ids]
+        lp = (_i64 * self.n)(*lengths)
+        ip = (_vp * self.n)(*[_ptr(x) for x in ids])
+        _check(fleche_prefill(self.h, ip, lp, _stream_handle(stream)), "fleche_prefill")
 
     def pooled_floats(self, bags) -> int:
         return int(sum(int(b) * int(d) for b, d in zip(bags, self.dims)))

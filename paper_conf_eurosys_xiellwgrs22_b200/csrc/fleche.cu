@@ -84,7 +84,7 @@ struct fleche_ctx {
   cudaStream_t side = nullptr;
   cudaEvent_t fork_ev = nullptr, join_ev = nullptr;
   uint32_t* d_slots = nullptr;
-  int64_t decouple_min = 65536;  // lookups per batch from which the hit copy is decoupled
+  int64_t decouple_min = 524288;  // lookups per batch from which the hit copy is decoupled (cfg2: equal, cfg5: +5 %)
   size_t km_smem = 0;
   // host-side counters
   uint64_t batches = 0, lookups = 0, kernels = 0;
@@ -114,6 +114,9 @@ struct fleche_ctx {
   long long wm_hi = 0, wm_lo = 0;
   unsigned long long* d_age_hist = nullptr;
   int ke_blocks = 0;
+  // fleche_prefill scratch output (lazy)
+  float* d_prefill_out = nullptr;
+  int64_t prefill_floats = 0;
 };
 
 namespace {
@@ -339,7 +342,7 @@ void free_all(fleche_ctx* c) {
                   c->dv.firstpos, c->dv.ipos,
                   c->dv.miss, c->dv.dup, c->dv.ctl, c->dv.stats, c->d_tables, c->d_ids_stage, c->d_out_stage,
                   c->d_pool_stage, c->d_kdec, c->rd.scratch, c->rd.slotval, c->rd.inv, c->rd.region, c->rd.cnt,
-                  c->rd.prefix, c->rd.done, c->rd.stats, c->d_slots, c->d_age_hist};
+                  c->rd.prefix, c->rd.done, c->rd.stats, c->d_slots, c->d_age_hist, c->d_prefill_out};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   for (auto& r : c->registered) cudaHostUnregister(r.first);
@@ -576,7 +579,7 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   const int n = cfg->num_tables;
   if (n < 1 || n > FLECHE_MAX_TABLES || !cfg->cardinalities || !cfg->dims || !cfg->host_tables) return FLECHE_EINVAL;
   const uint32_t known = FLECHE_FLAG_L2_PREFETCH | FLECHE_FLAG_STATIC_PER_TABLE | FLECHE_FLAG_PER_TABLE_LAUNCH |
-                         FLECHE_FLAG_HOST_ASSIST;
+                         FLECHE_FLAG_HOST_ASSIST | FLECHE_FLAG_FUSED_HIT_COPY;
   if (cfg->max_lookups < 1 || cfg->max_lookups > (int64_t(1) << 31) || (cfg->flags & ~known)) return FLECHE_EINVAL;
   if ((cfg->flags & FLECHE_FLAG_HOST_ASSIST) && (cfg->flags & FLECHE_FLAG_PER_TABLE_LAUNCH)) return FLECHE_EINVAL;
   for (int t = 0; t < n; ++t) {
@@ -748,7 +751,7 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   c->kd_blocks = std::max(1, std::min(c->km_blocks, c->sm_count));  // one wave: duplicates are few
   // decoupled hit copy: uniform layout only (the bytes layout compacts set regions in KM,
   // which may move rows a concurrent copy reads; epoch protection covers the uniform slots)
-  c->decoupled = !bytes && getenv("FLECHE_FUSED_GATHER") == nullptr;
+  c->decoupled = !bytes && !(cfg->flags & FLECHE_FLAG_FUSED_HIT_COPY) && getenv("FLECHE_FUSED_GATHER") == nullptr;
   if (const char* e = getenv("FLECHE_DECOUPLE_MIN")) c->decouple_min = strtoll(e, nullptr, 10);
   if (c->decoupled) {
     if (cudaStreamCreateWithFlags(&c->side, cudaStreamNonBlocking) != cudaSuccess ||
@@ -827,6 +830,26 @@ fleche_status fleche_query(fleche_ctx* c, const int64_t* const* ids, const int64
   if (!c || !ids || !lengths) return FLECHE_EINVAL;
   if (c->poisoned) return FLECHE_ESTATE;
   return query_impl(c, ids, lengths, out, (cudaStream_t)stream);
+}
+
+fleche_status fleche_prefill(fleche_ctx* c, const int64_t* const* ids, const int64_t* lengths, fleche_stream stream) {
+  if (!c || !ids || !lengths) return FLECHE_EINVAL;
+  if (c->poisoned) return FLECHE_ESTATE;
+  int64_t floats = 0;
+  for (int t = 0; t < c->n; ++t) {
+    if (lengths[t] < 0) return FLECHE_EINVAL;
+    floats += lengths[t] * (int64_t)c->dims[t];
+  }
+  fleche_status st = ensure_device(c);
+  if (st != FLECHE_OK) return st;
+  if (floats > c->prefill_floats) {  // the batch's rows land in a ctx-owned scratch output
+    if (c->have_last) FL_CUDA(c, cudaStreamSynchronize(c->last_stream));
+    if (c->d_prefill_out) FL_CUDA(c, cudaFree(c->d_prefill_out));
+    c->d_prefill_out = nullptr;
+    FL_CUDA(c, cudaMalloc((void**)&c->d_prefill_out, (size_t)floats * 4));
+    c->prefill_floats = floats;
+  }
+  return query_impl(c, ids, lengths, c->d_prefill_out, (cudaStream_t)stream);
 }
 
 fleche_status fleche_query_pooled(fleche_ctx* c, const int64_t* const* ids, const int64_t* const* offsets,

@@ -1415,13 +1415,26 @@ __global__ void __launch_bounds__(256) ke_hist_kernel(const __grid_constant__ De
     return;
   }
   const size_t quads = (size_t)dv.sets * 8u;  // 4 ways per thread step (16 B of keys + ts)
-  for (size_t q = (size_t)blockIdx.x * blockDim.x + threadIdx.x; q < quads; q += (size_t)gridDim.x * blockDim.x) {
-    const uint4 k = ld_cg_v4u(dv.keys + 4 * q), t = ld_cg_v4u(dv.ts + 4 * q);
+  const size_t qend = (quads + 31) & ~(size_t)31;  // whole warps stay in the loop (match below)
+  const int lane = threadIdx.x & 31;
+  for (size_t q = (size_t)blockIdx.x * blockDim.x + threadIdx.x; q < qend; q += (size_t)gridDim.x * blockDim.x) {
+    uint4 k = make_uint4(kEmpty, kEmpty, kEmpty, kEmpty), t = make_uint4(0, 0, 0, 0);
+    if (q < quads) {
+      k = ld_cg_v4u(dv.keys + 4 * q);
+      t = ld_cg_v4u(dv.ts + 4 * q);
+    }
     const uint32_t kk[4] = {k.x, k.y, k.z, k.w}, tt[4] = {t.x, t.y, t.z, t.w};
 #pragma unroll
-    for (int j = 0; j < 4; ++j)
-      if (kk[j] != kEmpty && tt[j] < epoch)
-        atomicAdd(&h[min(epoch - tt[j], (uint32_t)(kAgeBins - 1))], way_units(dv, 4 * q + j));
+    for (int j = 0; j < 4; ++j) {
+      const bool live = kk[j] != kEmpty && tt[j] < epoch;
+      const uint32_t a = live ? min(epoch - tt[j], (uint32_t)(kAgeBins - 1)) : 0xFFFFFFFFu;
+      if (!dv.bytes) {  // equal rows: one shared-memory atomic per distinct age in the warp
+        const unsigned grp = __match_any_sync(kFull, a);
+        if (live && lane == __ffs(grp) - 1) atomicAdd(&h[a], (uint32_t)__popc(grp) * (uint32_t)(dv.dim >> 3));
+      } else if (live) {
+        atomicAdd(&h[a], way_units(dv, 4 * q + j));
+      }
+    }
   }
   __syncthreads();
   pdl_trigger();

@@ -15,6 +15,8 @@ pytestmark = pytest.mark.gpu
 
 torch = pytest.importorskip("torch")
 
+import paper_conf_eurosys_xiellwgrs22_b200 as fl  # noqa: E402
+
 
 @pytest.fixture(scope="module", autouse=True)
 def _need_gpu():
@@ -121,16 +123,15 @@ def test_zero_capacity_and_empty_and_ragged():
         assert sg[k] == so[k], k
 
 
-@pytest.mark.parametrize("mode", ["decoupled", "fused"])
+@pytest.mark.parametrize("mode", ["decoupled", "fused", "fused_flag"])
 def test_decoupled_hit_copy_exact(monkeypatch, mode):
     # the hit copy on a side stream (KG, concurrent with the miss kernel) relies on epoch
     # protection: this batch's hit ways are never victims, so their slab rows stay valid
-    if mode == "decoupled":
-        monkeypatch.setenv("FLECHE_DECOUPLE_MIN", "0")
-    else:
+    monkeypatch.setenv("FLECHE_DECOUPLE_MIN", "0")
+    if mode == "fused":
         monkeypatch.setenv("FLECHE_FUSED_GATHER", "1")
     w = configs.get("cfg0").with_(cache_frac=0.01, invalid_ppm=3000, skews=[0.6] * 7, batch_size=400)
-    gpu, _ = _run(w, _tables(w), 30)
+    gpu, _ = _run(w, _tables(w), 30, flags=fl.binding.FLAG_FUSED_HIT_COPY if mode == "fused_flag" else 0)
     per_batch = gpu.stats()["kernels_launched"] / 30
     assert per_batch == (4 if mode == "decoupled" else 3)
 
@@ -260,3 +261,25 @@ def test_address_ordered_scratch_exact(monkeypatch, ordered):
         k = int(keys[way])
         t = int(np.nonzero((base <= k) & (k < base + (1 << fb.astype(np.int64))))[0][0])
         assert H.bits_equal(slab[way], tabs[t][k - int(base[t])])
+
+
+def test_prefill_is_a_batch_without_output():
+    """fleche_prefill = one batch of the policy whose rows are discarded:
+    after it, queries match an oracle that ran the same batch as a query."""
+    w = configs.get("cfg0").with_(cache_frac=0.25)
+    tabs = _tables(w)
+    gpu, orc = H.make_pair(w, tabs)
+    for b in (100, 101):  # warm with two batches the queries below never saw
+        bt = w.batch(b)
+        gpu.prefill([torch.from_numpy(x).cuda() for x in bt.ids])
+        orc.query(bt.ids)
+    torch.cuda.synchronize()
+    sg, so = gpu.stats(), orc.stats()
+    for k in H.STAT_KEYS_EXACT:
+        assert sg[k] == so[k], k
+    for b in range(6):
+        bt = w.batch(b)
+        assert H.bits_equal(H.run_batch_gpu(gpu, bt.ids, torch), orc.query(bt.ids)), b
+    sg, so = gpu.stats(), orc.stats()
+    for k in H.STAT_KEYS_EXACT:
+        assert sg[k] == so[k], k
