@@ -670,6 +670,7 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   dv.admit_thr = dv.admit_all ? ~0ull : (uint64_t)ldexp(p, 64);
   dv.admit_seed = cfg->admit_seed;
   dv.prefetch = (cfg->flags & FLECHE_FLAG_L2_PREFETCH) ? 1 : 0;
+  if (const char* e = getenv("FLECHE_PREFETCH_MODE")) dv.prefetch = atoi(e);  // A/B: 2 = prefetch.global.L2 per line
   if (const char* e = getenv("FLECHE_KM_BLOCKS_PER_SM")) c->km_bps = std::max(1, atoi(e));
 #ifdef FLECHE_EXPERIMENTS
   if (const char* e = getenv("FLECHE_EXP_MODE")) dv.exp_mode = atoi(e);

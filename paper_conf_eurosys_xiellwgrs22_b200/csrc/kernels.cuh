@@ -676,9 +676,13 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
         if (dv.ha)  // published by KM's doorbell (after this grid completes)
           dv.ha_req[(size_t)par * dv.ha_req_cap + li] =
               HaReq{((unsigned long long)(qa.t0 + t) << 48) | (unsigned long long)id, hst};
-        if (dv.prefetch) {  // experimental: start the host-link transfer now
+        if (dv.prefetch == 1) {  // experimental: start the host-link transfer now
           const float* hrow = ti->host + (size_t)id * (size_t)d;
           asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(hrow), "r"(4u * (unsigned)d) : "memory");
+        } else if (dv.prefetch >= 2) {  // experimental: per-line L2 prefetch (warms the address translation)
+          const char* hrow = (const char*)(ti->host + (size_t)id * (size_t)d);
+          const int lines = dv.prefetch == 2 ? 1 : (4 * d + 127) / 128;
+          for (int q = 0; q < lines; ++q) asm volatile("prefetch.global.L2 [%0];" ::"l"(hrow + 128 * q) : "memory");
         }
       }
     }
