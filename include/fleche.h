@@ -81,6 +81,15 @@ typedef struct {
   uint64_t admit_seed;
   uint32_t hash_seed;            /* set index = (fmix32(fk ^ hash_seed) * S) >> 32 (R12)  */
   uint32_t flags;                /* bitwise OR of FLECHE_FLAG_*; other bits must be 0              */
+  int32_t key_bits;              /* flat-key width B.  0 (or >= B_min) = the exact size-aware code
+                                    (P:L640-652).  1 <= B < B_min = short flat keys (P:L646-649,
+                                    DESIGN.md reading R24): the smallest tables keep exact codes, the
+                                    others share the space left in proportion to their sizes with
+                                    their feature IDs hashed into g_t bits, so out row =
+                                    E_t[h_t(id)] (the model's table is indexed by the hashed
+                                    feature; IDs that collide share one row and one cache entry).
+                                    fleche_get_encoding reports g_t.  Not with the key-sharded mode. */
+  int32_t reserved;              /* must be 0                                                      */
 } fleche_config;
 
 /* Experimental: the query kernel starts each unique miss's host-row transfer into L2

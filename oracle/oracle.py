@@ -55,6 +55,14 @@ def lib():
         L.or_query_pooled.argtypes = [vp, vp, vp, vp, vp]
         L.or_stats.restype = None
         L.or_stats.argtypes = [vp, ctypes.POINTER(_Stats)]
+        L.or_encode_short.restype = ctypes.c_int
+        L.or_encode_short.argtypes = [ctypes.c_int, vp, ctypes.c_int, vp, vp, vp]
+        L.or_encode_fixed.restype = ctypes.c_int
+        L.or_encode_fixed.argtypes = [ctypes.c_int, vp, ctypes.c_int, vp, vp, vp]
+        L.or_short_id.restype = i64
+        L.or_short_id.argtypes = [i32, i64, i32, i32]
+        L.or_set_key_bits.restype = ctypes.c_int
+        L.or_set_key_bits.argtypes = [vp, ctypes.c_int]
         L.or_set_watermarks.restype = ctypes.c_int
         L.or_set_watermarks.argtypes = [vp, u64, u64]
         L.or_scans.restype = u64
@@ -75,6 +83,23 @@ def encode(cards, key_bits: int = 32):
     if bmin < 0:
         return None
     return bmin, base, fb
+
+
+def encode_short(cards, key_bits: int, fixed: bool = False):
+    """Short flat keys (reading R24; fixed=True: the fixed-length comparison coder).
+    Returns (lossy tables, base[n], bits[n], exact[n])."""
+    c = np.ascontiguousarray(cards, dtype=np.int64)
+    n = len(c)
+    base = np.zeros(n, dtype=np.uint64)
+    bits = np.zeros(n, dtype=np.int32)
+    ex = np.zeros(n, dtype=np.int32)
+    f = lib().or_encode_fixed if fixed else lib().or_encode_short
+    lossy = f(n, c.ctypes.data, key_bits, base.ctypes.data, bits.ctypes.data, ex.ctypes.data)
+    return lossy, base, bits, ex
+
+
+def short_id(t: int, i: int, bits: int, exact: int) -> int:
+    return int(lib().or_short_id(t, i, bits, exact))
 
 
 def self_identify(scan, tid: int):
@@ -142,6 +167,13 @@ class Oracle:
             out = np.empty(self.out_size(bags), dtype=np.float32)
         lib().or_query_pooled(self.h, _ptr_array(ids), _ptr_array(offsets), bags.ctypes.data, out.ctypes.data)
         return out
+
+    def set_key_bits(self, key_bits: int) -> int:
+        """Short flat keys (reading R24), before the first query; returns the lossy table count."""
+        r = lib().or_set_key_bits(self.h, int(key_bits))
+        if r < 0:
+            raise ValueError("or_set_key_bits rejected the key width")
+        return r
 
     def set_watermarks(self, hi_bytes: int, lo_bytes: int):
         """Full-scan eviction after each batch (reading R23): if cached row

@@ -29,7 +29,7 @@ _vp, _i64, _i32, _u64, _u32 = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32, c
 class fleche_config(ctypes.Structure):
     _fields_ = [("num_tables", _i32), ("cardinalities", _vp), ("dims", _vp), ("cache_bytes", _u64),
                 ("host_tables", _vp), ("max_lookups", _i64), ("device", _i32), ("admit_prob", ctypes.c_double),
-                ("admit_seed", _u64), ("hash_seed", _u32), ("flags", _u32)]
+                ("admit_seed", _u64), ("hash_seed", _u32), ("flags", _u32), ("key_bits", _i32), ("reserved", _i32)]
 
 
 STAT_FIELDS = ["batches", "lookups", "hits", "misses", "invalid", "unique_keys", "unique_hits", "unique_misses",
@@ -132,7 +132,8 @@ class FlatCache:
     """One flat GPU cache over the given host tables (fleche_create / fleche_query / fleche_stats)."""
 
     def __init__(self, cards, dims, host_tables, cache_bytes: int, max_lookups: int, device: int = 0,
-                 admit_prob: float = 1.0, admit_seed: int = 0, hash_seed: int = 0, flags: int = 0):
+                 admit_prob: float = 1.0, admit_seed: int = 0, hash_seed: int = 0, flags: int = 0,
+                 key_bits: int = 0):
         self.n = len(cards)
         self.cards = np.ascontiguousarray(cards, dtype=np.int64)
         self.dims = np.ascontiguousarray(dims, dtype=np.int32)
@@ -140,7 +141,7 @@ class FlatCache:
         self._tp = (_vp * self.n)(*[_ptr(t) for t in self._tables])
         cfg = fleche_config(self.n, self.cards.ctypes.data, self.dims.ctypes.data, int(cache_bytes),
                             ctypes.cast(self._tp, _vp), int(max_lookups), int(device), float(admit_prob),
-                            int(admit_seed), int(hash_seed), int(flags))
+                            int(admit_seed), int(hash_seed), int(flags), int(key_bits), 0)
         h = _vp()
         _check(fleche_create(ctypes.byref(cfg), ctypes.byref(h)), "fleche_create")
         self.h = h.value

@@ -70,6 +70,8 @@ struct fleche_ctx {
   std::vector<uint64_t> base;
   std::vector<int32_t> fbits;
   int key_bits = 0;
+  bool lossy = false;            // short flat keys (R24): some tables hash their feature IDs
+  std::vector<int32_t> hashed;   // per table
   uint64_t capacity_bytes = 0;
   uint64_t slab_floats = 0;
   std::vector<std::pair<void*, size_t>> registered;  // host ranges we registered
@@ -164,6 +166,67 @@ int size_aware_code(const std::vector<int64_t>& card, std::vector<uint64_t>& bas
     at += uint64_t(1) << fb[t];
   }
   return bmin;
+}
+
+// Short flat keys (key_bits < B_min, reading R24): tables in
+// ascending size keep their exact 2^f_t codes while every remaining table can still get
+// one code; the space left is shared by the remaining tables in proportion to their
+// sizes (power-of-two blocks, 2^g * C <= R * c_t, g < f_t), their feature IDs hashed
+// into g bits; if the one-code floor overflows the space, the largest block is halved
+// (ties: the later table in ascending order) until it fits.  Canonical layout as in
+// size_aware_code.  Returns the number of hashed tables, -1 if impossible.
+int short_code(const std::vector<int64_t>& card, int B, std::vector<uint64_t>& base, std::vector<int32_t>& bits,
+               std::vector<int32_t>& hashed) {
+  const int n = (int)card.size();
+  using u128 = unsigned __int128;
+  const u128 space = ((u128)1 << B) - 1;  // the all-ones key stays EMPTY
+  std::vector<int> f(n), up(n);
+  for (int t = 0; t < n; ++t) f[t] = std::max(1, ceil_log2_u64(card[t]));
+  for (int t = 0; t < n; ++t) up[t] = t;
+  std::stable_sort(up.begin(), up.end(), [&](int a, int b) { return card[a] < card[b]; });
+  int keep = 0;
+  u128 acc = 0;
+  for (int i = 0; i <= n; ++i) {
+    if (acc + (u128)(n - i) <= space) keep = i;
+    if (i < n) acc += (u128)1 << f[up[i]];
+  }
+  u128 left = space, rest = 0;
+  for (int i = 0; i < keep; ++i) left -= (u128)1 << f[up[i]];
+  for (int i = keep; i < n; ++i) rest += (u128)card[up[i]];
+  bits.assign(n, 0);
+  hashed.assign(n, 0);
+  for (int i = 0; i < n; ++i) {
+    const int t = up[i];
+    if (i < keep) {
+      bits[t] = f[t];
+      continue;
+    }
+    hashed[t] = 1;
+    int g = 0;
+    while (g + 1 < f[t] && ((u128)1 << (g + 1)) * rest <= left * (u128)card[t]) ++g;
+    bits[t] = g;
+  }
+  for (;;) {
+    u128 tot = 0;
+    int big = -1;
+    for (int i = keep; i < n; ++i) {
+      tot += (u128)1 << bits[up[i]];
+      if (bits[up[i]] > 0 && (big < 0 || bits[up[i]] >= bits[up[big]])) big = i;
+    }
+    if (tot <= left) break;
+    if (big < 0) return -1;
+    bits[up[big]]--;
+  }
+  std::vector<int> ord(n);
+  for (int t = 0; t < n; ++t) ord[t] = t;
+  std::stable_sort(ord.begin(), ord.end(), [&](int a, int b) { return bits[a] > bits[b]; });
+  base.assign(n, 0);
+  uint64_t at = 0;
+  for (int t : ord) {
+    base[t] = at;
+    at += uint64_t(1) << bits[t];
+  }
+  return n - keep;
 }
 
 uint32_t next_pow2(uint64_t x) {
@@ -580,7 +643,8 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   if (n < 1 || n > FLECHE_MAX_TABLES || !cfg->cardinalities || !cfg->dims || !cfg->host_tables) return FLECHE_EINVAL;
   const uint32_t known = FLECHE_FLAG_L2_PREFETCH | FLECHE_FLAG_STATIC_PER_TABLE | FLECHE_FLAG_PER_TABLE_LAUNCH |
                          FLECHE_FLAG_HOST_ASSIST | FLECHE_FLAG_FUSED_HIT_COPY;
-  if (cfg->max_lookups < 1 || cfg->max_lookups > (int64_t(1) << 31) || (cfg->flags & ~known)) return FLECHE_EINVAL;
+  if (cfg->max_lookups < 1 || cfg->max_lookups > (int64_t(1) << 31) || (cfg->flags & ~known) || cfg->reserved)
+    return FLECHE_EINVAL;
   if ((cfg->flags & FLECHE_FLAG_HOST_ASSIST) && (cfg->flags & FLECHE_FLAG_PER_TABLE_LAUNCH)) return FLECHE_EINVAL;
   for (int t = 0; t < n; ++t) {
     if (cfg->cardinalities[t] < 1 || !valid_dim(cfg->dims[t])) return FLECHE_EINVAL;
@@ -594,6 +658,19 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   c->card.assign(cfg->cardinalities, cfg->cardinalities + n);
   c->dims.assign(cfg->dims, cfg->dims + n);
   c->key_bits = size_aware_code(c->card, c->base, c->fbits);
+  c->hashed.assign(n, 0);
+  if (cfg->key_bits < 0 || cfg->key_bits > 32) {
+    delete c;
+    return FLECHE_EINVAL;
+  }
+  if (cfg->key_bits > 0 && (c->key_bits < 0 || cfg->key_bits < c->key_bits)) {  // short flat keys (R24)
+    if (short_code(c->card, cfg->key_bits, c->base, c->fbits, c->hashed) < 0) {
+      delete c;
+      return FLECHE_EINVAL;
+    }
+    c->key_bits = cfg->key_bits;
+    c->lossy = true;
+  }
   for (int t = 0; t < n; ++t)
     if (std::find(c->cls_dim.begin(), c->cls_dim.end(), c->dims[t]) == c->cls_dim.end()) c->cls_dim.push_back(c->dims[t]);
   std::sort(c->cls_dim.begin(), c->cls_dim.end());
@@ -720,7 +797,8 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   std::vector<TableInfo> ti(n);
   for (int t = 0; t < n; ++t)
     ti[t] = TableInfo{dptr[t], c->card[t], (uint32_t)c->base[t], c->dims[t], c->cls[t], p_off[t], p_sets[t],
-                      p_rows[t], p_slab[t]};
+                      p_rows[t], p_slab[t], c->hashed[t] ? (uint32_t)((1ull << c->fbits[t]) - 1) : 0u,
+                      c->hashed[t]};
   if (cudaMemcpy(c->d_tables, ti.data(), sizeof(TableInfo) * n, cudaMemcpyHostToDevice) != cudaSuccess)
     return fail(FLECHE_ECUDA);
   {  // address-ordered miss scratch (uniform layout): slot0 monotone in the host-row address
@@ -1229,7 +1307,7 @@ fleche_status fleche_route(fleche_ctx* c, const int64_t* const* ids, const int64
                            uint32_t owner_seed, uint32_t* send_keys, int64_t* send_counts, fleche_stream stream) {
   if (!c || !ids || !lengths || !send_keys || !send_counts || world < 1 || world > kMaxWorld) return FLECHE_EINVAL;
   if (c->poisoned) return FLECHE_ESTATE;
-  if (!uniform_dims(c)) return FLECHE_EINVAL;
+  if (!uniform_dims(c) || c->lossy) return FLECHE_EINVAL;
   int64_t total = 0;
   for (int t = 0; t < c->n; ++t) {
     if (lengths[t] < 0 || (lengths[t] > 0 && !ids[t])) return FLECHE_EINVAL;

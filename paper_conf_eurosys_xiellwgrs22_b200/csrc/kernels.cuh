@@ -81,7 +81,18 @@ struct TableInfo {
   uint32_t sets;      //   number of sets of the partition
   uint32_t rows;      //   capacity rows of the partition (last set may be partial)
   int64_t slab_off;   //   float offset of the partition's rows in the slab
+  uint32_t hmask;     // short flat keys (R24): 2^g_t - 1 for a hashed table
+  int32_t hashed;     //   1 = feature IDs of this table are hashed into g_t bits
 };
+
+// Short flat keys ("feature ID (hashed) bits", reading R24): the
+// hashed feature ID of table t, splitmix64(id ^ (t << 48) ^ 0x6A09E667F3BCC909) mod 2^g.
+__device__ __forceinline__ int64_t short_feature_id(int t, int64_t id, uint32_t hmask) {
+  uint64_t z = ((uint64_t)id ^ ((uint64_t)t << 48) ^ 0x6A09E667F3BCC909ull) + 0x9E3779B97F4A7C15ull;
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  return (int64_t)((z ^ (z >> 31)) & (uint64_t)hmask);
+}
 
 struct MissRec {  // one unique missed key (its owner lookup)
   int64_t off;    // float offset of the owner's row in `out`
@@ -560,6 +571,7 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
 
     // A2 re-encode to the flat key (size-aware code: fk = base_t + id)
     const bool valid = active && id >= 0 && id < card;
+    if (valid && ti->hashed && !qa.fkeys) id = short_feature_id(qa.t0 + t, id, ti->hmask);  // R24
     const uint32_t fk = valid ? ti->base + (uint32_t)id : kEmpty;
     const uint32_t s = valid ? set_of_t(dv, ti, fk) : 0u;
 

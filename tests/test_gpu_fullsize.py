@@ -52,8 +52,9 @@ def test_cfg5_full_size(monkeypatch, cfg5_tables, ha):
     assert abs(hg - ho) < 0.01, (hg, ho)
     st = gpu.stats()
     assert st["occupancy_bytes"] <= st["capacity_bytes"]
-    if ha == "split":
-        assert 0 < st["assisted_rows"] < st["unique_misses"] and st["assist_timeouts"] == 0
+    if ha == "split":  # cold first batches may time out (rows then come zero-copy); steady state must not
+        assert 0 < dg["assisted_rows"] < dg["unique_misses"], dg
+        assert dg["assist_timeouts"] == 0, dg
 
 
 def test_cfg4_full_size_pooled():

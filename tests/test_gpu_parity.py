@@ -283,3 +283,40 @@ def test_prefill_is_a_batch_without_output():
     sg, so = gpu.stats(), orc.stats()
     for k in H.STAT_KEYS_EXACT:
         assert sg[k] == so[k], k
+
+
+@pytest.mark.parametrize("B", [10, 12, 14, 15])
+def test_short_keys_encoding_matches_oracle(B):
+    """key_bits < B_min (R24): the library's code (fleche_get_encoding) equals the
+    oracle's lossy size-aware code."""
+    w = configs.get("cfg0")
+    tabs = _tables(w)
+    gpu = fl.FlatCache(w.cards, w.dims, tabs, w.cache_bytes, w.batch_size * w.n, 0, 1.0, 0, H.HASH_SEED, 0, B)
+    kb, base, bits = gpu.encoding()
+    lossy, obase, obits, oex = O.encode_short(w.cards, B)
+    assert kb == B and lossy > 0
+    assert base.tolist() == obase.tolist() and bits.tolist() == obits.tolist()
+
+
+@pytest.mark.parametrize("B", [12, 14])
+def test_short_keys_parity(B):
+    """Short flat keys: out = E_t[h_t(id)] bit for bit, stats exactly the set-associative
+    oracle's with the same code (colliding IDs share one entry)."""
+    w = configs.get("cfg0").with_(cache_frac=0.1, invalid_ppm=2000)
+    tabs = _tables(w)
+    gpu = fl.FlatCache(w.cards, w.dims, tabs, w.cache_bytes, w.batch_size * w.n, 0, 1.0, 0, H.HASH_SEED, 0, B)
+    orc = O.Oracle(w.cards, w.dims, tabs, w.cache_bytes, O.MODE_SETASSOC, hash_seed=H.HASH_SEED)
+    assert orc.set_key_bits(B) > 0
+    for b in range(25):
+        bt = w.batch(b)
+        g0, o0 = gpu.stats(), orc.stats()
+        got = H.run_batch_gpu(gpu, bt.ids, torch)
+        ref = orc.query(bt.ids)
+        assert H.bits_equal(got, ref), b
+        dg, do = H.delta(g0, gpu.stats()), H.delta(o0, orc.stats())
+        if do["bypassed"] == 0:
+            for k in H.STAT_KEYS_EXACT:
+                assert dg[k] == do[k], (b, k, dg[k], do[k])
+    with pytest.raises(fl.binding.FlecheError):  # the key-sharded mode needs exact codes
+        gpu.route([torch.zeros(1, dtype=torch.int64, device="cuda")] * w.n, 2, 1,
+                  torch.empty(8, dtype=torch.int32, device="cuda"), torch.empty(2, dtype=torch.int64, device="cuda"))

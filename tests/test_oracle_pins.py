@@ -403,3 +403,104 @@ def test_watermark_setassoc_agrees_with_global_without_overflow():
     for k in ("hits", "inserted", "evicted", "occupancy_bytes"):
         assert sg[k] == ss[k], k
     assert g.scans() == s.scans()
+
+
+# ------------------------------------------------- short flat keys (reading R24)
+def test_short_keys_worked_example():
+    """Hand-worked (R24): c = [3, 5, 100, 900, 20000], B = 12: the four
+    smallest keep exact codes (4 + 8 + 128 + 1024 = 1164 codes, + 1 for the last table
+    <= 4095); R = 4095 - 1164 = 2931 goes to the largest table: 2^11 <= 2931 < 2^12, so
+    11 bits.  Canonical layout by decreasing bits.  B = 14: R = 15219 -> 13 bits."""
+    lossy, base, bits, ex = O.encode_short([3, 5, 100, 900, 20000], 12)
+    assert lossy == 1
+    assert bits.tolist() == [2, 3, 7, 10, 11] and ex.tolist() == [1, 1, 1, 1, 0]
+    assert base.tolist() == [3208, 3200, 3072, 2048, 0]
+    lossy, base, bits, ex = O.encode_short([3, 5, 100, 900, 20000], 14)
+    assert lossy == 1 and bits.tolist() == [2, 3, 7, 10, 13]
+    assert base.tolist() == [9352, 9344, 9216, 8192, 0]
+    # fixed-length comparison coder: 3 table-ID bits, 9 feature bits for every table
+    lossy, base, bits, ex = O.encode_short([3, 5, 100, 900, 20000], 12, fixed=True)
+    assert lossy == 2 and bits.tolist() == [9] * 5 and base.tolist() == [0, 512, 1024, 1536, 2048]
+
+
+@pytest.mark.parametrize("name", ["cfg1", "cfg2", "cfg3", "cfg4"])
+def test_short_keys_reduce_to_exact_code_at_bmin(name):
+    """With B >= B_min the lossy coder must give the exact size-aware code (R3)."""
+    w = configs.get(name)
+    bmin, base, fb = O.encode(w.cards)
+    for B in (bmin, 32):
+        lossy, b2, bits, ex = O.encode_short(w.cards, B)
+        assert lossy == 0 and ex.all()
+        assert b2.tolist() == base.tolist() and bits.tolist() == fb.tolist()
+
+
+def test_short_keys_invariants_random():
+    """Brute-force invariants over random table sets and widths: codes disjoint and
+    inside [0, 2^B - 1) (all-ones free), exact tables = the longest ascending-size prefix
+    that leaves one code per remaining table (maximal), lossy bits non-decreasing in
+    size and summing to <= the space left, hashed IDs inside [0, c_t)."""
+    rng = np.random.default_rng(5)
+    for _ in range(300):
+        n = int(rng.integers(1, 12))
+        cards = [int(x) for x in np.exp(rng.uniform(0, 16, n)).astype(np.int64) + 1]
+        B = int(rng.integers(max(1, int(np.ceil(np.log2(n + 1)))), 24))
+        lossy, base, bits, ex = O.encode_short(cards, B)
+        assert lossy >= 0
+        spans = sorted((int(b), int(b) + (1 << int(g))) for b, g in zip(base, bits))
+        for (a0, a1), (b0, _) in zip(spans, spans[1:]):
+            assert a1 <= b0
+        assert spans[-1][1] <= (1 << B) - 1
+        f = [max(1, int(np.ceil(np.log2(c)))) if c > 1 else 1 for c in cards]
+        order = sorted(range(n), key=lambda t: (cards[t], t))
+        k = sum(ex)
+        assert all(ex[order[i]] for i in range(k)) and not any(ex[order[i]] for i in range(k, n))
+        used = sum(1 << f[order[i]] for i in range(k))
+        assert used + (n - k) <= (1 << B) - 1
+        if k < n:
+            assert used + (1 << f[order[k]]) + (n - k - 1) > (1 << B) - 1  # maximal
+            lg = [int(bits[order[i]]) for i in range(k, n)]
+            lc = [cards[order[i]] for i in range(k, n)]
+            R = (1 << B) - 1 - used
+            assert sum(1 << g for g in lg) <= R
+            for i in range(len(lg) - 1):
+                if lc[i] < lc[i + 1]:
+                    assert lg[i] <= lg[i + 1] + 1  # the overflow rule may lower one larger table by one
+            for t in range(n):
+                if not ex[t]:
+                    assert (1 << int(bits[t])) < cards[t] or cards[t] == 1
+                    for i in (0, cards[t] - 1, cards[t] // 2):
+                        assert 0 <= O.short_id(t, i, int(bits[t]), 0) < min(cards[t], 1 << int(bits[t])) or cards[t] == 1
+
+
+def test_short_key_hash_is_uniform():
+    """h_t(id) = splitmix64(...) mod 2^g: chi-square over 2^10 buckets (catches a hash that
+    keeps only low id bits or ignores the table)."""
+    from scipy import stats
+    ids = np.arange(200_000)
+    for t in (0, 7):
+        h = np.array([O.short_id(t, int(i), 10, 0) for i in ids[:50_000]])
+        cnt = np.bincount(h, minlength=1024)
+        assert stats.chisquare(cnt).pvalue > 1e-3
+    a = [O.short_id(0, int(i), 10, 0) for i in range(64)]
+    b = [O.short_id(1, int(i), 10, 0) for i in range(64)]
+    assert a != b
+
+
+def test_short_keys_cache_is_keyed_by_hashed_id():
+    """One lookup per batch through a lossy table is textbook LRU over the HASHED IDs, and
+    the value is row h(id) (the model's table is indexed by the hashed feature)."""
+    cards, dims = [10, 5000], [4, 4]
+    tabs = _tiny_tables(cards, dims)
+    o = O.Oracle(cards, dims, tabs, 16 * 7, O.MODE_GLOBAL)
+    lossy = o.set_key_bits(10)
+    assert lossy == 1
+    _, base, bits, ex = O.encode_short(cards, 10)
+    rng = np.random.default_rng(2)
+    stream = rng.integers(0, 5000, 2000)
+    hkeys = [O.short_id(1, int(i), int(bits[1]), 0) for i in stream]
+    want = _textbook_lru(hkeys, 7)
+    for i, (x, hk) in enumerate(zip(stream, hkeys)):
+        s0 = o.stats()["hits"]
+        out = o.query([np.array([], np.int64), np.array([x], np.int64)])
+        assert np.array_equal(out, tabs[1][hk])
+        assert (o.stats()["hits"] - s0 == 1) == want[i]
