@@ -289,6 +289,9 @@ fleche_status fleche_kernel_times(fleche_ctx* ctx, double* kq_ms, double* ki_ms,
 /* Same accumulation split per kernel: ms4 = {query (KQ), miss (KM), restore (KD),
  * pooling (KP; 0 for one-hot)} summed over the profiled queries; resets. */
 fleche_status fleche_kernel_times_ex(fleche_ctx* ctx, double* ms4, uint64_t* queries);
+/* Tools only: copy the device control block (sizeof = bytes >= its size) to host on a
+ * private non-blocking stream, so it can be read while the ctx's streams are stuck. */
+fleche_status fleche_debug_ctl(fleche_ctx* ctx, void* host, size_t bytes);
 fleche_status fleche_probe_host_read(const void* host, uint64_t bytes, int32_t row_bytes, int64_t rows, uint64_t seed,
                                      fleche_stream stream, double* gbps);
 

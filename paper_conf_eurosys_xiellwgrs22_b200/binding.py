@@ -76,6 +76,7 @@ fleche_query_keys = _sig("fleche_query_keys", ctypes.c_int, [_vp, _vp, _i64, _vp
 fleche_restore = _sig("fleche_restore", ctypes.c_int, [_vp, _vp, _vp, _vp, _vp])
 fleche_shard_stats = _sig("fleche_shard_stats", ctypes.c_int, [_vp, ctypes.POINTER(_u64), ctypes.POINTER(_u64),
                                                                ctypes.POINTER(_u64), ctypes.POINTER(_u64)])
+fleche_debug_ctl = _sig("fleche_debug_ctl", ctypes.c_int, [_vp, _vp, ctypes.c_size_t])
 fleche_set_watermarks = _sig("fleche_set_watermarks", ctypes.c_int, [_vp, ctypes.c_double, ctypes.c_double])
 fleche_debug_locations = _sig("fleche_debug_locations", ctypes.c_int, [_vp, _vp, ctypes.c_size_t])
 
@@ -83,7 +84,7 @@ EXPORTED = ["fleche_create", "fleche_query", "fleche_query_pooled", "fleche_quer
             "fleche_reset_stats", "fleche_destroy", "fleche_strerror", "fleche_get_encoding", "fleche_get_geometry",
             "fleche_debug_snapshot", "fleche_debug_locations", "fleche_set_profiling", "fleche_kernel_times",
             "fleche_probe_host_read", "fleche_route", "fleche_query_keys", "fleche_restore", "fleche_shard_stats",
-            "fleche_kernel_times_ex", "fleche_set_watermarks", "fleche_prefill"]
+            "fleche_kernel_times_ex", "fleche_set_watermarks", "fleche_prefill", "fleche_debug_ctl"]
 
 
 def probe_host_read(host_ptr: int, nbytes: int, row_bytes: int, rows: int, seed: int = 1, stream=None) -> float:

@@ -86,6 +86,9 @@ struct fleche_ctx {
   cudaStream_t side = nullptr;
   cudaEvent_t fork_ev = nullptr, join_ev = nullptr;
   uint32_t* d_slots = nullptr;
+  bool early = false;            // early miss fetch: KF on the side stream, concurrent with KQ
+  size_t kf_smem = 0;
+  cudaEvent_t kf_ev = nullptr;
   int64_t decouple_min = 524288;  // lookups per batch from which the hit copy is decoupled (cfg2: equal, cfg5: +5 %)
   size_t km_smem = 0;
   // host-side counters
@@ -405,7 +408,8 @@ void free_all(fleche_ctx* c) {
                   c->dv.firstpos, c->dv.ipos,
                   c->dv.miss, c->dv.dup, c->dv.ctl, c->dv.stats, c->d_tables, c->d_ids_stage, c->d_out_stage,
                   c->d_pool_stage, c->d_kdec, c->rd.scratch, c->rd.slotval, c->rd.inv, c->rd.region, c->rd.cnt,
-                  c->rd.prefix, c->rd.done, c->rd.stats, c->d_slots, c->d_age_hist, c->d_prefill_out};
+                  c->rd.prefix, c->rd.done, c->rd.stats, c->d_slots, c->d_age_hist, c->d_prefill_out,
+                  c->dv.mready};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   for (auto& r : c->registered) cudaHostUnregister(r.first);
@@ -413,6 +417,7 @@ void free_all(fleche_ctx* c) {
   if (c->chain_ev) cudaEventDestroy(c->chain_ev);
   if (c->fork_ev) cudaEventDestroy(c->fork_ev);
   if (c->join_ev) cudaEventDestroy(c->join_ev);
+  if (c->kf_ev) cudaEventDestroy(c->kf_ev);
   if (c->side) cudaStreamDestroy(c->side);
   for (cudaEvent_t e : c->ev_pool) cudaEventDestroy(e);
   c->ev_pool.clear();
@@ -521,8 +526,19 @@ fleche_status launch_query(fleche_ctx* c, const int64_t* const* ids, const int64
   fleche_status st = prof_event(c, s, true, nev);
   if (st != FLECHE_OK) return st;
   // small batches: the fork/join costs more than the overlap saves (cfg1 measured +5 %)
-  const bool decouple = c->decoupled && total >= c->decouple_min && !c->per_table_launch;
+  const bool early = c->early && total > 0 && !c->per_table_launch;
+  const bool decouple = !early && c->decoupled && total >= c->decouple_min && !c->per_table_launch;
   if (decouple) qa.slots = c->d_slots;
+  if (early) {  // fork: KF waits on the side stream for the miss records KQ publishes
+    qa.early = 1;
+    ka.early = 1;
+    FL_CUDA(c, cudaEventRecord(c->fork_ev, s));
+    FL_CUDA(c, cudaStreamWaitEvent(c->side, c->fork_ev, 0));
+    KFArgs fa{out, (uint32_t)((total + 127) / 128), c->max_dim};
+    launch_k(kPdlNone, kf_fn(c->max_dim), (unsigned)c->sm_count, kKfWarps * 32, c->kf_smem, c->side, c->dv, fa);
+    c->kernels++;
+    FL_CUDA(c, cudaEventRecord(c->kf_ev, c->side));
+  }
   if (total > 0 && !c->per_table_launch) {
     const int64_t blocks = (total + 127) / 128;
     launch_k(kPdlKQ, kq_fn<MAXT>(), (unsigned)blocks, 128, 0, s, qa, c->dv);
@@ -553,6 +569,7 @@ fleche_status launch_query(fleche_ctx* c, const int64_t* const* ids, const int64
     }
   }
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
+  if (early) FL_CUDA(c, cudaStreamWaitEvent(s, c->kf_ev, 0));  // join: every missed row is in `out`
   launch_k(kPdlKM, km_fn(c->dv.bytes != 0, c->cls_dim.size() == 1 ? c->max_dim : 0), c->km_blocks, 128, c->km_smem, s, c->dv, ka);
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
   launch_k(kPdlKD, kd_fn(), c->kd_blocks, 128, 0, s, c->dv, out);
@@ -839,6 +856,38 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
         cudaMalloc((void**)&c->d_slots, (size_t)cfg->max_lookups * 4) != cudaSuccess)
       return fail(FLECHE_ENOMEM);
   }
+  // early miss fetch (KF concurrent with KQ): uniform single-width layout, row <= 512 B,
+  // not with the host-assisted fetch or per-table launches.  FLECHE_EARLY_FETCH=0/1 (A/B)
+  {
+    const char* e = getenv("FLECHE_EARLY_FETCH");
+    const bool want = e ? atoi(e) != 0 : false;
+    c->early = want && !bytes && !part && c->cls_dim.size() == 1 && c->max_dim <= 128 &&
+               !(cfg->flags & FLECHE_FLAG_HOST_ASSIST) && !c->per_table_launch;
+  }
+  if (c->early) {
+    // KF spins on KQ's progress, so KQ must never wait for KF: load every kernel of the
+    // batch now.  Under lazy module loading (the CUDA 12 default) a kernel's first launch
+    // loads its module, which waits for the running kernels -- KF -- to finish: deadlock.
+    cudaFuncAttributes fa_;
+    if (cudaFuncGetAttributes(&fa_, (const void*)kq_fn<32>()) != cudaSuccess ||
+        cudaFuncGetAttributes(&fa_, (const void*)kq_fn<128>()) != cudaSuccess ||
+        cudaFuncGetAttributes(&fa_, (const void*)kq_fn<FLECHE_MAX_TABLES>()) != cudaSuccess ||
+        cudaFuncGetAttributes(&fa_, (const void*)km_fn(false, c->max_dim)) != cudaSuccess ||
+        cudaFuncGetAttributes(&fa_, (const void*)kd_fn()) != cudaSuccess ||
+        cudaFuncGetAttributes(&fa_, (const void*)ke_hist_fn()) != cudaSuccess ||
+        cudaFuncGetAttributes(&fa_, (const void*)ke_evict_fn()) != cudaSuccess)
+      return fail(FLECHE_ECUDA);
+    const int rounds = std::min(4, 128 / c->max_dim);
+    c->kf_smem = (size_t)kKfWarps * rounds * 32 * (size_t)c->max_dim * 4;
+    if ((!c->side && cudaStreamCreateWithFlags(&c->side, cudaStreamNonBlocking) != cudaSuccess) ||
+        (!c->fork_ev && cudaEventCreateWithFlags(&c->fork_ev, cudaEventDisableTiming) != cudaSuccess) ||
+        cudaEventCreateWithFlags(&c->kf_ev, cudaEventDisableTiming) != cudaSuccess ||
+        cudaMalloc((void**)&dv.mready, (size_t)cfg->max_lookups * 4) != cudaSuccess ||
+        cudaMemset(dv.mready, 0, (size_t)cfg->max_lookups * 4) != cudaSuccess ||
+        cudaFuncSetAttribute((const void*)kf_fn(c->max_dim), cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)c->kf_smem) != cudaSuccess)
+      return fail(FLECHE_ENOMEM);
+  }
   if (cfg->flags & FLECHE_FLAG_HOST_ASSIST) {
     HostAssist* h = c->ha = new (std::nothrow) HostAssist();
     if (!h) return fail(FLECHE_ENOMEM);
@@ -1101,6 +1150,18 @@ fleche_status fleche_debug_locations(fleche_ctx* c, uint16_t* loc, size_t ways_c
   if (c->have_last) FL_CUDA(c, cudaStreamSynchronize(c->last_stream));
   FL_CUDA(c, cudaMemcpy(loc, c->dv.loc, ways * 2, cudaMemcpyDeviceToHost));
   return FLECHE_OK;
+}
+
+// Diagnostics (tools only): copy the device control block to host on a private
+// non-blocking stream, so it can be read while the ctx's own streams are stuck.
+fleche_status fleche_debug_ctl(fleche_ctx* c, void* host, size_t bytes) {
+  if (!c || !host || bytes < sizeof(Ctl)) return FLECHE_EINVAL;
+  cudaStream_t t;
+  if (cudaStreamCreateWithFlags(&t, cudaStreamNonBlocking) != cudaSuccess) return FLECHE_ECUDA;
+  cudaMemcpyAsync(host, c->dv.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, t);
+  const cudaError_t e = cudaStreamSynchronize(t);
+  cudaStreamDestroy(t);
+  return e == cudaSuccess ? FLECHE_OK : FLECHE_ECUDA;
 }
 
 fleche_status fleche_set_watermarks(fleche_ctx* c, double hi, double lo) {
