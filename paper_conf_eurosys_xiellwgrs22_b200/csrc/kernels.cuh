@@ -529,9 +529,7 @@ template <int MAXT>
 __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_constant__ QArgs<MAXT> qa,
                                                                    const __grid_constant__ Dev dv) {
   __shared__ int64_t s_scan[MAXT + 1];
-  __shared__ unsigned long long s_ctr[kNumCtr];
   for (int i = threadIdx.x; i <= qa.n; i += blockDim.x) s_scan[i] = qa.scan[i];
-  if (threadIdx.x < kNumCtr) s_ctr[threadIdx.x] = 0;
   pdl_wait();  // the previous batch (or the caller's producer of ids) has completed
   __syncthreads();
 
@@ -715,28 +713,31 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
 
     if (qa.hit_flags && active) qa.hit_flags[g] = hit ? 1 : 0;  // key-sharded: per-key hit back to requester
 
-    // A9 stats, warp-aggregated then block-aggregated
+    // A9 stats, warp-aggregated, straight into a striped counter row (fire-and-forget
+    // reductions: no block barrier, so a finished warp retires without waiting for the
+    // slowest warp of its CTA)
     const unsigned hm = __ballot_sync(kFull, hit), mm = __ballot_sync(kFull, miss);
     const unsigned im = __ballot_sync(kFull, active && !valid), um = __ballot_sync(kFull, uhit);
     if (lane == 0) {
-      if (hm) atomicAdd(&s_ctr[C_HITS], (unsigned long long)__popc(hm));
-      if (mm) atomicAdd(&s_ctr[C_MISSES], (unsigned long long)__popc(mm));
+      unsigned long long* row = dv.stats + ((blockIdx.x * 4u + (threadIdx.x >> 5)) % kStripes) * kNumCtr;
+      if (hm) atomicAdd(row + C_HITS, (unsigned long long)__popc(hm));
+      if (mm) atomicAdd(row + C_MISSES, (unsigned long long)__popc(mm));
       if (im) {
-        atomicAdd(&s_ctr[C_INVALID], (unsigned long long)__popc(im));
+        atomicAdd(row + C_INVALID, (unsigned long long)__popc(im));
         dv.ctl->err_invalid = 1u;
       }
-      if (um) atomicAdd(&s_ctr[C_UHITS], (unsigned long long)__popc(um));
-      if (own_m) atomicAdd(&s_ctr[C_UMISS], (unsigned long long)__popc(own_m));
-      if (dup_m) atomicAdd(&s_ctr[C_DUPS], (unsigned long long)__popc(dup_m));
+      if (um) atomicAdd(row + C_UHITS, (unsigned long long)__popc(um));
+      if (own_m) atomicAdd(row + C_UMISS, (unsigned long long)__popc(own_m));
+      if (dup_m) atomicAdd(row + C_DUPS, (unsigned long long)__popc(dup_m));
     }
   }
   pdl_trigger();  // KM may be scheduled now; its pdl_wait still waits for this grid
-  __syncthreads();
-  if (threadIdx.x < kNumCtr && s_ctr[threadIdx.x])
-    atomicAdd(dv.stats + (blockIdx.x % kStripes) * kNumCtr + threadIdx.x, s_ctr[threadIdx.x]);
-  if (qa.early && threadIdx.x == 0) {  // every record of this CTA is published: count it for KF
-    __threadfence();
-    atomicAdd(&dv.ctl->kq_cnt[*(volatile uint32_t*)&dv.ctl->epoch & 1u], 1u);
+  if (qa.early) {  // every record of this CTA is published: count it for KF
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      __threadfence();
+      atomicAdd(&dv.ctl->kq_cnt[*(volatile uint32_t*)&dv.ctl->epoch & 1u], 1u);
+    }
   }
 }
 
