@@ -48,3 +48,36 @@ sc = torch.empty(4, dtype=torch.int64, device="cuda")
 g.route(ids, 4, 7, sk, sc)
 torch.cuda.synchronize()
 print("route ok", sc.cpu().tolist())
+
+# later round-1 paths: watermark scan (uniform + bytes layout), short flat keys, prefill,
+# decoupled hit copy, host-assisted split.  (Not the early fetch: KF spins on KQ's
+# progress, and the sanitizer serialises kernels.)
+for name, kw, flags, extra in [("watermark", dict(cache_frac=0.25), 0, "wm"),
+                               ("watermark_mixed", dict(cache_frac=0.2, dims=[8, 16, 32, 64, 128, 8, 256]), 0, "wm"),
+                               ("short_keys", dict(cache_frac=0.1), 0, "kb"),
+                               ("prefill", dict(cache_frac=0.1), 0, "pf"),
+                               ("decoupled", dict(cache_frac=0.05), 0, "dc"),
+                               ("ha_split", dict(cache_frac=0.05), 8, "ha")]:
+    if extra == "dc":
+        os.environ["FLECHE_DECOUPLE_MIN"] = "0"
+    if extra == "ha":
+        os.environ["FLECHE_HA_FRAC"] = "0.5"
+    w = configs.get("cfg0").with_(batch_size=100, **kw)
+    tabs = [np.ascontiguousarray(t) for t in w.make_tables()[1]]
+    g = fl.FlatCache(w.cards, w.dims, tabs, w.cache_bytes, w.batch_size * w.n, 0, 1.0, 0, H.HASH_SEED, flags,
+                     12 if extra == "kb" else 0)
+    o = O.Oracle(w.cards, w.dims, tabs, w.cache_bytes, O.MODE_GLOBAL)
+    if extra == "kb":
+        o.set_key_bits(12)
+    if extra == "wm":
+        g.set_watermarks(0.5, 0.3)
+    if extra == "pf":
+        g.prefill([torch.from_numpy(x).cuda() for x in w.batch(50).ids])
+        o.query(w.batch(50).ids)
+    for b in range(nb):
+        bt = w.batch(b)
+        got = H.run_batch_gpu(g, bt.ids, torch)
+        assert H.bits_equal(got, o.query(bt.ids)), (name, b)
+    print(name, "ok", g.stats()["hits"], g.stats()["scans"])
+    os.environ.pop("FLECHE_DECOUPLE_MIN", None)
+    os.environ.pop("FLECHE_HA_FRAC", None)
