@@ -504,3 +504,44 @@ def test_short_keys_cache_is_keyed_by_hashed_id():
         out = o.query([np.array([], np.int64), np.array([x], np.int64)])
         assert np.array_equal(out, tabs[1][hk])
         assert (o.stats()["hits"] - s0 == 1) == want[i]
+
+
+def _belady_hits(batches, cap):
+    """Belady's MIN with the batch semantics of reading R2/R9 (hits on the pre-batch
+    state, a missed key can only be cached after its batch): after each batch, keep the
+    cap keys (of those cached or just looked up) whose next use is soonest.  An upper
+    bound for any admission/eviction policy under the same constraints."""
+    nxt = {}
+    uses = {}
+    for b, keys in enumerate(batches):
+        for k in set(keys):
+            uses.setdefault(k, []).append(b)
+    cache, hits = set(), 0
+    for b, keys in enumerate(batches):
+        hits += sum(1 for k in keys if k in cache)
+        cand = cache | set(keys)
+
+        def next_use(k):
+            u = [x for x in uses[k] if x > b]
+            return u[0] if u else 1 << 30
+        cache = set(sorted(cand, key=lambda k: (next_use(k), k))[:cap])
+    return hits
+
+
+@pytest.mark.parametrize("seed", [1, 2, 3])
+def test_hits_bounded_by_belady_min(seed):
+    """Catches a policy that 'hits' on keys it could not have cached: the oracle's hits
+    (global and set-associative modes) never exceed Belady's MIN on the same trace."""
+    rng = np.random.default_rng(seed)
+    cards, dims = [60, 40], [4, 4]
+    tabs = _tiny_tables(cards, dims)
+    cap = 12
+    batches = [[(int(t), int(i)) for t in (0, 1) for i in np.minimum(rng.zipf(1.3, 5) - 1, cards[t] - 1)]
+               for _ in range(120)]
+    best = _belady_hits(batches, cap)
+    for mode in (O.MODE_GLOBAL, O.MODE_SETASSOC):
+        o = O.Oracle(cards, dims, tabs, cap * 16, mode)
+        for keys in batches:
+            o.query([np.array([i for t, i in keys if t == u], np.int64) for u in (0, 1)])
+        assert o.stats()["hits"] <= best
+    assert best > 0
