@@ -446,6 +446,15 @@ def main():
     for kd in kern.values():
         kd["achieved"] = kd["bytes"] / (kd["ms"] * 1e-3) / 1e9
         kd["frac"] = kd["achieved"] / kd["peak"]
+    km = kern["km_kernel"]
+    if not ha and km["achieved"] > km["peak"]:
+        # the misses have page locality (e.g. cfg4: most misses fall in a few hot tables), so
+        # the uniform-random ceiling understates what the link gives them: take the next
+        # measured ceiling, the link's rate inside a 1 GiB window
+        km["peak"] = host_link
+        km["peak_source"] = ("measured in-run: random-row zero-copy read inside a 1 GiB window (the misses beat "
+                             "the whole-tier random-row rate %.1f GB/s: they have page locality)" % host_rand)
+        km["frac"] = km["achieved"] / km["peak"]
     dom = max(kern, key=lambda k: kern[k]["ms"])
     kd = kern[dom]
     traffic, traffic_src = None, None
@@ -462,7 +471,7 @@ def main():
             "frac_of_link_bw": kern["km_kernel"]["achieved"] / host_link, "kernels": kern,
             "algorithmic_bytes_per_step": {"hbm": ab["kq_hbm"] + ab["km_hbm"] + ab["kd_hbm"] + ab["kp_hbm"], "host": ab["km_host"]}}
     t_roof_step = max((ab["kq_hbm"] + ab["km_hbm"] + ab["kd_hbm"] + ab["kp_hbm"]) / (hbm_peak * 1e9),
-                      ab["km_host"] / ((host_stage if ha else host_rand) * 1e9))
+                      ab["km_host"] / (kern["km_kernel"]["peak"] * 1e9))
     roof["step_roofline_us"] = t_roof_step * 1e6
     roof["step_frac"] = t_roof_step / (ms / K * 1e-3)
 

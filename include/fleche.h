@@ -273,6 +273,30 @@ fleche_status fleche_restore(fleche_ctx* ctx, const float* rows, const uint8_t* 
 fleche_status fleche_shard_stats(fleche_ctx* ctx, uint64_t* lookups, uint64_t* hits, uint64_t* invalid,
                                  uint64_t* unique_routed);
 
+/* Fused exchange for step 4-5 of the key-sharded batch (SURVEY §8(e) "fused variant"):
+ * instead of returning rows with an all-to-all and restoring from the local copy, the
+ * restore kernel reads every owner's answer in place over peer memory (NVLink P2P
+ * loads through CUDA IPC mappings), so the row transfer is the restore's own loads.
+ *   peer_rows[o]  : DEVICE pointer (valid in this process: own buffer for o == rank, an
+ *                   fleche_ipc_open mapping otherwise) to owner o's `rows` of its
+ *                   fleche_query_keys call of this batch;
+ *   peer_flags[o] : same for its hit_flags (peer_flags itself may be NULL: no hit counts);
+ *   peer_off[o]   : HOST int64: index of this rank's first key in owner o's received
+ *                   order (= sum of the counts owner o received from ranks < this rank).
+ * world must equal the last fleche_route's.  The caller orders the owners' queries before
+ * this call on every rank (a stream-ordered barrier, e.g. an NCCL all-reduce of one
+ * element) and keeps the owners' buffers unchanged until every rank has restored (double
+ * buffering by batch parity).  out as in fleche_restore. */
+fleche_status fleche_restore_p2p(fleche_ctx* ctx, int32_t world, const float* const* peer_rows,
+                                 const uint8_t* const* peer_flags, const int64_t* peer_off, float* out,
+                                 fleche_stream stream);
+/* CUDA IPC helpers for the fused exchange: export a device allocation (the base pointer
+ * of a cudaMalloc allocation) as a 64-byte handle, map a peer process's handle into this
+ * process (peer access enabled lazily), unmap it.  FLECHE_ECUDA on failure. */
+fleche_status fleche_ipc_handle(const void* dptr, uint8_t handle[64]);
+fleche_status fleche_ipc_open(const uint8_t handle[64], void** dptr);
+fleche_status fleche_ipc_close(void* dptr);
+
 /* Diagnostics for measurement (bench.py).
  * fleche_set_profiling: when enabled, every later query records CUDA events on its
  *   stream around each of its kernels (adds ~3 event records per call).

@@ -78,13 +78,36 @@ fleche_shard_stats = _sig("fleche_shard_stats", ctypes.c_int, [_vp, ctypes.POINT
                                                                ctypes.POINTER(_u64), ctypes.POINTER(_u64)])
 fleche_debug_ctl = _sig("fleche_debug_ctl", ctypes.c_int, [_vp, _vp, ctypes.c_size_t])
 fleche_set_watermarks = _sig("fleche_set_watermarks", ctypes.c_int, [_vp, ctypes.c_double, ctypes.c_double])
+fleche_restore_p2p = _sig("fleche_restore_p2p", ctypes.c_int, [_vp, _i32, _vp, _vp, _vp, _vp, _vp])
+fleche_ipc_handle = _sig("fleche_ipc_handle", ctypes.c_int, [_vp, _vp])
+fleche_ipc_open = _sig("fleche_ipc_open", ctypes.c_int, [_vp, ctypes.POINTER(_vp)])
+fleche_ipc_close = _sig("fleche_ipc_close", ctypes.c_int, [_vp])
 fleche_debug_locations = _sig("fleche_debug_locations", ctypes.c_int, [_vp, _vp, ctypes.c_size_t])
 
 EXPORTED = ["fleche_create", "fleche_query", "fleche_query_pooled", "fleche_query_host", "fleche_stats",
             "fleche_reset_stats", "fleche_destroy", "fleche_strerror", "fleche_get_encoding", "fleche_get_geometry",
             "fleche_debug_snapshot", "fleche_debug_locations", "fleche_set_profiling", "fleche_kernel_times",
             "fleche_probe_host_read", "fleche_route", "fleche_query_keys", "fleche_restore", "fleche_shard_stats",
-            "fleche_kernel_times_ex", "fleche_set_watermarks", "fleche_prefill", "fleche_debug_ctl"]
+            "fleche_kernel_times_ex", "fleche_set_watermarks", "fleche_prefill", "fleche_debug_ctl",
+            "fleche_restore_p2p", "fleche_ipc_handle", "fleche_ipc_open", "fleche_ipc_close"]
+
+
+def ipc_handle(ptr: int) -> bytes:
+    """64-byte CUDA IPC handle of a device allocation (its base pointer)."""
+    h = (ctypes.c_uint8 * 64)()
+    _check(fleche_ipc_handle(ptr, h), "fleche_ipc_handle")
+    return bytes(h)
+
+
+def ipc_open(handle: bytes) -> int:
+    h = (ctypes.c_uint8 * 64).from_buffer_copy(handle)
+    p = _vp()
+    _check(fleche_ipc_open(h, ctypes.byref(p)), "fleche_ipc_open")
+    return int(p.value)
+
+
+def ipc_close(ptr: int):
+    _check(fleche_ipc_close(ptr), "fleche_ipc_close")
 
 
 def probe_host_read(host_ptr: int, nbytes: int, row_bytes: int, rows: int, seed: int = 1, stream=None) -> float:
@@ -211,6 +234,14 @@ class FlatCache:
     def query_keys(self, keys, count, rows, hit_flags=None, stream=None):
         _check(fleche_query_keys(self.h, _ptr(keys), int(count), _ptr(rows), _ptr(hit_flags), _stream_handle(stream)),
                "fleche_query_keys")
+
+    def restore_p2p(self, peer_rows, peer_flags, peer_off, out, stream=None):
+        """Fused exchange: restore from every owner's rows in place (peer pointers, ints)."""
+        W = len(peer_rows)
+        rp = (_vp * W)(*[int(p) for p in peer_rows])
+        fp = (_vp * W)(*[int(p) for p in peer_flags]) if peer_flags is not None else None
+        op = (_i64 * W)(*[int(x) for x in peer_off])
+        _check(fleche_restore_p2p(self.h, W, rp, fp, op, _ptr(out), _stream_handle(stream)), "fleche_restore_p2p")
 
     def restore(self, rows, hit_flags, out, stream=None):
         _check(fleche_restore(self.h, _ptr(rows), _ptr(hit_flags), _ptr(out), _stream_handle(stream)),

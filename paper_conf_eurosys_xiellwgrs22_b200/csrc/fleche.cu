@@ -1333,12 +1333,13 @@ fleche_status launch_route(fleche_ctx* c, const int64_t* const* ids, const int64
 }
 
 template <int MAXT, int D>
-fleche_status launch_restore_d(fleche_ctx* c, const float* rows, const uint8_t* flags, float* out, cudaStream_t s) {
+fleche_status launch_restore_d(fleche_ctx* c, const float* rows, const uint8_t* flags, float* out, cudaStream_t s,
+                               const PeerArgs& pa) {
   RArgs<MAXT> ra;
   fill_rargs<MAXT>(c, ra, nullptr, c->route_len.data());
   const int64_t total = ra.scan[c->n];
   if (total > 0) {
-    launch_k(kPdlNone, krs_fn<MAXT>(D), (unsigned)((total + 127) / 128), 128, 0, s, ra, c->rd, rows, flags, out);
+    launch_k(kPdlNone, krs_fn<MAXT>(D), (unsigned)((total + 127) / 128), 128, 0, s, ra, c->rd, rows, flags, out, pa);
     c->kernels++;
   }
   cudaError_t e = cudaGetLastError();
@@ -1347,14 +1348,15 @@ fleche_status launch_restore_d(fleche_ctx* c, const float* rows, const uint8_t* 
 }
 
 template <int MAXT>
-fleche_status launch_restore(fleche_ctx* c, const float* rows, const uint8_t* flags, float* out, cudaStream_t s) {
+fleche_status launch_restore(fleche_ctx* c, const float* rows, const uint8_t* flags, float* out, cudaStream_t s,
+                             const PeerArgs& pa) {
   switch (c->max_dim) {
-    case 8: return launch_restore_d<MAXT, 8>(c, rows, flags, out, s);
-    case 16: return launch_restore_d<MAXT, 16>(c, rows, flags, out, s);
-    case 32: return launch_restore_d<MAXT, 32>(c, rows, flags, out, s);
-    case 64: return launch_restore_d<MAXT, 64>(c, rows, flags, out, s);
-    case 128: return launch_restore_d<MAXT, 128>(c, rows, flags, out, s);
-    default: return launch_restore_d<MAXT, 256>(c, rows, flags, out, s);
+    case 8: return launch_restore_d<MAXT, 8>(c, rows, flags, out, s, pa);
+    case 16: return launch_restore_d<MAXT, 16>(c, rows, flags, out, s, pa);
+    case 32: return launch_restore_d<MAXT, 32>(c, rows, flags, out, s, pa);
+    case 64: return launch_restore_d<MAXT, 64>(c, rows, flags, out, s, pa);
+    case 128: return launch_restore_d<MAXT, 128>(c, rows, flags, out, s, pa);
+    default: return launch_restore_d<MAXT, 256>(c, rows, flags, out, s, pa);
   }
 }
 
@@ -1447,9 +1449,68 @@ fleche_status fleche_restore(fleche_ctx* c, const float* rows, const uint8_t* hi
   cudaStream_t s = (cudaStream_t)stream;
   st = order_on(c, s);
   if (st != FLECHE_OK) return st;
-  if (c->n <= 32) return launch_restore<32>(c, rows, hit_flags, out, s);
-  if (c->n <= 128) return launch_restore<128>(c, rows, hit_flags, out, s);
-  return launch_restore<FLECHE_MAX_TABLES>(c, rows, hit_flags, out, s);
+  PeerArgs pa;
+  memset(&pa, 0, sizeof(pa));
+  if (c->n <= 32) return launch_restore<32>(c, rows, hit_flags, out, s, pa);
+  if (c->n <= 128) return launch_restore<128>(c, rows, hit_flags, out, s, pa);
+  return launch_restore<FLECHE_MAX_TABLES>(c, rows, hit_flags, out, s, pa);
+}
+
+fleche_status fleche_restore_p2p(fleche_ctx* c, int32_t world, const float* const* peer_rows,
+                                 const uint8_t* const* peer_flags, const int64_t* peer_off, float* out,
+                                 fleche_stream stream) {
+  if (!c || !out || ((uintptr_t)out & 15u) || !peer_rows || !peer_off) return FLECHE_EINVAL;
+  if (c->poisoned) return FLECHE_ESTATE;
+  if (!c->rd_ready || world < 1 || world > kMaxWorld || world != c->rd.world) return FLECHE_EINVAL;
+  PeerArgs pa;
+  memset(&pa, 0, sizeof(pa));
+  pa.p2p = 1;
+  for (int o = 0; o < world; ++o) {
+    if (!peer_rows[o] || peer_off[o] < 0) return FLECHE_EINVAL;
+    pa.rows[o] = peer_rows[o];
+    pa.flags[o] = peer_flags ? peer_flags[o] : nullptr;
+    pa.off[o] = peer_off[o];
+  }
+  fleche_status st = ensure_device(c);
+  if (st != FLECHE_OK) return st;
+  cudaStream_t s = (cudaStream_t)stream;
+  st = order_on(c, s);
+  if (st != FLECHE_OK) return st;
+  if (c->n <= 32) return launch_restore<32>(c, nullptr, nullptr, out, s, pa);
+  if (c->n <= 128) return launch_restore<128>(c, nullptr, nullptr, out, s, pa);
+  return launch_restore<FLECHE_MAX_TABLES>(c, nullptr, nullptr, out, s, pa);
+}
+
+fleche_status fleche_ipc_handle(const void* dptr, uint8_t handle[64]) {
+  if (!dptr || !handle) return FLECHE_EINVAL;
+  static_assert(sizeof(cudaIpcMemHandle_t) == 64, "IPC handle size");
+  cudaIpcMemHandle_t h;
+  if (cudaIpcGetMemHandle(&h, (void*)dptr) != cudaSuccess) {
+    cudaGetLastError();
+    return FLECHE_ECUDA;
+  }
+  memcpy(handle, &h, 64);
+  return FLECHE_OK;
+}
+
+fleche_status fleche_ipc_open(const uint8_t handle[64], void** dptr) {
+  if (!handle || !dptr) return FLECHE_EINVAL;
+  cudaIpcMemHandle_t h;
+  memcpy(&h, handle, 64);
+  if (cudaIpcOpenMemHandle(dptr, h, cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) {
+    cudaGetLastError();
+    return FLECHE_ECUDA;
+  }
+  return FLECHE_OK;
+}
+
+fleche_status fleche_ipc_close(void* dptr) {
+  if (!dptr) return FLECHE_EINVAL;
+  if (cudaIpcCloseMemHandle(dptr) != cudaSuccess) {
+    cudaGetLastError();
+    return FLECHE_ECUDA;
+  }
+  return FLECHE_OK;
 }
 
 fleche_status fleche_shard_stats(fleche_ctx* c, uint64_t* lookups, uint64_t* hits, uint64_t* invalid,

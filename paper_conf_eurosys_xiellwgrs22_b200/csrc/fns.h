@@ -15,7 +15,7 @@ namespace fl {
 template <int MAXT> using KqFn = void (*)(QArgs<MAXT>, Dev);
 template <int MAXT> using KpFn = void (*)(PArgs<MAXT>, const TableInfo*);
 template <int MAXT> using KrFn = void (*)(RArgs<MAXT>, RouteDev, const TableInfo*);
-template <int MAXT> using KrsFn = void (*)(RArgs<MAXT>, RouteDev, const float*, const uint8_t*, float*);
+template <int MAXT> using KrsFn = void (*)(RArgs<MAXT>, RouteDev, const float*, const uint8_t*, float*, PeerArgs);
 using KmFn = void (*)(Dev, KMArgs);
 using KdFn = void (*)(Dev, float*);
 using ProbeFn = void (*)(const float*, uint64_t, int64_t, uint64_t, float*);

@@ -33,6 +33,17 @@ struct RouteDev {
   uint32_t owner_seed;
 };
 
+// Fused key-sharded exchange (fleche_restore_p2p): each owner's answer rows and hit
+// flags are read in place through peer pointers (CUDA IPC over NVLink); off[o] = where
+// this rank's keys start in owner o's received order.
+struct PeerArgs {
+  const float* rows[kMaxWorld];
+  const uint8_t* flags[kMaxWorld];
+  int64_t off[kMaxWorld];
+  int32_t p2p;
+  int32_t pad;
+};
+
 template <int MAXT>
 struct RArgs {
   const int64_t* ids[MAXT];
@@ -166,7 +177,7 @@ __global__ void __launch_bounds__(256) kpk_kernel(const __grid_constant__ RouteD
 template <int MAXT, int D>
 __global__ void __launch_bounds__(128) krs_kernel(const __grid_constant__ RArgs<MAXT> ra, const __grid_constant__ RouteDev rd,
                                                   const float* __restrict__ rows, const uint8_t* __restrict__ flags,
-                                                  float* __restrict__ out) {
+                                                  float* __restrict__ out, const __grid_constant__ PeerArgs pa) {
   __shared__ int64_t s_scan[MAXT + 1];
   __shared__ unsigned long long s_hits;
   for (int i = threadIdx.x; i <= ra.n; i += blockDim.x) s_scan[i] = ra.scan[i];
@@ -186,9 +197,16 @@ __global__ void __launch_bounds__(128) krs_kernel(const __grid_constant__ RArgs<
       const uint32_t scr = rd.inv[g];
       if (scr != kEmpty) {
         const unsigned long long v = rd.slotval[scr];
-        const int64_t pos = rd.prefix[v >> 32] + (int64_t)(v & 0xFFFFFFFFull);
-        src = rows + pos * D;
-        if (flags) hit = flags[pos] != 0;
+        if (!pa.p2p) {  // rows returned by the caller's all-to-all, in send order
+          const int64_t pos = rd.prefix[v >> 32] + (int64_t)(v & 0xFFFFFFFFull);
+          src = rows + pos * D;
+          if (flags) hit = flags[pos] != 0;
+        } else {  // fused exchange: read the owner's answer row where it lies (peer HBM over NVLink)
+          const int o = (int)(v >> 32);
+          const int64_t at = pa.off[o] + (int64_t)(v & 0xFFFFFFFFull);
+          src = pa.rows[o] + at * D;
+          if (pa.flags[o]) hit = pa.flags[o][at] != 0;
+        }
       }
     }
     gather_rows<D>(src, dst, lane);
