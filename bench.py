@@ -50,6 +50,8 @@ def parse():
     p.add_argument("--host-assist", action="store_true",
                    help="FLECHE_FLAG_HOST_ASSIST: host threads stage the missed rows (paper Fig 8b CPU-DRAM layer)")
     p.add_argument("--cache-frac", type=float, default=None, help="override the config's cache fraction (sweeps)")
+    p.add_argument("--p2p", action="store_true",
+                   help="--mode sharded: fused exchange (owners' rows read in place over peer memory)")
     p.add_argument("--watermarks", default=None,
                    help="hi,lo: full-scan eviction between these fractions of capacity (P:L660-662, reading R23)")
     p.add_argument("--ha-frac", type=float, default=None,
@@ -221,6 +223,8 @@ def log(*a):
 
 
 def main():
+    # NCCL's version banner goes to stdout, which must carry exactly one JSON line
+    os.environ["NCCL_DEBUG"] = os.environ.get("BENCH_NCCL_DEBUG", "WARN")
     faulthandler.enable()
     args = parse()
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -283,7 +287,7 @@ def main():
             dist.init_process_group("nccl", init_method="tcp://127.0.0.1:%d" % (29600 + os.getpid() % 300),
                                     rank=0, world_size=1, device_id=torch.device("cuda", local))
         from paper_conf_eurosys_xiellwgrs22_b200.sharded import ShardedCache
-        shard = ShardedCache(cache, row_floats=d)
+        shard = ShardedCache(cache, row_floats=d, p2p=args.p2p)
     stream = torch.cuda.current_stream()
 
     def gen_batch(b):
@@ -534,7 +538,9 @@ def main():
                        "tables": w.n, "dim": d if uniform else sorted(set(w.dims)), "batch": w.batch_size,
                        "lookups_per_step": dst["lookups"] / K,
                        "cache_bytes": w.cache_bytes, "host_table_bytes": w.table_bytes,
-                       "parallelism": (f"key-sharded x{world} (NCCL all-to-all)" if sharded else
+                       "parallelism": (f"key-sharded x{world} (" + ("NCCL keys + peer-memory row reads in the restore"
+                                                                     if args.p2p else "NCCL all-to-all") + ")"
+                                       if sharded else
                                        (f"replicated x{world}" if world > 1 else "single GPU")),
                        "prefill_batches": P, "distinct_timed_batches": min(R, K), "admit_prob": args.admit_prob,
                        "miss_fetch": ("host-assisted: %s host threads stage the missed rows (FLECHE_FLAG_HOST_ASSIST)"

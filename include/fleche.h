@@ -293,6 +293,8 @@ fleche_status fleche_restore_p2p(fleche_ctx* ctx, int32_t world, const float* co
 /* CUDA IPC helpers for the fused exchange: export a device allocation (the base pointer
  * of a cudaMalloc allocation) as a 64-byte handle, map a peer process's handle into this
  * process (peer access enabled lazily), unmap it.  FLECHE_ECUDA on failure. */
+fleche_status fleche_ipc_alloc(size_t bytes, void** dptr); /* a cudaMalloc allocation to export */
+fleche_status fleche_ipc_free(void* dptr);
 fleche_status fleche_ipc_handle(const void* dptr, uint8_t handle[64]);
 fleche_status fleche_ipc_open(const uint8_t handle[64], void** dptr);
 fleche_status fleche_ipc_close(void* dptr);

@@ -79,6 +79,8 @@ fleche_shard_stats = _sig("fleche_shard_stats", ctypes.c_int, [_vp, ctypes.POINT
 fleche_debug_ctl = _sig("fleche_debug_ctl", ctypes.c_int, [_vp, _vp, ctypes.c_size_t])
 fleche_set_watermarks = _sig("fleche_set_watermarks", ctypes.c_int, [_vp, ctypes.c_double, ctypes.c_double])
 fleche_restore_p2p = _sig("fleche_restore_p2p", ctypes.c_int, [_vp, _i32, _vp, _vp, _vp, _vp, _vp])
+fleche_ipc_alloc = _sig("fleche_ipc_alloc", ctypes.c_int, [ctypes.c_size_t, ctypes.POINTER(_vp)])
+fleche_ipc_free = _sig("fleche_ipc_free", ctypes.c_int, [_vp])
 fleche_ipc_handle = _sig("fleche_ipc_handle", ctypes.c_int, [_vp, _vp])
 fleche_ipc_open = _sig("fleche_ipc_open", ctypes.c_int, [_vp, ctypes.POINTER(_vp)])
 fleche_ipc_close = _sig("fleche_ipc_close", ctypes.c_int, [_vp])
@@ -89,7 +91,18 @@ EXPORTED = ["fleche_create", "fleche_query", "fleche_query_pooled", "fleche_quer
             "fleche_debug_snapshot", "fleche_debug_locations", "fleche_set_profiling", "fleche_kernel_times",
             "fleche_probe_host_read", "fleche_route", "fleche_query_keys", "fleche_restore", "fleche_shard_stats",
             "fleche_kernel_times_ex", "fleche_set_watermarks", "fleche_prefill", "fleche_debug_ctl",
-            "fleche_restore_p2p", "fleche_ipc_handle", "fleche_ipc_open", "fleche_ipc_close"]
+            "fleche_restore_p2p", "fleche_ipc_handle", "fleche_ipc_open", "fleche_ipc_close", "fleche_ipc_alloc",
+            "fleche_ipc_free"]
+
+
+def ipc_alloc(nbytes: int) -> int:
+    p = _vp()
+    _check(fleche_ipc_alloc(int(nbytes), ctypes.byref(p)), "fleche_ipc_alloc")
+    return int(p.value)
+
+
+def ipc_free(ptr: int):
+    _check(fleche_ipc_free(ptr), "fleche_ipc_free")
 
 
 def ipc_handle(ptr: int) -> bytes:

@@ -1481,6 +1481,20 @@ fleche_status fleche_restore_p2p(fleche_ctx* c, int32_t world, const float* cons
   return launch_restore<FLECHE_MAX_TABLES>(c, nullptr, nullptr, out, s, pa);
 }
 
+fleche_status fleche_ipc_alloc(size_t bytes, void** dptr) {
+  if (!dptr || !bytes) return FLECHE_EINVAL;
+  if (cudaMalloc(dptr, bytes) != cudaSuccess) {
+    cudaGetLastError();
+    return FLECHE_ENOMEM;
+  }
+  return FLECHE_OK;
+}
+
+fleche_status fleche_ipc_free(void* dptr) {
+  if (!dptr) return FLECHE_EINVAL;
+  return cudaFree(dptr) == cudaSuccess ? FLECHE_OK : FLECHE_ECUDA;
+}
+
 fleche_status fleche_ipc_handle(const void* dptr, uint8_t handle[64]) {
   if (!dptr || !handle) return FLECHE_EINVAL;
   static_assert(sizeof(cudaIpcMemHandle_t) == 64, "IPC handle size");

@@ -8,6 +8,15 @@ size the variable all-to-alls.
 
 Owner of a flat key: (fmix32(fk ^ seed ^ 0x85EBCA77) * G) >> 32 (include/fleche.h), so
 rank r caches only its share of the key space and the per-GPU cache budgets aggregate.
+
+p2p=True (the fused exchange): the rows never travel in a collective.  Each
+owner answers into a buffer every rank has mapped (CUDA IPC, peer access over NVLink),
+double-buffered by batch parity; after a one-element all-reduce (a stream-ordered
+barrier: every owner's answers are written) each requester's restore kernel
+(fleche_restore_p2p) reads its rows in place from the owners' HBM.  Counts go by a small
+all-gather (it also gives each rank its offset in every owner's received order), keys by
+the all-to-all.  With the gloo backend (CPU tests) the small collectives go through host
+copies.
 """
 from __future__ import annotations
 
@@ -25,7 +34,8 @@ class ShardedCache:
     which bounds both this rank's batch and the keys it may receive as an owner: create
     the FlatCache with max_lookups >= world x the per-rank batch."""
 
-    def __init__(self, cache, row_floats: int, group=None, owner_seed: int = DEFAULT_OWNER_SEED, device=None):
+    def __init__(self, cache, row_floats: int, group=None, owner_seed: int = DEFAULT_OWNER_SEED, device=None,
+                 p2p: bool = False):
         self.cache = cache
         self.group = group
         self.world = dist.get_world_size(group)
@@ -44,9 +54,92 @@ class ShardedCache:
         self.rows_back = torch.empty((n, self.d), dtype=torch.float32, device=dev)
         self.flags_back = torch.empty(n, dtype=torch.uint8, device=dev)
         self.last_exchange = None
+        self.p2p = bool(p2p)
+        self.batch = 0
+        self.cpu_coll = dist.get_backend(group) == "gloo"
+        if self.p2p:
+            self._setup_p2p(n)
+
+    def _setup_p2p(self, n):
+        from . import binding as B
+        W, me = self.world, self.rank
+        # [parity] owner answer buffers, exported to every rank
+        self.own_rows = [B.ipc_alloc(n * self.d * 4) for _ in range(2)]
+        self.own_flags = [B.ipc_alloc(max(n, 16)) for _ in range(2)]
+        mine = [B.ipc_handle(p) for p in self.own_rows + self.own_flags]
+        allh = [None] * W
+        dist.all_gather_object(allh, mine, group=self.group)
+        self.peer_rows, self.peer_flags, self._opened = [[], []], [[], []], []
+        for o in range(W):
+            for par in range(2):
+                if o == me:
+                    r, f = self.own_rows[par], self.own_flags[par]
+                else:
+                    r, f = B.ipc_open(allh[o][par]), B.ipc_open(allh[o][2 + par])
+                    self._opened += [r, f]
+                self.peer_rows[par].append(r)
+                self.peer_flags[par].append(f)
+        self.bar = torch.zeros(1, dtype=torch.int32, device="cpu" if self.cpu_coll else self.send_counts.device)
+
+    def close(self):
+        if getattr(self, "p2p", False) and getattr(self, "own_rows", None):
+            from . import binding as B
+            torch.cuda.synchronize()
+            dist.barrier(group=self.group)  # no peer reads our buffers any more
+            for p in self._opened:
+                B.ipc_close(p)
+            for p in self.own_rows + self.own_flags:
+                B.ipc_free(p)
+            self.own_rows = None
+
+    def _all_gather_counts(self):
+        if self.cpu_coll:
+            torch.cuda.synchronize()
+            mine = self.send_counts.cpu()
+            allc = [torch.zeros_like(mine) for _ in range(self.world)]
+            dist.all_gather(allc, mine, group=self.group)
+            return torch.stack(allc)
+        allc = [torch.zeros_like(self.send_counts) for _ in range(self.world)]
+        dist.all_gather(allc, self.send_counts, group=self.group)
+        return torch.stack(allc).cpu()
+
+    def _keys_all_to_all(self, nr, ns, R, S):
+        if self.cpu_coll:
+            torch.cuda.synchronize()
+            rk = torch.empty(nr, dtype=torch.int32)
+            dist.all_to_all_single(rk, self.send_keys[:ns].cpu(), R, S, group=self.group)
+            self.recv_keys[:nr].copy_(rk)
+        else:
+            dist.all_to_all_single(self.recv_keys[:nr], self.send_keys[:ns], R, S, group=self.group)
+
+    def _barrier(self):
+        if self.cpu_coll:
+            torch.cuda.synchronize()
+        dist.all_reduce(self.bar, group=self.group)
+
+    def query_p2p(self, ids, out, lengths=None):
+        """One batch through the fused exchange (see the module docstring)."""
+        c, W, me = self.cache, self.world, self.rank
+        par = self.batch & 1
+        self.batch += 1
+        c.route(ids, W, self.seed, self.send_keys, self.send_counts, lengths=lengths)
+        C = self._all_gather_counts()  # C[src][owner]
+        S = [int(x) for x in C[me]]
+        R = [int(x) for x in C[:, me]]
+        off = [int(C[:me, o].sum()) for o in range(W)]
+        ns, nr = sum(S), sum(R)
+        self._keys_all_to_all(nr, ns, R, S)
+        c.query_keys(self.recv_keys, nr, self.own_rows[par], self.own_flags[par])
+        self._barrier()  # every owner's answers of this batch are in place
+        c.restore_p2p(self.peer_rows[par], self.peer_flags[par], off, out)
+        self.last_exchange = {"sent_keys": ns, "recv_keys": nr, "nvlink_bytes_out": ns * 4,
+                              "nvlink_bytes_in_p2p": ns * (4 * self.d + 1)}
+        return self.last_exchange
 
     def query(self, ids, out, lengths=None):
         """One batch: this rank's per-table ID lists -> `out` (layout of fleche_query)."""
+        if self.p2p:
+            return self.query_p2p(ids, out, lengths=lengths)
         c = self.cache
         c.route(ids, self.world, self.seed, self.send_keys, self.send_counts, lengths=lengths)
         dist.all_to_all_single(self.recv_counts, self.send_counts, group=self.group)

@@ -87,3 +87,26 @@ def test_sharded_one_rank_nccl_bit_exact_and_exact_hits():
             assert sg[k] == so[k], k
     finally:
         dist.destroy_process_group()
+
+
+def test_p2p_two_processes_one_gpu(tmp_path):
+    """The fused exchange (fleche_restore_p2p: every requester reads its rows in place from
+    the owners' answer buffers through CUDA IPC mappings) with two ranks sharing cuda:0
+    (gloo for the small collectives): `out` bit-exact on both ranks; the requesters saw
+    hits, and never more than their valid lookups."""
+    import json
+    import subprocess
+    import sys
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    procs = [subprocess.Popen([sys.executable, "tests/p2p_worker.py", str(r), "2", str(tmp_path / f"r{r}.json"),
+                               str(port)]) for r in range(2)]
+    for p in procs:
+        assert p.wait(timeout=300) == 0
+    res = [json.load(open(tmp_path / f"r{r}.json")) for r in range(2)]
+    assert all(r["ok"] for r in res), res
+    for r in res:
+        assert 0 < r["req_hits"] <= r["req_lookups"] - r["invalid"], r
+        assert r["owner_hits"] > 0
