@@ -290,6 +290,20 @@ fleche_status fleche_shard_stats(fleche_ctx* ctx, uint64_t* lookups, uint64_t* h
 fleche_status fleche_restore_p2p(fleche_ctx* ctx, int32_t world, const float* const* peer_rows,
                                  const uint8_t* const* peer_flags, const int64_t* peer_off, float* out,
                                  fleche_stream stream);
+/* Fused exchange, key side: fleche_route whose pack step stores each unique key straight
+ * into its owner's receive buffer (peer HBM through CUDA IPC) instead of send_keys:
+ * peer_slots[o] = DEVICE pointer to this rank's slot in owner o's buffer (room for
+ * max_lookups keys).  send_counts as in fleche_route.  The owner answers the keys of all
+ * sources with fleche_query_keys_seg once every rank's route has completed (e.g. after
+ * the counts all-gather, itself stream-ordered behind the routes). */
+fleche_status fleche_route_p2p(fleche_ctx* ctx, const int64_t* const* ids, const int64_t* lengths, int32_t world,
+                               uint32_t owner_seed, uint32_t* const* peer_slots, int64_t* send_counts,
+                               fleche_stream stream);
+/* fleche_query_keys over nseg segments (one per source rank, in rank order): segs[i] is a
+ * DEVICE pointer to counts[i] (HOST) flat keys; row g of `rows` answers the g-th key of
+ * their concatenation.  One batch of the owner's cache. */
+fleche_status fleche_query_keys_seg(fleche_ctx* ctx, const uint32_t* const* segs, const int64_t* counts, int32_t nseg,
+                                    float* rows, uint8_t* hit_flags, fleche_stream stream);
 /* CUDA IPC helpers for the fused exchange: export a device allocation (the base pointer
  * of a cudaMalloc allocation) as a 64-byte handle, map a peer process's handle into this
  * process (peer access enabled lazily), unmap it.  FLECHE_ECUDA on failure. */

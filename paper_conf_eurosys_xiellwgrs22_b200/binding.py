@@ -78,6 +78,8 @@ fleche_shard_stats = _sig("fleche_shard_stats", ctypes.c_int, [_vp, ctypes.POINT
                                                                ctypes.POINTER(_u64), ctypes.POINTER(_u64)])
 fleche_debug_ctl = _sig("fleche_debug_ctl", ctypes.c_int, [_vp, _vp, ctypes.c_size_t])
 fleche_set_watermarks = _sig("fleche_set_watermarks", ctypes.c_int, [_vp, ctypes.c_double, ctypes.c_double])
+fleche_route_p2p = _sig("fleche_route_p2p", ctypes.c_int, [_vp, _vp, _vp, _i32, _u32, _vp, _vp, _vp])
+fleche_query_keys_seg = _sig("fleche_query_keys_seg", ctypes.c_int, [_vp, _vp, _vp, _i32, _vp, _vp, _vp])
 fleche_restore_p2p = _sig("fleche_restore_p2p", ctypes.c_int, [_vp, _i32, _vp, _vp, _vp, _vp, _vp])
 fleche_ipc_alloc = _sig("fleche_ipc_alloc", ctypes.c_int, [ctypes.c_size_t, ctypes.POINTER(_vp)])
 fleche_ipc_free = _sig("fleche_ipc_free", ctypes.c_int, [_vp])
@@ -92,7 +94,7 @@ EXPORTED = ["fleche_create", "fleche_query", "fleche_query_pooled", "fleche_quer
             "fleche_probe_host_read", "fleche_route", "fleche_query_keys", "fleche_restore", "fleche_shard_stats",
             "fleche_kernel_times_ex", "fleche_set_watermarks", "fleche_prefill", "fleche_debug_ctl",
             "fleche_restore_p2p", "fleche_ipc_handle", "fleche_ipc_open", "fleche_ipc_close", "fleche_ipc_alloc",
-            "fleche_ipc_free"]
+            "fleche_ipc_free", "fleche_route_p2p", "fleche_query_keys_seg"]
 
 
 def ipc_alloc(nbytes: int) -> int:
@@ -247,6 +249,22 @@ class FlatCache:
     def query_keys(self, keys, count, rows, hit_flags=None, stream=None):
         _check(fleche_query_keys(self.h, _ptr(keys), int(count), _ptr(rows), _ptr(hit_flags), _stream_handle(stream)),
                "fleche_query_keys")
+
+    def route_p2p(self, ids, world, owner_seed, peer_slots, send_counts, stream=None, lengths=None):
+        if lengths is None:
+            lengths = [int(x.numel()) for x in ids]
+        lp = (_i64 * self.n)(*lengths)
+        ip = (_vp * self.n)(*[_ptr(x) for x in ids])
+        sp = (_vp * world)(*[int(p) for p in peer_slots])
+        _check(fleche_route_p2p(self.h, ip, lp, int(world), int(owner_seed), sp, _ptr(send_counts),
+                                _stream_handle(stream)), "fleche_route_p2p")
+
+    def query_keys_seg(self, segs, counts, rows, hit_flags=None, stream=None):
+        G = len(segs)
+        sp = (_vp * G)(*[int(p) for p in segs])
+        cp = (_i64 * G)(*[int(x) for x in counts])
+        _check(fleche_query_keys_seg(self.h, sp, cp, G, _ptr(rows), _ptr(hit_flags), _stream_handle(stream)),
+               "fleche_query_keys_seg")
 
     def restore_p2p(self, peer_rows, peer_flags, peer_off, out, stream=None):
         """Fused exchange: restore from every owner's rows in place (peer pointers, ints)."""

@@ -119,6 +119,7 @@ struct fleche_ctx {
   long long wm_hi = 0, wm_lo = 0;
   unsigned long long* d_age_hist = nullptr;
   int ke_blocks = 0;
+  PeerKeys route_peer{};         // fleche_route_p2p: owners' receive slots for this rank
   // fleche_prefill scratch output (lazy)
   float* d_prefill_out = nullptr;
   int64_t prefill_floats = 0;
@@ -1267,7 +1268,8 @@ namespace {
 
 template <int MAXT>
 fleche_status launch_keys(fleche_ctx* c, const uint32_t* keys, int64_t count, float* rows, uint8_t* flags,
-                          cudaStream_t s) {
+                          cudaStream_t s, const uint32_t* const* segs = nullptr, const int64_t* seg_counts = nullptr,
+                          int nseg = 0) {
   QArgs<MAXT> qa;
   memset(&qa, 0, sizeof(qa));  // out_off[t] = 0: row g of `rows` answers keys[g]
   qa.n = 1;
@@ -1275,6 +1277,18 @@ fleche_status launch_keys(fleche_ctx* c, const uint32_t* keys, int64_t count, fl
   qa.out = rows;
   qa.fkeys = keys;
   qa.hit_flags = flags;
+  if (segs) {  // segments in order: row g answers the g-th key of their concatenation
+    qa.fkseg = 1;
+    qa.n = nseg;
+    int64_t acc = 0;
+    for (int i = 0; i < nseg; ++i) {
+      qa.ids[i] = (const int64_t*)segs[i];
+      qa.scan[i] = acc;
+      acc += seg_counts[i];
+    }
+    qa.scan[nseg] = acc;
+    qa.fkeys = segs[0];  // non-null: the flat-key path
+  }
   KMArgs ka;
   memset(&ka, 0, sizeof(ka));
   ka.out = rows;
@@ -1325,7 +1339,7 @@ fleche_status launch_route(fleche_ctx* c, const int64_t* const* ids, const int64
     c->kernels++;
   }
   launch_k(kPdlNone, kpk_fn(), (unsigned)std::max(1, std::min(2 * c->sm_count, (int)((total + 255) / 256))), 256, 0, s,
-           c->rd, send_keys, send_counts);
+           c->rd, send_keys, send_counts, c->route_peer);
   c->kernels++;
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return poison(c, e, "kernel launch");
@@ -1436,6 +1450,49 @@ fleche_status fleche_query_keys(fleche_ctx* c, const uint32_t* keys, int64_t cou
     c->batches++;
     c->lookups += (uint64_t)count;
   }
+  return st;
+}
+
+fleche_status fleche_query_keys_seg(fleche_ctx* c, const uint32_t* const* segs, const int64_t* counts, int32_t nseg,
+                                    float* rows, uint8_t* hit_flags, fleche_stream stream) {
+  if (!c || !segs || !counts || nseg < 1 || nseg > kMaxWorld || !rows || ((uintptr_t)rows & 15u)) return FLECHE_EINVAL;
+  if (c->poisoned) return FLECHE_ESTATE;
+  int64_t count = 0;
+  for (int i = 0; i < nseg; ++i) {
+    if (counts[i] < 0 || (counts[i] > 0 && !segs[i])) return FLECHE_EINVAL;
+    count += counts[i];
+  }
+  if (!uniform_dims(c) || c->dv.part || count > c->max_lookups) return FLECHE_EINVAL;
+  fleche_status st = ensure_device(c);
+  if (st != FLECHE_OK) return st;
+  cudaStream_t s = (cudaStream_t)stream;
+  st = order_on(c, s);
+  if (st != FLECHE_OK) return st;
+  std::vector<const uint32_t*> sg(segs, segs + nseg);
+  for (auto& p : sg)
+    if (!p) p = segs[0] ? segs[0] : reinterpret_cast<const uint32_t*>(rows);  // empty segments are never read
+  st = launch_keys<128>(c, sg[0], count, rows, hit_flags, s, sg.data(), counts, nseg);
+  if (st == FLECHE_OK) {
+    c->batches++;
+    c->lookups += (uint64_t)count;
+  }
+  return st;
+}
+
+fleche_status fleche_route_p2p(fleche_ctx* c, const int64_t* const* ids, const int64_t* lengths, int32_t world,
+                               uint32_t owner_seed, uint32_t* const* peer_slots, int64_t* send_counts,
+                               fleche_stream stream) {
+  if (!c || !peer_slots || world < 1 || world > kMaxWorld) return FLECHE_EINVAL;
+  PeerKeys pk{};
+  pk.p2p = 1;
+  for (int o = 0; o < world; ++o) {
+    if (!peer_slots[o]) return FLECHE_EINVAL;
+    pk.dst[o] = peer_slots[o];
+  }
+  c->route_peer = pk;
+  uint32_t dummy_keys = 0;  // not written in this mode
+  const fleche_status st = fleche_route(c, ids, lengths, world, owner_seed, &dummy_keys, send_counts, stream);
+  c->route_peer = PeerKeys{};
   return st;
 }
 

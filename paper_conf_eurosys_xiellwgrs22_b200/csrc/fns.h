@@ -19,7 +19,7 @@ template <int MAXT> using KrsFn = void (*)(RArgs<MAXT>, RouteDev, const float*, 
 using KmFn = void (*)(Dev, KMArgs);
 using KdFn = void (*)(Dev, float*);
 using ProbeFn = void (*)(const float*, uint64_t, int64_t, uint64_t, float*);
-using KpkFn = void (*)(RouteDev, uint32_t*, int64_t*);
+using KpkFn = void (*)(RouteDev, uint32_t*, int64_t*, PeerKeys);
 using KeFn = void (*)(Dev, KEArgs);
 using KfFn = void (*)(Dev, KFArgs);
 

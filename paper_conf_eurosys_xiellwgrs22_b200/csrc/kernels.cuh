@@ -215,7 +215,7 @@ struct QArgs {
   int32_t n;
   int32_t t0;                // first table of this launch (per-table launches: t0 = t, n = 1)
   int32_t early;             // early fetch: publish each miss record for KF, count finished CTAs
-  int32_t pad;
+  int32_t fkseg;             // key-sharded fused exchange: fkeys come in n segments (ids[], scan[])
 };
 
 struct KMArgs {
@@ -557,7 +557,17 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
     } else if (active) {
       // key-sharded owner side: lookups arrive as flat keys; decode the table by prefix
       // match (largest base <= fk, the canonical size-aware code) and id = fk - base_t
-      const uint32_t fk0 = qa.fkeys[g];
+      uint32_t fk0;
+      if (qa.fkseg) {  // fused exchange: one segment per source rank (ids[] hold the segment pointers)
+        int a = 0, b2 = qa.n;
+        while (b2 - a > 1) {
+          const int mid = (a + b2) >> 1;
+          if (s_scan[mid] <= g) a = mid; else b2 = mid;
+        }
+        fk0 = ((const uint32_t*)qa.ids[a])[g - s_scan[a]];
+      } else {
+        fk0 = qa.fkeys[g];
+      }
       int lo = 0, hi = dv.ntables;
       while (hi - lo > 1) {
         const int mid = (lo + hi) >> 1;

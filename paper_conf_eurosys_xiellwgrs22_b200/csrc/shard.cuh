@@ -44,6 +44,14 @@ struct PeerArgs {
   int32_t pad;
 };
 
+// Fused exchange, key side (fleche_route_p2p): dst[o] = this rank's slot in owner o's
+// receive buffer (a peer pointer through CUDA IPC; own buffer for o == rank).
+struct PeerKeys {
+  uint32_t* dst[kMaxWorld];
+  int32_t p2p;
+  int32_t pad;
+};
+
 template <int MAXT>
 struct RArgs {
   const int64_t* ids[MAXT];
@@ -138,7 +146,7 @@ __global__ void __launch_bounds__(128) kr_kernel(const __grid_constant__ RArgs<M
 // per-owner counters for the next batch.
 template <int = 0>
 __global__ void __launch_bounds__(256) kpk_kernel(const __grid_constant__ RouteDev rd, uint32_t* __restrict__ send_keys,
-                                                  int64_t* __restrict__ send_counts) {
+                                                  int64_t* __restrict__ send_counts, const __grid_constant__ PeerKeys pk) {
   __shared__ int64_t s_pre[kMaxWorld + 1];
   __shared__ uint32_t s_cnt[kMaxWorld];
   if (threadIdx.x == 0) {
@@ -155,7 +163,9 @@ __global__ void __launch_bounds__(256) kpk_kernel(const __grid_constant__ RouteD
   for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < total; k += (int64_t)gridDim.x * blockDim.x) {
     int o = 0;
     while (s_pre[o + 1] <= k) ++o;
-    send_keys[k] = rd.region[(size_t)o * rd.cap + (k - s_pre[o])];
+    const uint32_t key = rd.region[(size_t)o * rd.cap + (k - s_pre[o])];
+    if (pk.p2p) pk.dst[o][k - s_pre[o]] = key;  // fused exchange: straight into owner o's slot (peer HBM)
+    else send_keys[k] = key;
   }
   if (blockIdx.x == 0 && threadIdx.x < rd.world) {
     send_counts[threadIdx.x] = s_cnt[threadIdx.x];

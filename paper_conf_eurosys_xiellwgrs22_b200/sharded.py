@@ -9,14 +9,17 @@ size the variable all-to-alls.
 Owner of a flat key: (fmix32(fk ^ seed ^ 0x85EBCA77) * G) >> 32 (include/fleche.h), so
 rank r caches only its share of the key space and the per-GPU cache budgets aggregate.
 
-p2p=True (the fused exchange): the rows never travel in a collective.  Each
-owner answers into a buffer every rank has mapped (CUDA IPC, peer access over NVLink),
-double-buffered by batch parity; after a one-element all-reduce (a stream-ordered
-barrier: every owner's answers are written) each requester's restore kernel
-(fleche_restore_p2p) reads its rows in place from the owners' HBM.  Counts go by a small
-all-gather (it also gives each rank its offset in every owner's received order), keys by
-the all-to-all.  With the gloo backend (CPU tests) the small collectives go through host
-copies.
+p2p=True (the fused exchange): neither keys nor rows travel in a
+collective.  Every rank maps every owner's receive and answer buffers (CUDA IPC, peer
+access over NVLink).  The route's pack kernel stores each unique key straight into its
+owner's slot for this rank (fleche_route_p2p); a G x G counts all-gather (stream-ordered
+behind every rank's route, so it is also the "keys are in place" barrier) sizes the
+owner query over its per-source segments (fleche_query_keys_seg) and gives each rank its
+offset in every owner's answer order; after a one-element all-reduce (a stream-ordered
+barrier: every owner's answers are written; answers are double-buffered by batch parity)
+each requester's restore kernel (fleche_restore_p2p) reads its rows in place from the
+owners' HBM.  With the gloo backend (CPU / one-GPU tests) the small collectives go
+through host copies.
 """
 from __future__ import annotations
 
@@ -66,7 +69,8 @@ class ShardedCache:
         # [parity] owner answer buffers, exported to every rank
         self.own_rows = [B.ipc_alloc(n * self.d * 4) for _ in range(2)]
         self.own_flags = [B.ipc_alloc(max(n, 16)) for _ in range(2)]
-        mine = [B.ipc_handle(p) for p in self.own_rows + self.own_flags]
+        self.own_recv = B.ipc_alloc(W * n * 4)  # [source][n] keys routed to this owner
+        mine = [B.ipc_handle(p) for p in self.own_rows + self.own_flags + [self.own_recv]]
         allh = [None] * W
         dist.all_gather_object(allh, mine, group=self.group)
         self.peer_rows, self.peer_flags, self._opened = [[], []], [[], []], []
@@ -79,6 +83,14 @@ class ShardedCache:
                     self._opened += [r, f]
                 self.peer_rows[par].append(r)
                 self.peer_flags[par].append(f)
+        # this rank's slot in every owner's receive buffer, and this owner's per-source segments
+        self.peer_slots = []
+        for o in range(W):
+            base = self.own_recv if o == me else B.ipc_open(allh[o][4])
+            if o != me:
+                self._opened.append(base)
+            self.peer_slots.append(base + me * n * 4)
+        self.own_segs = [self.own_recv + src * n * 4 for src in range(W)]
         self.bar = torch.zeros(1, dtype=torch.int32, device="cpu" if self.cpu_coll else self.send_counts.device)
 
     def close(self):
@@ -88,7 +100,7 @@ class ShardedCache:
             dist.barrier(group=self.group)  # no peer reads our buffers any more
             for p in self._opened:
                 B.ipc_close(p)
-            for p in self.own_rows + self.own_flags:
+            for p in self.own_rows + self.own_flags + [self.own_recv]:
                 B.ipc_free(p)
             self.own_rows = None
 
@@ -122,18 +134,20 @@ class ShardedCache:
         c, W, me = self.cache, self.world, self.rank
         par = self.batch & 1
         self.batch += 1
-        c.route(ids, W, self.seed, self.send_keys, self.send_counts, lengths=lengths)
+        # keys: the route's pack kernel stores them straight into the owners' slots (peer HBM)
+        c.route_p2p(ids, W, self.seed, self.peer_slots, self.send_counts, lengths=lengths)
+        # counts: all-gather (stream-ordered behind every rank's route: the keys are in place)
         C = self._all_gather_counts()  # C[src][owner]
         S = [int(x) for x in C[me]]
         R = [int(x) for x in C[:, me]]
         off = [int(C[:me, o].sum()) for o in range(W)]
         ns, nr = sum(S), sum(R)
-        self._keys_all_to_all(nr, ns, R, S)
-        c.query_keys(self.recv_keys, nr, self.own_rows[par], self.own_flags[par])
+        c.query_keys_seg(self.own_segs, R, self.own_rows[par], self.own_flags[par])
         self._barrier()  # every owner's answers of this batch are in place
+        # rows: each requester reads its answers in place from the owners' HBM
         c.restore_p2p(self.peer_rows[par], self.peer_flags[par], off, out)
-        self.last_exchange = {"sent_keys": ns, "recv_keys": nr, "nvlink_bytes_out": ns * 4,
-                              "nvlink_bytes_in_p2p": ns * (4 * self.d + 1)}
+        self.last_exchange = {"sent_keys": ns, "recv_keys": nr, "p2p_bytes_out": ns * 4,
+                              "p2p_bytes_in": ns * (4 * self.d + 1)}
         return self.last_exchange
 
     def query(self, ids, out, lengths=None):
