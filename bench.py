@@ -538,7 +538,7 @@ def main():
                        "tables": w.n, "dim": d if uniform else sorted(set(w.dims)), "batch": w.batch_size,
                        "lookups_per_step": dst["lookups"] / K,
                        "cache_bytes": w.cache_bytes, "host_table_bytes": w.table_bytes,
-                       "parallelism": (f"key-sharded x{world} (" + ("NCCL keys + peer-memory row reads in the restore"
+                       "parallelism": (f"key-sharded x{world} (" + ("keys and rows over peer memory, fused in the route and restore kernels"
                                                                      if args.p2p else "NCCL all-to-all") + ")"
                                        if sharded else
                                        (f"replicated x{world}" if world > 1 else "single GPU")),
