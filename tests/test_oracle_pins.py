@@ -545,3 +545,25 @@ def test_hits_bounded_by_belady_min(seed):
             o.query([np.array([i for t, i in keys if t == u], np.int64) for u in (0, 1)])
         assert o.stats()["hits"] <= best
     assert best > 0
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("frac,paper", [(0.05, 0.69), (0.10, 0.78)])
+def test_paper_synthetic_hit_rates_loose(frac, paper):
+    """LOOSE pin (SURVEY c-6, reading R1): the paper's synthetic workload -- 40 tables of
+    0.25M features, power law alpha = -1.2 -- reaches hit rates of 69 % and
+    78 % at 5 % and 10 % cache.  The batch size is not stated; at 2,048
+    samples the oracle's PER-UNIQUE-KEY hit ratio lands within 3 pp of both (per lookup it
+    is ~0.91 / 0.93), which is why bench.py reports both ratios.  Catches a gross error in
+    the replacement policy (e.g. evicting the hottest entries) that still passes the LRU
+    reductions."""
+    w = configs.Workload("syn", 6, [250_000] * 40, [4] * 40, [1.2] * 40, 2048, frac)
+    tabs = [np.ascontiguousarray(t) for t in w.make_tables()[1]]
+    o = O.Oracle(w.cards, w.dims, tabs, w.cache_bytes, O.MODE_GLOBAL)
+    for b in range(260):
+        if b == 230:
+            s0 = o.stats()
+        o.query(w.batch(b).ids)
+    s = o.stats()
+    uh = (s["unique_hits"] - s0["unique_hits"]) / (s["unique_keys"] - s0["unique_keys"])
+    assert abs(uh - paper) < 0.03, (uh, paper)
