@@ -50,6 +50,8 @@ def parse():
     p.add_argument("--host-assist", action="store_true",
                    help="FLECHE_FLAG_HOST_ASSIST: host threads stage the missed rows (paper Fig 8b CPU-DRAM layer)")
     p.add_argument("--cache-frac", type=float, default=None, help="override the config's cache fraction (sweeps)")
+    p.add_argument("--dim", type=int, default=None, help="override every table's row width (sensitivity sweeps)")
+    p.add_argument("--batch", type=int, default=None, help="override the samples per table per batch (sweeps)")
     p.add_argument("--p2p", action="store_true",
                    help="--mode sharded: fused exchange (owners' rows read in place over peer memory)")
     p.add_argument("--watermarks", default=None,
@@ -233,6 +235,10 @@ def main():
     w = configs.get(args.config)
     if args.cache_frac is not None:
         w = w.with_(cache_frac=args.cache_frac)
+    if args.dim is not None:
+        w = w.with_(dims=[args.dim] * w.n)
+    if args.batch is not None:
+        w = w.with_(batch_size=args.batch)
     P = PREFILL.get(args.config, 300) if args.prefill is None else args.prefill
     if args.prefill is None and args.config.startswith("cfg3"):
         P = PREFILL_CFG3.get(round(w.cache_frac, 2), 360)
@@ -465,7 +471,8 @@ def main():
     try:  # committed ncu --set full summary of this config's kernels (profiles/ncu_traffic_r01.json)
         tr = json.load(open(os.path.join(os.path.dirname(os.path.abspath(__file__)), "profiles",
                                          "ncu_traffic_r01.json")))[args.config][dom]
-        if not args.flags and not args.watermarks:
+        if not (args.flags or args.watermarks or args.dim or args.batch or args.cache_frac or args.mode != "replicated"
+                or args.admit_prob != 1.0):  # only the exact captured configuration
             traffic, traffic_src = tr["dram_bytes"], tr["source"]
     except (OSError, KeyError, ValueError):
         pass
