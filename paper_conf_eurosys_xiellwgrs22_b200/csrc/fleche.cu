@@ -839,9 +839,7 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   // KM: enough warps for the expected unique misses, km_bps CTAs of 4 warps per SM
   c->km_blocks = (int)std::min<int64_t>((int64_t)c->km_bps * c->sm_count,
                                         std::max<int64_t>(1, (cfg->max_lookups + 255) / 256));
-  if (const char* e = getenv("FLECHE_KM_WIDE")) dv.km_wide = atoi(e) != 0 && !bytes && !part && dv.ordered;
-  c->km_smem = (size_t)kKmWarps * ((bytes ? kKmSmemF4 : (dv.km_wide ? 32 * c->max_dim / 4 : 0)) +
-                                   ((cfg->flags & FLECHE_FLAG_HOST_ASSIST) ? kHaSmemF4 : 0)) *
+  c->km_smem = (size_t)kKmWarps * ((bytes ? kKmSmemF4 : 0) + ((cfg->flags & FLECHE_FLAG_HOST_ASSIST) ? kHaSmemF4 : 0)) *
                sizeof(float4);
   if (c->km_smem > 48 * 1024 &&
       cudaFuncSetAttribute((const void*)km_fn(bytes, c->cls_dim.size() == 1 ? c->max_dim : 0),

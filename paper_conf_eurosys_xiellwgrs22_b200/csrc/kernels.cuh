@@ -176,7 +176,7 @@ struct Dev {
   // monotone in its host-row address, slot0 = ((addr - host_lo) * host_mul) >> 64, so KM
   // can hand each warp a contiguous address window (host-link reads in address order)
   int32_t ordered;
-  int32_t km_wide;   // ordered uniform path: a warp's misses (up to 32) fly at once via cp.async into smem
+  int32_t pad2;
   uint64_t host_lo, host_mul;
   // host-assisted miss fetch (mapped pinned host memory; see HaReq)
   int32_t ha;                  // 1 = host-assisted miss fetch on
@@ -382,11 +382,6 @@ __device__ __forceinline__ uint32_t ha_kcut(const Dev& dv, const KMArgs& ka, int
 // programmatic stream serialization, so a kernel's launch and prologue overlap the tail
 // of its predecessor; pdl_wait() (griddepcontrol.wait) then blocks until the
 // predecessor grid has completed and its writes are visible.  No-ops otherwise.
-__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
-  const unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(sa), "l"(gmem) : "memory");
-}
-
 __device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
 __device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
 
@@ -1196,75 +1191,6 @@ __device__ __forceinline__ void km_rows(const Dev& dv, float* __restrict__ out, 
     first_chunk = false;
   };
 
-  // wide chunk (dv.km_wide, uniform layout): lane r holds miss r (up to 32); every row of
-  // the chunk goes host -> shared memory with cp.async at once (no registers held), so a
-  // warp whose address window holds more than M misses still waits one link round trip
-  // instead of one per M misses
-  auto wide_chunk = [&](bool has, MissRec m) {
-    if constexpr (!BYTES) {
-      constexpr int VEC = D / 4;
-      float4* myrow = wsm + (size_t)lane * VEC;
-      const TableInfo* ti = dv.tables + (has ? m.t : 0);
-      if (has) {
-        const float* src = ti->host + (size_t)(m.fk - ti->base) * D;
-#pragma unroll
-        for (int c = 0; c < VEC; ++c) cp_async16(myrow + c, src + 4 * c);
-        hostb += 4ull * D;
-      }
-      asm volatile("cp.async.commit_group;" ::: "memory");
-      bool admit = false;
-      if (has)
-        admit = dv.admit_all ||
-                splitmix64(dv.admit_seed ^ (uint64_t)m.fk ^ ((uint64_t)(epoch - 1u) << 32)) < dv.admit_thr;
-      bool pending = has && admit;
-      if (has && !admit) ++byp;
-      const uint32_t pos = pending ? (uint32_t)ld_cg_u64(dv.firstpos + m.scr) : 0u;
-      bool landed = false;
-      while (__any_sync(kFull, pending)) {  // rounds, as in chunk()
-        float* slab_dst = nullptr;
-        int64_t slot = kClaimRetry;
-        if (pending) {
-          uint32_t old_key = kEmpty;
-          bool took = false;
-          slot = claim_victim(dv, ti, m.fk, epoch, pos, &old_key, &took);
-          if (slot >= 0) {
-            pending = false;
-            if (took) {
-              ++byp;
-            } else {
-              ++ins;
-              docc += 4ll * D;
-              if (old_key != kEmpty) { ++ev; docc -= 4ll * D; }
-            }
-            slab_dst = slot_row(dv, ti, (uint32_t)slot, D);
-          } else if (slot == kClaimBypass) {
-            pending = false;
-            ++byp;
-          }
-        }
-        if (!landed) {  // first use of the rows: wait for this warp's copies
-          asm volatile("cp.async.wait_all;" ::: "memory");
-          __syncwarp();
-          landed = true;
-        }
-        copy_rows_generic<D>((const float*)myrow, slab_dst, lane);
-        __syncwarp();
-        if (slab_dst) {
-          dv.keys[slot] = m.fk;
-          __threadfence();
-          *(volatile unsigned long long*)(dv.ipos + slot) = ((unsigned long long)epoch << 32) | ((unsigned long long)pos << 1);
-        }
-        if (slot == kClaimRetry && pending) __nanosleep(100);
-      }
-      if (!landed) {
-        asm volatile("cp.async.wait_all;" ::: "memory");
-        __syncwarp();
-      }
-      copy_rows_generic<D>((const float*)myrow, has ? out + m.off : nullptr, lane);  // owners' output rows
-      __syncwarp();
-    }
-  };
-
   if (BYTES || !dv.ordered) {  // misses from this width's region of the miss list
     for (uint32_t base = gw * M; base < nmiss; base += nw * M) {
       const uint32_t k = base + lane;
@@ -1281,7 +1207,6 @@ __device__ __forceinline__ void km_rows(const Dev& dv, float* __restrict__ out, 
     const uint32_t lo = min(nslots, gw * per), hi = min(nslots, lo + per);
     uint32_t my_slot = 0;
     int P = 0;  // misses collected so far (lanes 0..P-1 hold their slots)
-    const int MW = (!BYTES && dv.km_wide) ? 32 : M;
     auto flush = [&]() {
       MissRec m{};
       const bool has = lane < P;
@@ -1297,8 +1222,7 @@ __device__ __forceinline__ void km_rows(const Dev& dv, float* __restrict__ out, 
         }
         m.t = (int32_t)(dv.kdec[a] & 0xFFFFu);
       }
-      if (MW > M) wide_chunk(has, m);
-      else chunk(has, m);
+      chunk(has, m);
       P = 0;
     };
     for (uint32_t s1 = lo; s1 < hi; s1 += 256) {  // 8 tag loads per lane in flight, then in order
@@ -1317,7 +1241,7 @@ __device__ __forceinline__ void km_rows(const Dev& dv, float* __restrict__ out, 
           found &= found - 1;
           const uint32_t fs = __shfl_sync(kFull, slot, f);
           if (lane == P) my_slot = fs;
-          if (++P == MW) flush();
+          if (++P == M) flush();
         }
       }
     }
@@ -1374,7 +1298,7 @@ __global__ void __launch_bounds__(128, 4) km_kernel(const __grid_constant__ Dev 
   const uint32_t gw = (threadIdx.x >> 5) * gridDim.x + blockIdx.x;
   const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
   // per warp: [kHaSmemF4 host-assisted rows][kKmSmemF4 bytes-layout staging + compaction]
-  const int wsm_f4 = (dv.ha ? kHaSmemF4 : 0) + (BYTES ? kKmSmemF4 : (dv.km_wide ? 32 * dv.dim / 4 : 0));
+  const int wsm_f4 = (dv.ha ? kHaSmemF4 : 0) + (BYTES ? kKmSmemF4 : 0);
   float4* hsm = s_dyn + (threadIdx.x >> 5) * wsm_f4;
   float4* wsm = hsm + (dv.ha ? kHaSmemF4 : 0);
   unsigned ins = 0, ev = 0, byp = 0, harows = 0, hato = 0;
@@ -1462,6 +1386,11 @@ struct KFArgs {
   uint32_t kq_blocks;  // KQ grid size: KQ is complete once kq_cnt reaches it
   int32_t dim;
 };
+
+__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
+  const unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(sa), "l"(gmem) : "memory");
+}
 
 template <int D>
 __global__ void __launch_bounds__(kKfWarps * 32, 16) kf_kernel(const __grid_constant__ Dev dv,

@@ -360,26 +360,3 @@ def test_early_fetch_cfg2_full_size(monkeypatch):
             for k in H.STAT_KEYS_EXACT:
                 assert dg[k] == do[k], (b, k)
 
-
-@pytest.mark.parametrize("case", ["small", "cfg2"])
-def test_km_wide_chunks_exact(monkeypatch, case):
-    """FLECHE_KM_WIDE=1: the address-ordered miss fetch takes up to 32 misses per warp at
-    once (cp.async into shared memory); values and every counter stay exact."""
-    monkeypatch.setenv("FLECHE_KM_WIDE", "1")
-    if case == "small":
-        monkeypatch.setenv("FLECHE_ORDER_MIN_SPAN", "0")
-        w = configs.get("cfg0").with_(cache_frac=0.02, invalid_ppm=3000, skews=[0.7] * 7)
-        _run(w, _tables(w), 25)
-    else:
-        w = configs.get("cfg2")
-        tabs = _tables(w)
-        gpu, seta = H.make_pair(w, tabs, O.MODE_SETASSOC)
-        for b in range(30):
-            bt = w.batch(b)
-            g0, o0 = gpu.stats(), seta.stats()
-            got = H.run_batch_gpu(gpu, bt.ids, torch)
-            assert H.bits_equal(got, seta.query(bt.ids)), b
-            dg, do = H.delta(g0, gpu.stats()), H.delta(o0, seta.stats())
-            if do["bypassed"] == 0:
-                for k in H.STAT_KEYS_EXACT:
-                    assert dg[k] == do[k], (b, k)
