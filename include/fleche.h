@@ -196,9 +196,12 @@ fleche_status fleche_query_pooled(fleche_ctx* ctx, const int64_t* const* ids, co
                                   const int64_t* bags, const int64_t* nnz, float* out, fleche_stream stream);
 
 /* Same lookups with HOST buffers: ids[t] are host pointers (ideally pinned), out is a
- * host buffer.  Enqueues host->device copies of the IDs, the query, and the
- * device->host copy of out on `stream` (ctx-owned device staging, allocated at the
- * first call).  Asynchronous: out is complete once the stream is synchronised. */
+ * host buffer.  Enqueues host->device copies of the IDs and the query on a ctx-owned
+ * stream (after whatever `stream` holds), and the device->host copy of out on a second
+ * ctx-owned stream from one of two staging buffers, so consecutive calls overlap one
+ * call's output copy with the next call's lookups; `stream` waits for the copy.
+ * Asynchronous: out is complete once `stream` is synchronised (ctx-owned device staging,
+ * allocated at the first call). */
 fleche_status fleche_query_host(fleche_ctx* ctx, const int64_t* const* ids, const int64_t* lengths, float* out,
                                 fleche_stream stream);
 

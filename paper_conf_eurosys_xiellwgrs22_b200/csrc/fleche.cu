@@ -100,6 +100,10 @@ struct fleche_ctx {
   // fleche_query_host staging and pooled staging (lazy)
   int64_t* d_ids_stage = nullptr;
   float* d_out_stage = nullptr;
+  float* d_out_stage2 = nullptr;   // fleche_query_host: second staging buffer (pipelined copies)
+  cudaStream_t hq = nullptr, hd = nullptr;
+  cudaEvent_t hq_ev[2] = {nullptr, nullptr}, hd_ev[2] = {nullptr, nullptr};
+  int hpar = 0;
   float* d_pool_stage = nullptr;
   uint64_t index_bytes = 0;
   // profiling (fleche_set_profiling)
@@ -410,7 +414,7 @@ void free_all(fleche_ctx* c) {
                   c->dv.miss, c->dv.dup, c->dv.ctl, c->dv.stats, c->d_tables, c->d_ids_stage, c->d_out_stage,
                   c->d_pool_stage, c->d_kdec, c->rd.scratch, c->rd.slotval, c->rd.inv, c->rd.region, c->rd.cnt,
                   c->rd.prefix, c->rd.done, c->rd.stats, c->d_slots, c->d_age_hist, c->d_prefill_out,
-                  c->dv.mready};
+                  c->dv.mready, c->d_out_stage2};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   for (auto& r : c->registered) cudaHostUnregister(r.first);
@@ -419,6 +423,12 @@ void free_all(fleche_ctx* c) {
   if (c->fork_ev) cudaEventDestroy(c->fork_ev);
   if (c->join_ev) cudaEventDestroy(c->join_ev);
   if (c->kf_ev) cudaEventDestroy(c->kf_ev);
+  for (int i = 0; i < 2; ++i) {
+    if (c->hq_ev[i]) cudaEventDestroy(c->hq_ev[i]);
+    if (c->hd_ev[i]) cudaEventDestroy(c->hd_ev[i]);
+  }
+  if (c->hq) cudaStreamDestroy(c->hq);
+  if (c->hd) cudaStreamDestroy(c->hd);
   if (c->side) cudaStreamDestroy(c->side);
   for (cudaEvent_t e : c->ev_pool) cudaEventDestroy(e);
   c->ev_pool.clear();
@@ -1016,11 +1026,30 @@ fleche_status fleche_query_host(fleche_ctx* c, const int64_t* const* ids, const 
   if (total > c->max_lookups || (total > 0 && !out)) return FLECHE_EINVAL;
   fleche_status st = ensure_device(c);
   if (st != FLECHE_OK) return st;
-  cudaStream_t s = (cudaStream_t)stream;
+  // Pipelined across calls: the lookups run on the ctx's host-call stream hq, the output
+  // copy on a second stream hd from one of two staging buffers, so call k's device->host
+  // copy overlaps call k+1's query; the caller's stream waits for this call's copy (out is
+  // complete once it is synchronised).
+  const cudaStream_t caller = (cudaStream_t)stream;
   if (!c->d_ids_stage) {
     FL_CUDA(c, cudaMalloc((void**)&c->d_ids_stage, (size_t)c->max_lookups * 8));
     FL_CUDA(c, cudaMalloc((void**)&c->d_out_stage, (size_t)c->max_lookups * (size_t)c->max_dim * 4));
+    FL_CUDA(c, cudaMalloc((void**)&c->d_out_stage2, (size_t)c->max_lookups * (size_t)c->max_dim * 4));
+    FL_CUDA(c, cudaStreamCreateWithFlags(&c->hq, cudaStreamNonBlocking));
+    FL_CUDA(c, cudaStreamCreateWithFlags(&c->hd, cudaStreamNonBlocking));
+    for (int i = 0; i < 2; ++i) {
+      FL_CUDA(c, cudaEventCreateWithFlags(&c->hq_ev[i], cudaEventDisableTiming));
+      FL_CUDA(c, cudaEventCreateWithFlags(&c->hd_ev[i], cudaEventDisableTiming));
+      FL_CUDA(c, cudaEventRecord(c->hd_ev[i], c->hd));
+    }
   }
+  const int par = c->hpar;
+  c->hpar ^= 1;
+  float* stage = par ? c->d_out_stage2 : c->d_out_stage;
+  const cudaStream_t s = c->hq;
+  FL_CUDA(c, cudaStreamWaitEvent(s, c->hd_ev[par], 0));  // the copy that last read this staging buffer
+  FL_CUDA(c, cudaEventRecord(c->hq_ev[par], caller));     // and whatever the caller enqueued before
+  FL_CUDA(c, cudaStreamWaitEvent(s, c->hq_ev[par], 0));
   st = order_on(c, s);
   if (st != FLECHE_OK) return st;
   std::vector<const int64_t*> dids(c->n);
@@ -1039,10 +1068,14 @@ fleche_status fleche_query_host(fleche_ctx* c, const int64_t* const* ids, const 
   }
   if (contiguous && total > 0)
     FL_CUDA(c, cudaMemcpyAsync(c->d_ids_stage, first, (size_t)total * 8, cudaMemcpyHostToDevice, s));
-  st = query_impl(c, dids.data(), lengths, c->d_out_stage, s);
+  st = query_impl(c, dids.data(), lengths, stage, s);
   if (st != FLECHE_OK) return st;
+  FL_CUDA(c, cudaEventRecord(c->hq_ev[par], s));
+  FL_CUDA(c, cudaStreamWaitEvent(c->hd, c->hq_ev[par], 0));
   if (out_floats > 0)
-    FL_CUDA(c, cudaMemcpyAsync(out, c->d_out_stage, (size_t)out_floats * 4, cudaMemcpyDeviceToHost, s));
+    FL_CUDA(c, cudaMemcpyAsync(out, stage, (size_t)out_floats * 4, cudaMemcpyDeviceToHost, c->hd));
+  FL_CUDA(c, cudaEventRecord(c->hd_ev[par], c->hd));
+  FL_CUDA(c, cudaStreamWaitEvent(caller, c->hd_ev[par], 0));
   return FLECHE_OK;
 }
 
@@ -1101,6 +1134,7 @@ fleche_status fleche_destroy(fleche_ctx* c) {
   cudaGetDevice(&cur);
   if (cur != c->device) cudaSetDevice(c->device);
   if (c->have_last) cudaStreamSynchronize(c->last_stream);
+  if (c->hd) cudaStreamSynchronize(c->hd);  // fleche_query_host's last output copy
   free_all(c);
   delete c;
   return FLECHE_OK;

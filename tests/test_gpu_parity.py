@@ -360,3 +360,34 @@ def test_early_fetch_cfg2_full_size(monkeypatch):
             for k in H.STAT_KEYS_EXACT:
                 assert dg[k] == do[k], (b, k)
 
+
+
+def test_host_buffer_calls_pipelined_back_to_back():
+    """fleche_query_host overlaps call k's output copy with call k+1's lookups (two staging
+    buffers): six calls enqueued without a sync, then a device-buffer query, must all equal
+    the oracle run in call order."""
+    w = configs.get("cfg0").with_(cache_frac=0.05, invalid_ppm=2000)
+    tabs = _tables(w)
+    gpu, orc = H.make_pair(w, tabs)
+    s = torch.cuda.Stream()
+    outs, refs = [], []
+    for b in range(6):
+        bt = w.batch(b)
+        lens = [x.size for x in bt.ids]
+        ids = [torch.from_numpy(x).pin_memory().numpy() for x in bt.ids]
+        out = torch.empty(gpu.out_floats(lens), dtype=torch.float32).pin_memory()
+        gpu.query_host(ids, out.numpy(), stream=s)
+        outs.append((out, ids))
+        refs.append(orc.query(bt.ids))
+    bt = w.batch(6)
+    dev_ids = [torch.from_numpy(x).cuda() for x in bt.ids]
+    dout = torch.empty(gpu.out_floats([x.size for x in bt.ids]), device="cuda")
+    gpu.query(dev_ids, dout)  # another stream: ordered after the host calls by the ctx
+    s.synchronize()
+    torch.cuda.synchronize()
+    for (out, _), ref in zip(outs, refs):
+        assert H.bits_equal(out.numpy(), ref)
+    assert H.bits_equal(dout.cpu().numpy(), orc.query(bt.ids))
+    so, sg = orc.stats(), gpu.stats()
+    for k in H.STAT_KEYS_EXACT:
+        assert sg[k] == so[k], k
