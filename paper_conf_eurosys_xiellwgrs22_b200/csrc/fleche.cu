@@ -942,6 +942,7 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
       const char* e = getenv("FLECHE_HA_FRAC");
       const double f = e ? std::min(1.0, std::max(0.0, atof(e))) : 0.5;
       dv.ha_frac_q16 = (uint32_t)(f * 65536.0 + 0.5);
+      dv.ha_min_rows = (uint32_t)env_u("FLECHE_HA_MIN_ROWS", 32768);
     }
     h->nt_stores = env_u("FLECHE_HA_NT", 1) != 0 && __builtin_cpu_supports("avx2");
     h->host.assign(cfg->host_tables, cfg->host_tables + n);

@@ -52,7 +52,7 @@ constexpr int kKmWarps = 4;     // KM CTA = 4 warps
 constexpr int kKmStageF4 = 256; // bytes layout, per warp: staged rows of a chunk (<= 4 KB) ...
 constexpr int kKmSmemF4 = 512;  // ... + the compaction buffer of one set region (<= 4 KB)
 constexpr int kHaBlock = 64;    // host-assisted miss fetch: rows per staging block (one ready flag)
-constexpr int kHaSmemF4 = 1024; // host-assisted KM, per warp: 16 KB of rows landed from the host
+constexpr int kHaSmemF4 = 512;  // host-assisted KM, per warp: 8 KB of rows landed from the host (4 KM CTAs per SM)
 
 enum Ctr : int {
   C_HITS = 0,
@@ -190,7 +190,7 @@ struct Dev {
   uint64_t ha_stage_floats;
   uint64_t ha_timeout_ns;
   uint32_t ha_frac_q16;        // share of the batch's staging blocks given to the host threads (x 2^-16)
-  uint32_t ha_pad2;
+  uint32_t ha_min_rows;        // batches with fewer unique misses stay all zero-copy (the split loses there)
 #ifdef FLECHE_EXPERIMENTS
   int32_t exp_mode;  // timing experiments only (libfleche_exp.so); breaks semantics
   int32_t exp_pad;
@@ -365,6 +365,16 @@ __device__ __forceinline__ bool ha_wait_block(const uint32_t* flag, const uint32
 // threads gather the first ceil(frac * nblocks) of them while KM's other warps read the
 // rest zero-copy from the tables at the same time (two independent paths to the rows:
 // host cores + contiguous link reads, and the GPU's own translated reads).
+// Host-assisted fetch active for this batch: enough unique misses (FLECHE_HA_MIN_ROWS) and
+// a non-zero share.  Otherwise KM takes the plain (address-ordered) zero-copy path and the
+// host threads are not woken.
+__device__ __forceinline__ bool ha_active(const Dev& dv, const KMArgs& ka, int par) {
+  if (!dv.ha || !dv.ha_frac_q16) return false;
+  uint32_t total = 0;
+  for (int c = 0; c < ka.ncls; ++c) total += *(volatile uint32_t*)&dv.ctl->counts[par][c];
+  return total >= dv.ha_min_rows;
+}
+
 __device__ __forceinline__ uint32_t ha_kcut(const Dev& dv, const KMArgs& ka, int par) {
   uint32_t lo = 0xFFFFFFFFu, hi = 0;
   for (int c = 0; c < ka.ncls; ++c) {
@@ -375,6 +385,9 @@ __device__ __forceinline__ uint32_t ha_kcut(const Dev& dv, const KMArgs& ka, int
   }
   if (hi == 0) return 0;
   const uint32_t kb0 = lo / kHaBlock, nb = (hi - 1) / kHaBlock - kb0 + 1;
+  uint32_t total = 0;
+  for (int c = 0; c < ka.ncls; ++c) total += *(volatile uint32_t*)&dv.ctl->counts[par][c];
+  if (total < dv.ha_min_rows) return kb0;  // small batch: the round trip to the host threads is not hidden
   return kb0 + (uint32_t)(((unsigned long long)nb * dv.ha_frac_q16 + 65535ull) >> 16);
 }
 
@@ -1274,7 +1287,8 @@ __global__ void __launch_bounds__(128, 4) km_kernel(const __grid_constant__ Dev 
   const uint32_t epoch = *(volatile uint32_t*)&dv.ctl->epoch;
   const int par = epoch & 1u;
   const int lane = threadIdx.x & 31;
-  if (dv.ha && blockIdx.x == 0 && threadIdx.x == 0) {
+  const bool use_ha = ha_active(dv, ka, par);
+  if (use_ha && blockIdx.x == 0 && threadIdx.x == 0) {
     // host-assisted: ring the doorbell.  KQ (the previous grid in stream order) wrote the
     // requests; this fence orders them before the doorbell for the host threads.
     HaDesc hd;
@@ -1303,14 +1317,14 @@ __global__ void __launch_bounds__(128, 4) km_kernel(const __grid_constant__ Dev 
   float4* wsm = hsm + (dv.ha ? kHaSmemF4 : 0);
   unsigned ins = 0, ev = 0, byp = 0, harows = 0, hato = 0;
   long long docc = 0;
-  const uint32_t kcut = dv.ha ? ha_kcut(dv, ka, par) : 0u;
+  const uint32_t kcut = use_ha ? ha_kcut(dv, ka, par) : 0u;
   unsigned long long hostb = 0;
   for (int c = 0; c < ka.ncls; ++c) {
     const uint32_t nmiss = *(volatile uint32_t*)&dv.ctl->counts[par][c];
     if (!nmiss) continue;
     const MissRec* ml = dv.miss + ka.cls_off[c];
 #define FL_KM(D)                                                                                              \
-  if (dv.ha)                                                                                                  \
+  if (use_ha)                                                                                                 \
     km_ha<BYTES, D>(dv, ka.out, ml, epoch, nmiss, lane, gw, nw, ins, ev, byp, docc, hostb, hsm, wsm, harows, hato, kcut); \
   else                                                                                                        \
     km_rows<BYTES, D, KmM<BYTES, D>::value>(dv, ka.out, ml, epoch, nmiss, lane, gw, nw, ins, ev, byp, docc, hostb, wsm, \

@@ -32,6 +32,7 @@ def _need_gpu():
 def _all_blocks_to_host(monkeypatch):
     # the tests below check the staged path itself: the host threads take every block
     monkeypatch.setenv("FLECHE_HA_FRAC", "1")
+    monkeypatch.setenv("FLECHE_HA_MIN_ROWS", "0")
 
 
 def _tables(w):
@@ -166,3 +167,13 @@ def test_split_between_host_threads_and_zero_copy(monkeypatch, frac):
         assert st["assisted_rows"] == 0
     else:
         assert 0 < st["assisted_rows"] < st["unique_misses"], st
+
+
+def test_small_batches_stay_zero_copy(monkeypatch):
+    """FLECHE_HA_MIN_ROWS: a batch with fewer unique misses is fetched all zero-copy (the
+    host threads get no blocks); values and counters stay exact."""
+    monkeypatch.setenv("FLECHE_HA_MIN_ROWS", "1000000")
+    w = configs.get("cfg0").with_(cache_frac=0.25)
+    gpu, orc = _run(w, _tables(w), 6)
+    st = gpu.stats()
+    assert st["assisted_rows"] == 0 and st["assist_timeouts"] == 0 and st["unique_misses"] > 0
