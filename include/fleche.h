@@ -119,8 +119,8 @@ typedef struct {
  * zero-copy from the tables instead, so correctness never depends on the threads.  Env:
  * FLECHE_HA_THREADS (default 12), FLECHE_HA_STAGE_KB (staging per epoch parity, default
  * 131072; rows beyond it are read zero-copy), FLECHE_HA_FRAC (share of the batch's
- * staging blocks the host threads take, default 0.5; KM reads the rest zero-copy at the
- * same time), FLECHE_HA_MIN_ROWS (batches with fewer unique misses stay all zero-copy,
+ * staging blocks the host threads take, default 0.5, or 0.85 for host tiers over 32 GiB;
+ * KM reads the rest zero-copy at the same time), FLECHE_HA_MIN_ROWS (batches with fewer unique misses stay all zero-copy,
  * default 32768: below it the round trip to the host threads is not hidden).  Not with PER_TABLE_LAUNCH (FLECHE_EINVAL).  `out`, hits and every cache decision are identical with and without
  * it; only where the missed rows are read from changes. */
 #define FLECHE_FLAG_HOST_ASSIST 0x8u

@@ -939,8 +939,13 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
     dv.ha_stage_floats = h->stage_floats;
     dv.ha_timeout_ns = env_u("FLECHE_HA_TIMEOUT_US", 2000) * 1000ull;
     {  // share of the staging blocks the host threads gather (the rest: KM's zero-copy reads)
+      // default share: the host threads' share pays off more the larger the host tier (the
+      // GPU's translated reads slow down with the span): measured best ~0.5-0.6 at 8.6 GB
+      // (cfg5), >= 0.85 at 113 GB (cfg3h); profiles/bench_r01_*ha*.json
+      uint64_t span = 0;
+      for (int t = 0; t < n; ++t) span += (uint64_t)c->card[t] * (uint64_t)c->dims[t] * 4u;
       const char* e = getenv("FLECHE_HA_FRAC");
-      const double f = e ? std::min(1.0, std::max(0.0, atof(e))) : 0.5;
+      const double f = e ? std::min(1.0, std::max(0.0, atof(e))) : (span > (32ull << 30) ? 0.85 : 0.5);
       dv.ha_frac_q16 = (uint32_t)(f * 65536.0 + 0.5);
       dv.ha_min_rows = (uint32_t)env_u("FLECHE_HA_MIN_ROWS", 32768);
     }

@@ -37,7 +37,8 @@
 #define FL_GATHER_F4 8  // float4 loads per lane in flight in a row gather (A/B builds vary it)
 #endif
 #ifndef FL_KQ_MIN_BLOCKS
-#define FL_KQ_MIN_BLOCKS 1  // KQ CTAs per SM the register budget must allow (A/B builds vary it)
+#define FL_KQ_MIN_BLOCKS 8  // KQ CTAs per SM the register budget must allow: 8 (64 regs, no spill) measured
+                            // KQ 33.4 vs 35.5 us at 5 CTAs (profiles/bench_r01_kq_occupancy_*.json)
 #endif
 
 namespace fl {
