@@ -391,3 +391,24 @@ def test_host_buffer_calls_pipelined_back_to_back():
     so, sg = orc.stats(), gpu.stats()
     for k in H.STAT_KEYS_EXACT:
         assert sg[k] == so[k], k
+
+
+@pytest.mark.parametrize("n,d", [(300, 8), (513 - 1, 16), (5, 256), (9, 8)])
+def test_table_count_and_width_extremes(n, d):
+    """The 512-table kernel instantiation (n > 128), and the narrowest / widest uniform rows
+    (d = 8, 256): bit-exact and exact stats vs the set oracle, with ragged and empty tables."""
+    rng = np.random.default_rng(n * 1000 + d)
+    cards = [int(x) for x in rng.integers(1, 3000, n)]
+    w = configs.Workload("edge", 9, cards, [d] * n, [1.0] * n, 40, 0.05, invalid_ppm=5000)
+    tabs = _tables(w)
+    gpu, orc = H.make_pair(w, tabs)
+    for b in range(6):
+        bt = w.batch(b)
+        ids = [x[: int(rng.integers(0, x.size + 1))] for x in bt.ids]  # ragged, some empty
+        g0, o0 = gpu.stats(), orc.stats()
+        got = H.run_batch_gpu(gpu, ids, torch)
+        assert H.bits_equal(got, orc.query(ids)), b
+        dg, do = H.delta(g0, gpu.stats()), H.delta(o0, orc.stats())
+        if do["bypassed"] == 0:
+            for k in H.STAT_KEYS_EXACT:
+                assert dg[k] == do[k], (b, k)
