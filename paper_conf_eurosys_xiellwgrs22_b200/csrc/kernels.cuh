@@ -918,25 +918,28 @@ static __device__ bool bytes_insert(const Dev& dv, uint32_t fk, int units, const
       }
       words[w] = __reduce_or_sync(kFull, mine);
     }
+    // first fit at an offset aligned to the row's size (row sizes are powers of two in
+    // 32 B units): aligned power-of-two blocks keep the region from fragmenting, so the
+    // compaction below is rarely needed (placement only; which rows are cached is unchanged)
     int start = -1;
     for (int base = 0; base < SU && start < 0; base += 32) {
       const int p = base + lane;
-      bool fits = p + units <= SU;
+      bool fits = p + units <= SU && (p & (units - 1)) == 0;
       for (int u = 0; u < units && fits; ++u) fits = !((words[(p + u) >> 5] >> ((p + u) & 31)) & 1u);
       const unsigned b = __ballot_sync(kFull, fits);
       if (b) start = base + __ffs(b) - 1;
     }
-    if (start < 0) {  // fragmented: pack the live rows to the front through smem
+    if (start < 0) {  // fragmented: pack the live rows to the front through smem, largest first
       float* region = dv.slab + (size_t)s * SU * 8u;
       for (int c = lane; c < SU * 2; c += 32) cbuf[c] = ld_cg_v4(region + 4 * c);
       __syncwarp();
-      int incl = my_sz;
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const int y = __shfl_up_sync(kFull, incl, o);
-        if (lane >= o) incl += y;
+      // new offset = bytes of the rows packed before mine: larger rows, then equal rows of
+      // lower way (descending power-of-two sizes keep every row aligned)
+      int new_off = 0;
+      for (int w = 0; w < 32; ++w) {
+        const int wsz = __shfl_sync(kFull, my_sz, w);
+        if (wsz > my_sz || (wsz == my_sz && w < lane)) new_off += wsz;
       }
-      const int new_off = incl - my_sz;
       for (int w = 0; w < 32; ++w) {
         const int wsz = __shfl_sync(kFull, my_sz, w);
         if (!wsz) continue;
@@ -944,7 +947,8 @@ static __device__ bool bytes_insert(const Dev& dv, uint32_t fk, int units, const
         for (int c = lane; c < wsz * 2; c += 32) st_v4(region + (size_t)(wn * 2 + c) * 4, cbuf[wo * 2 + c]);
       }
       if (live) *lp = (uint16_t)((my_sz << 8) | new_off);
-      start = used;
+      const int aligned = (used + units - 1) & ~(units - 1);
+      start = aligned + units <= SU ? aligned : used;
       __syncwarp();
     }
     float* dst = dv.slab + ((size_t)s * SU + start) * 8u;
