@@ -36,6 +36,9 @@
 #ifndef FL_GATHER_F4
 #define FL_GATHER_F4 8  // float4 loads per lane in flight in a row gather (A/B builds vary it)
 #endif
+#ifndef FL_KQ_PROBE
+#define FL_KQ_PROBE 32  // index lines per lane in flight in KQ's probe (a divisor of 32; A/B builds vary it)
+#endif
 #ifndef FL_KQ_MIN_BLOCKS
 #define FL_KQ_MIN_BLOCKS 8  // KQ CTAs per SM the register budget must allow: 8 (64 regs, no spill) measured
                             // KQ 33.4 vs 35.5 us at 5 CTAs (profiles/bench_r01_kq_occupancy_*.json)
@@ -602,18 +605,22 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
     const uint32_t s = valid ? set_of_t(dv, ti, fk) : 0u;
 
     // A3 probe: lane k holds way k of each of the warp's 32 sets (one 128 B line each)
-    uint32_t kw[32];
-#pragma unroll
-    for (int i = 0; i < 32; ++i) {
-      const uint32_t si = __shfl_sync(kFull, s, i);
-      kw[i] = ld_nc_u32(dv.keys + (size_t)si * 32u + lane);
-    }
+    // (FL_KQ_PROBE lines in flight per lane: fewer registers, more CTAs per SM)
     int way = -1;
 #pragma unroll
-    for (int i = 0; i < 32; ++i) {
-      const uint32_t fki = __shfl_sync(kFull, fk, i);
-      const unsigned m = __ballot_sync(kFull, kw[i] == fki);
-      if (lane == i && m) way = __ffs(m) - 1;
+    for (int i0 = 0; i0 < 32; i0 += FL_KQ_PROBE) {
+      uint32_t kw[FL_KQ_PROBE];
+#pragma unroll
+      for (int i = 0; i < FL_KQ_PROBE; ++i) {
+        const uint32_t si = __shfl_sync(kFull, s, i0 + i);
+        kw[i] = ld_nc_u32(dv.keys + (size_t)si * 32u + lane);
+      }
+#pragma unroll
+      for (int i = 0; i < FL_KQ_PROBE; ++i) {
+        const uint32_t fki = __shfl_sync(kFull, fk, i0 + i);
+        const unsigned m = __ballot_sync(kFull, kw[i] == fki);
+        if (lane == i0 + i && m) way = __ffs(m) - 1;
+      }
     }
     const bool hit = valid && way >= 0;
     const bool miss = valid && way < 0;
