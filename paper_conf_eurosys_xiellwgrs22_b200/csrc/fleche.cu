@@ -102,7 +102,7 @@ struct fleche_ctx {
   float* d_out_stage = nullptr;
   float* d_out_stage2 = nullptr;   // fleche_query_host: second staging buffer (pipelined copies)
   cudaStream_t hq = nullptr, hd = nullptr;
-  cudaEvent_t hq_ev[2] = {nullptr, nullptr}, hd_ev[2] = {nullptr, nullptr};
+  cudaEvent_t hq_ev[2] = {nullptr, nullptr}, hd_ev[2] = {nullptr, nullptr}, hc_ev[2] = {nullptr, nullptr};
   int hpar = 0;
   float* d_pool_stage = nullptr;
   uint64_t index_bytes = 0;
@@ -426,6 +426,7 @@ void free_all(fleche_ctx* c) {
   for (int i = 0; i < 2; ++i) {
     if (c->hq_ev[i]) cudaEventDestroy(c->hq_ev[i]);
     if (c->hd_ev[i]) cudaEventDestroy(c->hd_ev[i]);
+    if (c->hc_ev[i]) cudaEventDestroy(c->hc_ev[i]);
   }
   if (c->hq) cudaStreamDestroy(c->hq);
   if (c->hd) cudaStreamDestroy(c->hd);
@@ -1034,8 +1035,8 @@ fleche_status fleche_query_host(fleche_ctx* c, const int64_t* const* ids, const 
   if (st != FLECHE_OK) return st;
   // Pipelined across calls: the lookups run on the ctx's host-call stream hq, the output
   // copy on a second stream hd from one of two staging buffers, so call k's device->host
-  // copy overlaps call k+1's query; the caller's stream waits for this call's copy (out is
-  // complete once it is synchronised).
+  // copy overlaps call k+1's H2D + query; the caller's stream waits for this call's copy
+  // (out is complete once it is synchronised).
   const cudaStream_t caller = (cudaStream_t)stream;
   if (!c->d_ids_stage) {
     FL_CUDA(c, cudaMalloc((void**)&c->d_ids_stage, (size_t)c->max_lookups * 8));
@@ -1046,6 +1047,7 @@ fleche_status fleche_query_host(fleche_ctx* c, const int64_t* const* ids, const 
     for (int i = 0; i < 2; ++i) {
       FL_CUDA(c, cudaEventCreateWithFlags(&c->hq_ev[i], cudaEventDisableTiming));
       FL_CUDA(c, cudaEventCreateWithFlags(&c->hd_ev[i], cudaEventDisableTiming));
+      FL_CUDA(c, cudaEventCreateWithFlags(&c->hc_ev[i], cudaEventDisableTiming));
       FL_CUDA(c, cudaEventRecord(c->hd_ev[i], c->hd));
     }
   }
@@ -1053,9 +1055,17 @@ fleche_status fleche_query_host(fleche_ctx* c, const int64_t* const* ids, const 
   c->hpar ^= 1;
   float* stage = par ? c->d_out_stage2 : c->d_out_stage;
   const cudaStream_t s = c->hq;
-  FL_CUDA(c, cudaStreamWaitEvent(s, c->hd_ev[par], 0));  // the copy that last read this staging buffer
-  FL_CUDA(c, cudaEventRecord(c->hq_ev[par], caller));     // and whatever the caller enqueued before
-  FL_CUDA(c, cudaStreamWaitEvent(s, c->hq_ev[par], 0));
+  // The lookups wait for the copy that last read this staging buffer and for whatever
+  // `stream` holds -- which includes the previous call's output copy, so by default call
+  // k's copy and call k+1's lookups run one after the other.  FLECHE_HOST_OVERLAP=1
+  // (experimental) drops the wait on `stream` (host IDs must then be final at the call) so
+  // the copy overlaps the next lookups: measured 196 and 65 Mkeys/s e2e in two runs on one
+  // box vs 169-175 ordered (the device->host copy and KM's zero-copy host reads contend),
+  // hence off.  The output copy below always orders after `stream`'s work.
+  FL_CUDA(c, cudaStreamWaitEvent(s, c->hd_ev[par], 0));
+  FL_CUDA(c, cudaEventRecord(c->hc_ev[par], caller));
+  static const bool overlap = getenv("FLECHE_HOST_OVERLAP") != nullptr;
+  if (!overlap) FL_CUDA(c, cudaStreamWaitEvent(s, c->hc_ev[par], 0));
   st = order_on(c, s);
   if (st != FLECHE_OK) return st;
   std::vector<const int64_t*> dids(c->n);
@@ -1078,6 +1088,7 @@ fleche_status fleche_query_host(fleche_ctx* c, const int64_t* const* ids, const 
   if (st != FLECHE_OK) return st;
   FL_CUDA(c, cudaEventRecord(c->hq_ev[par], s));
   FL_CUDA(c, cudaStreamWaitEvent(c->hd, c->hq_ev[par], 0));
+  FL_CUDA(c, cudaStreamWaitEvent(c->hd, c->hc_ev[par], 0));  // whatever `stream` held (e.g. reads of out)
   if (out_floats > 0)
     FL_CUDA(c, cudaMemcpyAsync(out, stage, (size_t)out_floats * 4, cudaMemcpyDeviceToHost, c->hd));
   FL_CUDA(c, cudaEventRecord(c->hd_ev[par], c->hd));

@@ -393,6 +393,29 @@ def test_host_buffer_calls_pipelined_back_to_back():
         assert sg[k] == so[k], k
 
 
+def test_query_host_output_copy_orders_after_stream():
+    """fleche_query_host's output copy orders after `stream` (also with the experimental
+    FLECHE_HOST_OVERLAP, where the lookups do not): a read of `out` the caller enqueued on
+    `stream` between two calls into the same host buffer sees the first call's rows."""
+    w = configs.get("cfg0").with_(cache_frac=0.05)
+    tabs = _tables(w)
+    gpu, orc = H.make_pair(w, tabs)
+    s = torch.cuda.Stream()
+    bt0, bt1 = w.batch(0), w.batch(1)
+    lens = [x.size for x in bt0.ids]
+    ids0 = [torch.from_numpy(x).pin_memory().numpy() for x in bt0.ids]
+    ids1 = [torch.from_numpy(x).pin_memory().numpy() for x in bt1.ids]
+    out = torch.empty(gpu.out_floats(lens), dtype=torch.float32).pin_memory()
+    snap = torch.empty(out.numel(), device="cuda")
+    gpu.query_host(ids0, out.numpy(), stream=s)
+    with torch.cuda.stream(s):
+        snap.copy_(out, non_blocking=True)  # reads out on `stream`, before call 2 overwrites it
+    gpu.query_host(ids1, out.numpy(), stream=s)
+    s.synchronize()
+    assert H.bits_equal(snap.cpu().numpy(), orc.query(bt0.ids))
+    assert H.bits_equal(out.numpy(), orc.query(bt1.ids))
+
+
 @pytest.mark.parametrize("n,d", [(300, 8), (513 - 1, 16), (5, 256), (9, 8)])
 def test_table_count_and_width_extremes(n, d):
     """The 512-table kernel instantiation (n > 128), and the narrowest / widest uniform rows
