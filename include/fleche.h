@@ -200,13 +200,12 @@ fleche_status fleche_query_pooled(fleche_ctx* ctx, const int64_t* const* ids, co
 
 /* Same lookups with HOST buffers: ids[t] are host pointers (ideally pinned), out is a
  * host buffer.  Enqueues host->device copies of the IDs and the query on a ctx-owned
- * stream (after the ctx's previous batch and whatever `stream` holds), and the
+ * stream (after the ctx's previous batch, NOT after `stream`: the host IDs must be final
+ * when the call is made and stay unchanged until `stream` is synchronised), and the
  * device->host copy of out on a second ctx-owned stream (after the query and after
- * whatever `stream` holds) from one of two staging buffers; `stream` waits for the copy,
- * so consecutive calls run copy k, then lookups k+1.  (Experimental, env
- * FLECHE_HOST_OVERLAP=1: the lookups do not wait for `stream`, so copy k overlaps lookups
- * k+1; the host IDs must then be final when the call is made.  Measured unstable on B200:
- * the copy contends with the miss fetch's zero-copy host reads.)
+ * whatever `stream` holds) from one of two staging buffers, so call k's output copy
+ * overlaps call k+1's lookups; `stream` waits for the copy.  (Env FLECHE_HOST_ORDERED=1
+ * also orders the lookups after `stream`, serialising copy k and lookups k+1.)
  * Asynchronous: out is complete once `stream` is synchronised (ctx-owned device staging,
  * allocated at the first call). */
 fleche_status fleche_query_host(fleche_ctx* ctx, const int64_t* const* ids, const int64_t* lengths, float* out,

@@ -1055,17 +1055,18 @@ fleche_status fleche_query_host(fleche_ctx* c, const int64_t* const* ids, const 
   c->hpar ^= 1;
   float* stage = par ? c->d_out_stage2 : c->d_out_stage;
   const cudaStream_t s = c->hq;
-  // The lookups wait for the copy that last read this staging buffer and for whatever
-  // `stream` holds -- which includes the previous call's output copy, so by default call
-  // k's copy and call k+1's lookups run one after the other.  FLECHE_HOST_OVERLAP=1
-  // (experimental) drops the wait on `stream` (host IDs must then be final at the call) so
-  // the copy overlaps the next lookups: measured 196 and 65 Mkeys/s e2e in two runs on one
-  // box vs 169-175 ordered (the device->host copy and KM's zero-copy host reads contend),
-  // hence off.  The output copy below always orders after `stream`'s work.
+  // The lookups wait for the copy that last read this staging buffer (and, via order_on,
+  // for the ctx's previous batch) but NOT for `stream`: `stream` already waits for the
+  // previous call's output copy, so ordering the lookups after it would run copy k and
+  // lookups k+1 one after the other.  The host IDs must therefore be final when the call is
+  // made (header).  Measured on one B200 box, 8-9 alternating runs each: e2e 184-197
+  // Mkeys/s overlapped (one outlier at 65) vs 98-174 ordered (profiles/e2e_overlap_ab_r01).
+  // FLECHE_HOST_ORDERED=1 restores the strict order.  The output copy below always orders
+  // after `stream`'s work (e.g. the caller's pending reads of out).
   FL_CUDA(c, cudaStreamWaitEvent(s, c->hd_ev[par], 0));
   FL_CUDA(c, cudaEventRecord(c->hc_ev[par], caller));
-  static const bool overlap = getenv("FLECHE_HOST_OVERLAP") != nullptr;
-  if (!overlap) FL_CUDA(c, cudaStreamWaitEvent(s, c->hc_ev[par], 0));
+  static const bool ordered = getenv("FLECHE_HOST_ORDERED") != nullptr;
+  if (ordered) FL_CUDA(c, cudaStreamWaitEvent(s, c->hc_ev[par], 0));
   st = order_on(c, s);
   if (st != FLECHE_OK) return st;
   std::vector<const int64_t*> dids(c->n);

@@ -394,8 +394,8 @@ def test_host_buffer_calls_pipelined_back_to_back():
 
 
 def test_query_host_output_copy_orders_after_stream():
-    """fleche_query_host's output copy orders after `stream` (also with the experimental
-    FLECHE_HOST_OVERLAP, where the lookups do not): a read of `out` the caller enqueued on
+    """fleche_query_host's lookups do not wait for `stream` (call k+1's lookups overlap call
+    k's output copy), but its output copy does: a read of `out` the caller enqueued on
     `stream` between two calls into the same host buffer sees the first call's rows."""
     w = configs.get("cfg0").with_(cache_frac=0.05)
     tabs = _tables(w)

@@ -1,4 +1,4 @@
-# e2e A/B: fleche_query_host ordered (default) vs FLECHE_HOST_OVERLAP=1, alternating, same box
+# e2e A/B (round-1 builds): fleche_query_host ordered vs FLECHE_HOST_OVERLAP=1 (now the default; FLECHE_HOST_ORDERED=1 gives the old order), alternating, same box
 B="python bench.py --no-cpu-baseline"
 for r in 4 5 6 7 8; do
   timeout 300 $B > gpurun_out/eab_ordered_$r.json 2>/dev/null
