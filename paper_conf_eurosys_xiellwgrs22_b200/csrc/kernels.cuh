@@ -39,6 +39,9 @@
 #ifndef FL_KQ_PROBE
 #define FL_KQ_PROBE 32  // index lines per lane in flight in KQ's probe (a divisor of 32; A/B builds vary it)
 #endif
+#ifndef FL_KQ_TS_DEFER
+#define FL_KQ_TS_DEFER 0  // 1: KQ's timestamp exchange result is consumed late (A/B builds)
+#endif
 #ifndef FL_KQ_MIN_BLOCKS
 #define FL_KQ_MIN_BLOCKS 8  // KQ CTAs per SM the register budget must allow: 8 (64 regs, no spill) measured
                             // KQ 33.4 vs 35.5 us at 5 CTAs (profiles/bench_r01_kq_occupancy_*.json)
@@ -656,8 +659,17 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
     }
 
     // hit: refresh the way's timestamp once per batch (approximate LRU)
+#if FL_KQ_TS_DEFER
+    // issued predicated (no branch) and consumed only at the stats ballot, so its L2 round
+    // trip overlaps the miss lanes' dedup CAS instead of preceding it
+    const uint32_t need = (hit && old_ts != epoch) ? 1u : 0u;
+    uint32_t prev_ts = epoch;
+    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p atom.global.exch.b32 %0, [%1], %3;\n\t}"
+                 : "+r"(prev_ts) : "l"(dv.ts + slot), "r"(need), "r"(epoch) : "memory");
+#else
     bool uhit = false;
     if (hit && old_ts != epoch) uhit = atomicExch(dv.ts + slot, epoch) != epoch;
+#endif
 
     // A5 miss dedup: the lane whose CAS installs (epoch, fk) owns the miss
     int kind = 0;  // 1 = owner, 2 = duplicate
@@ -748,6 +760,9 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
     // reductions: no block barrier, so a finished warp retires without waiting for the
     // slowest warp of its CTA)
     const unsigned hm = __ballot_sync(kFull, hit), mm = __ballot_sync(kFull, miss);
+#if FL_KQ_TS_DEFER
+    const bool uhit = need && prev_ts != epoch;
+#endif
     const unsigned im = __ballot_sync(kFull, active && !valid), um = __ballot_sync(kFull, uhit);
     if (lane == 0) {
       unsigned long long* row = dv.stats + ((blockIdx.x * 4u + (threadIdx.x >> 5)) % kStripes) * kNumCtr;
