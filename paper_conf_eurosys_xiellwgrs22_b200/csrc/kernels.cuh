@@ -40,7 +40,7 @@
 #define FL_KQ_PROBE 32  // index lines per lane in flight in KQ's probe (a divisor of 32; A/B builds vary it)
 #endif
 #ifndef FL_KQ_TS_DEFER
-#define FL_KQ_TS_DEFER 0  // 1: KQ's timestamp exchange result is consumed late (A/B builds)
+#define FL_KQ_TS_DEFER 1  // KQ consumes its timestamp-exchange result late (0 = right after it; A/B builds)
 #endif
 #ifndef FL_KQ_MIN_BLOCKS
 #define FL_KQ_MIN_BLOCKS 8  // KQ CTAs per SM the register budget must allow: 8 (64 regs, no spill) measured
