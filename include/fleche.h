@@ -92,10 +92,8 @@ typedef struct {
   int32_t reserved;              /* must be 0                                                      */
 } fleche_config;
 
-/* Experimental: the query kernel starts each unique miss's host-row transfer into L2
- * (cp.async.bulk.prefetch.L2) so the miss kernel's loads hit L2.  Off by default: it
- * measured slower on B200 (profiles/README.md, round 1). */
-#define FLECHE_FLAG_L2_PREFETCH 0x1u
+/* Flag bit 0x1 is reserved (was an L2-prefetch experiment, measured slower and removed;
+ * profiles/README.md, round 1): fleche_create rejects it with FLECHE_EINVAL. */
 /* Baseline / ablation modes (the paper's comparison point):
  * STATIC_PER_TABLE: replace the flat cache by one static cache per table, each with
  *   floor(frac * c_t) rows where frac = cache_bytes / sum_t 4 c_t d_t ("the same

@@ -19,7 +19,6 @@ if not os.path.exists(LIB_PATH):
 _lib = ctypes.CDLL(LIB_PATH)
 
 OK, EINVAL, ENOMEM, ECUDA, ENCCL, ERANGE, ESTATE = 0, -1, -2, -3, -4, -5, -6
-FLAG_L2_PREFETCH = 0x1
 FLAG_STATIC_PER_TABLE, FLAG_PER_TABLE_LAUNCH, FLAG_HOST_ASSIST, FLAG_FUSED_HIT_COPY = 0x2, 0x4, 0x8, 0x10
 MAX_TABLES = 512
 

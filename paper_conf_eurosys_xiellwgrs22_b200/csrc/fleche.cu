@@ -86,9 +86,6 @@ struct fleche_ctx {
   cudaStream_t side = nullptr;
   cudaEvent_t fork_ev = nullptr, join_ev = nullptr;
   uint32_t* d_slots = nullptr;
-  bool early = false;            // early miss fetch: KF on the side stream, concurrent with KQ
-  size_t kf_smem = 0;
-  cudaEvent_t kf_ev = nullptr;
   int64_t decouple_min = 524288;  // lookups per batch from which the hit copy is decoupled (cfg2: equal, cfg5: +5 %)
   size_t km_smem = 0;
   // host-side counters
@@ -414,7 +411,7 @@ void free_all(fleche_ctx* c) {
                   c->dv.miss, c->dv.dup, c->dv.ctl, c->dv.stats, c->d_tables, c->d_ids_stage, c->d_out_stage,
                   c->d_pool_stage, c->d_kdec, c->rd.scratch, c->rd.slotval, c->rd.inv, c->rd.region, c->rd.cnt,
                   c->rd.prefix, c->rd.done, c->rd.stats, c->d_slots, c->d_age_hist, c->d_prefill_out,
-                  c->dv.mready, c->d_out_stage2};
+                  c->d_out_stage2};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   for (auto& r : c->registered) cudaHostUnregister(r.first);
@@ -422,7 +419,6 @@ void free_all(fleche_ctx* c) {
   if (c->chain_ev) cudaEventDestroy(c->chain_ev);
   if (c->fork_ev) cudaEventDestroy(c->fork_ev);
   if (c->join_ev) cudaEventDestroy(c->join_ev);
-  if (c->kf_ev) cudaEventDestroy(c->kf_ev);
   for (int i = 0; i < 2; ++i) {
     if (c->hq_ev[i]) cudaEventDestroy(c->hq_ev[i]);
     if (c->hd_ev[i]) cudaEventDestroy(c->hd_ev[i]);
@@ -538,19 +534,8 @@ fleche_status launch_query(fleche_ctx* c, const int64_t* const* ids, const int64
   fleche_status st = prof_event(c, s, true, nev);
   if (st != FLECHE_OK) return st;
   // small batches: the fork/join costs more than the overlap saves (cfg1 measured +5 %)
-  const bool early = c->early && total > 0 && !c->per_table_launch;
-  const bool decouple = !early && c->decoupled && total >= c->decouple_min && !c->per_table_launch;
+  const bool decouple = c->decoupled && total >= c->decouple_min && !c->per_table_launch;
   if (decouple) qa.slots = c->d_slots;
-  if (early) {  // fork: KF waits on the side stream for the miss records KQ publishes
-    qa.early = 1;
-    ka.early = 1;
-    FL_CUDA(c, cudaEventRecord(c->fork_ev, s));
-    FL_CUDA(c, cudaStreamWaitEvent(c->side, c->fork_ev, 0));
-    KFArgs fa{out, (uint32_t)((total + 127) / 128), c->max_dim};
-    launch_k(kPdlNone, kf_fn(c->max_dim), (unsigned)c->sm_count, kKfWarps * 32, c->kf_smem, c->side, c->dv, fa);
-    c->kernels++;
-    FL_CUDA(c, cudaEventRecord(c->kf_ev, c->side));
-  }
   if (total > 0 && !c->per_table_launch) {
     const int64_t blocks = (total + 127) / 128;
     launch_k(kPdlKQ, kq_fn<MAXT>(), (unsigned)blocks, 128, 0, s, qa, c->dv);
@@ -581,7 +566,6 @@ fleche_status launch_query(fleche_ctx* c, const int64_t* const* ids, const int64
     }
   }
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
-  if (early) FL_CUDA(c, cudaStreamWaitEvent(s, c->kf_ev, 0));  // join: every missed row is in `out`
   launch_k(kPdlKM, km_fn(c->dv.bytes != 0, c->cls_dim.size() == 1 ? c->max_dim : 0), c->km_blocks, 128, c->km_smem, s, c->dv, ka);
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
   launch_k(kPdlKD, kd_fn(), c->kd_blocks, 128, 0, s, c->dv, out);
@@ -670,7 +654,7 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   *out = nullptr;
   const int n = cfg->num_tables;
   if (n < 1 || n > FLECHE_MAX_TABLES || !cfg->cardinalities || !cfg->dims || !cfg->host_tables) return FLECHE_EINVAL;
-  const uint32_t known = FLECHE_FLAG_L2_PREFETCH | FLECHE_FLAG_STATIC_PER_TABLE | FLECHE_FLAG_PER_TABLE_LAUNCH |
+  const uint32_t known = FLECHE_FLAG_STATIC_PER_TABLE | FLECHE_FLAG_PER_TABLE_LAUNCH |
                          FLECHE_FLAG_HOST_ASSIST | FLECHE_FLAG_FUSED_HIT_COPY;
   if (cfg->max_lookups < 1 || cfg->max_lookups > (int64_t(1) << 31) || (cfg->flags & ~known) || cfg->reserved)
     return FLECHE_EINVAL;
@@ -775,8 +759,6 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   dv.admit_all = (p <= 0.0 || p >= 1.0) ? 1 : 0;
   dv.admit_thr = dv.admit_all ? ~0ull : (uint64_t)ldexp(p, 64);
   dv.admit_seed = cfg->admit_seed;
-  dv.prefetch = (cfg->flags & FLECHE_FLAG_L2_PREFETCH) ? 1 : 0;
-  if (const char* e = getenv("FLECHE_PREFETCH_MODE")) dv.prefetch = atoi(e);  // A/B: 2 = prefetch.global.L2 per line
   if (const char* e = getenv("FLECHE_KM_BLOCKS_PER_SM")) c->km_bps = std::max(1, atoi(e));
 #ifdef FLECHE_EXPERIMENTS
   if (const char* e = getenv("FLECHE_EXP_MODE")) dv.exp_mode = atoi(e);
@@ -866,38 +848,6 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
         cudaEventCreateWithFlags(&c->fork_ev, cudaEventDisableTiming) != cudaSuccess ||
         cudaEventCreateWithFlags(&c->join_ev, cudaEventDisableTiming) != cudaSuccess ||
         cudaMalloc((void**)&c->d_slots, (size_t)cfg->max_lookups * 4) != cudaSuccess)
-      return fail(FLECHE_ENOMEM);
-  }
-  // early miss fetch (KF concurrent with KQ): uniform single-width layout, row <= 512 B,
-  // not with the host-assisted fetch or per-table launches.  FLECHE_EARLY_FETCH=0/1 (A/B)
-  {
-    const char* e = getenv("FLECHE_EARLY_FETCH");
-    const bool want = e ? atoi(e) != 0 : false;
-    c->early = want && !bytes && !part && c->cls_dim.size() == 1 && c->max_dim <= 128 &&
-               !(cfg->flags & FLECHE_FLAG_HOST_ASSIST) && !c->per_table_launch;
-  }
-  if (c->early) {
-    // KF spins on KQ's progress, so KQ must never wait for KF: load every kernel of the
-    // batch now.  Under lazy module loading (the CUDA 12 default) a kernel's first launch
-    // loads its module, which waits for the running kernels -- KF -- to finish: deadlock.
-    cudaFuncAttributes fa_;
-    if (cudaFuncGetAttributes(&fa_, (const void*)kq_fn<32>()) != cudaSuccess ||
-        cudaFuncGetAttributes(&fa_, (const void*)kq_fn<128>()) != cudaSuccess ||
-        cudaFuncGetAttributes(&fa_, (const void*)kq_fn<FLECHE_MAX_TABLES>()) != cudaSuccess ||
-        cudaFuncGetAttributes(&fa_, (const void*)km_fn(false, c->max_dim)) != cudaSuccess ||
-        cudaFuncGetAttributes(&fa_, (const void*)kd_fn()) != cudaSuccess ||
-        cudaFuncGetAttributes(&fa_, (const void*)ke_hist_fn()) != cudaSuccess ||
-        cudaFuncGetAttributes(&fa_, (const void*)ke_evict_fn()) != cudaSuccess)
-      return fail(FLECHE_ECUDA);
-    const int rounds = std::min(4, 128 / c->max_dim);
-    c->kf_smem = (size_t)kKfWarps * rounds * 32 * (size_t)c->max_dim * 4;
-    if ((!c->side && cudaStreamCreateWithFlags(&c->side, cudaStreamNonBlocking) != cudaSuccess) ||
-        (!c->fork_ev && cudaEventCreateWithFlags(&c->fork_ev, cudaEventDisableTiming) != cudaSuccess) ||
-        cudaEventCreateWithFlags(&c->kf_ev, cudaEventDisableTiming) != cudaSuccess ||
-        cudaMalloc((void**)&dv.mready, (size_t)cfg->max_lookups * 4) != cudaSuccess ||
-        cudaMemset(dv.mready, 0, (size_t)cfg->max_lookups * 4) != cudaSuccess ||
-        cudaFuncSetAttribute((const void*)kf_fn(c->max_dim), cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             (int)c->kf_smem) != cudaSuccess)
       return fail(FLECHE_ENOMEM);
   }
   if (cfg->flags & FLECHE_FLAG_HOST_ASSIST) {

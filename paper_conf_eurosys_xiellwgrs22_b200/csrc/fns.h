@@ -21,14 +21,12 @@ using KdFn = void (*)(Dev, float*);
 using ProbeFn = void (*)(const float*, uint64_t, int64_t, uint64_t, float*);
 using KpkFn = void (*)(RouteDev, uint32_t*, int64_t*, PeerKeys);
 using KeFn = void (*)(Dev, KEArgs);
-using KfFn = void (*)(Dev, KFArgs);
 
 template <int MAXT> KqFn<MAXT> kq_fn();   // fused query (k_query.cu)
 template <int MAXT> KqFn<MAXT> kg_fn();   // decoupled hit copy (k_query.cu)
 template <int MAXT> KpFn<MAXT> kp_fn();   // pooling (k_query.cu)
 KmFn km_fn(bool bytes, int dim);          // miss kernel: bytes layout / uniform width dim / 0 = per class (k_miss.cu)
 KdFn kd_fn();                             // duplicate restore (k_misc.cu)
-KfFn kf_fn(int dim);                      // early miss fetch, concurrent with KQ (k_misc.cu)
 KeFn ke_hist_fn();                        // watermark scan: age histogram (k_misc.cu)
 KeFn ke_evict_fn();                       // watermark scan: threshold + evict (k_misc.cu)
 ProbeFn probe_fn(int dim);                // host-link probe (k_misc.cu)

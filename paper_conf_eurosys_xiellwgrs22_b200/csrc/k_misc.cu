@@ -6,16 +6,6 @@
 namespace fl {
 
 KdFn kd_fn() { return kd_kernel<0>; }
-KfFn kf_fn(int dim) {
-  switch (dim) {
-    case 8: return kf_kernel<8>;
-    case 16: return kf_kernel<16>;
-    case 32: return kf_kernel<32>;
-    case 64: return kf_kernel<64>;
-    case 128: return kf_kernel<128>;
-    default: return nullptr;
-  }
-}
 KeFn ke_hist_fn() { return ke_hist_kernel<0>; }
 KeFn ke_evict_fn() { return ke_evict_kernel<0>; }
 

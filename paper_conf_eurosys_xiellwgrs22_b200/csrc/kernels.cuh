@@ -127,7 +127,6 @@ struct Ctl {
   long long occ_bytes;    // row bytes currently cached
   uint32_t ke_done;       // watermark eviction: KE2 CTA arrival counter
   uint32_t ke_pad;
-  uint32_t kq_cnt[2];     // early fetch: [epoch & 1] KQ CTAs finished (KF stops at the last one)
 };
 
 // Host-assisted miss fetch (FLECHE_FLAG_HOST_ASSIST).  The owner lane of each unique
@@ -165,15 +164,12 @@ struct Dev {
   unsigned long long* ipos;      // uniform layout: [sets][32] (epoch << 32 | inserter's first occurrence << 1 | busy)
   MissRec* miss;                 // [max_lookups], split into per-class regions per call
   DupRec* dup;                   // [max_lookups]
-  uint32_t* mready;              // early fetch: [max_lookups] epoch once miss record i is written
   Ctl* ctl;
   unsigned long long* stats;  // [kStripes][kNumCtr]
   const TableInfo* tables;    // [n]
   uint32_t sets, rows, scr_mask, hash_seed;
   int32_t dim, admit_all;     // dim: row width of the uniform layout
   uint64_t admit_thr, admit_seed;
-  int32_t prefetch;  // KQ starts each unique miss's host-row transfer into L2
-  int32_t km_pad;
   int32_t bytes;     // 0 = uniform layout, 1 = bytes layout
   uint32_t set_units;  // bytes layout: region of a set in 32 B units (<= 256)
   int32_t part;      // static per-table partitions (HugeCTR-like baseline, NEXT-1)
@@ -221,7 +217,6 @@ struct QArgs {
   uint32_t* slots;           // decoupled copy: per-lookup hit slot / kSlotMiss / kSlotZero for KG
   int32_t n;
   int32_t t0;                // first table of this launch (per-table launches: t0 = t, n = 1)
-  int32_t early;             // early fetch: publish each miss record for KF, count finished CTAs
   int32_t fkseg;             // key-sharded fused exchange: fkeys come in n segments (ids[], scan[])
 };
 
@@ -230,7 +225,6 @@ struct KMArgs {
   int64_t cls_off[8];
   int32_t cls_dim[8];
   int32_t ncls;
-  int32_t early;  // early fetch: KF already put every missed row in `out`; KM reads it from HBM
 };
 
 template <int MAXT>
@@ -727,24 +721,12 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
         if (dv.ha && !dv.bytes && (uint64_t)(li + 1) * (uint64_t)d <= dv.ha_stage_floats) hst = (uint64_t)li * d;
         dv.miss[li] = MissRec{off, fk, scr, qa.t0 + t, 0, hst};
         dv.owner_off[scr] = off;
-        if (qa.early) {  // early fetch: KF (running concurrently) may take the record now
-          __threadfence();
-          *(volatile uint32_t*)(dv.mready + li) = epoch;
-        }
 #ifdef FLECHE_EXPERIMENTS
         if (dv.exp_mode != 4)
 #endif
         if (dv.ha)  // published by KM's doorbell (after this grid completes)
           dv.ha_req[(size_t)par * dv.ha_req_cap + li] =
               HaReq{((unsigned long long)(qa.t0 + t) << 48) | (unsigned long long)id, hst};
-        if (dv.prefetch == 1) {  // experimental: start the host-link transfer now
-          const float* hrow = ti->host + (size_t)id * (size_t)d;
-          asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(hrow), "r"(4u * (unsigned)d) : "memory");
-        } else if (dv.prefetch >= 2) {  // experimental: per-line L2 prefetch (warms the address translation)
-          const char* hrow = (const char*)(ti->host + (size_t)id * (size_t)d);
-          const int lines = dv.prefetch == 2 ? 1 : (4 * d + 127) / 128;
-          for (int q = 0; q < lines; ++q) asm volatile("prefetch.global.L2 [%0];" ::"l"(hrow + 128 * q) : "memory");
-        }
       }
     }
     if (dup_m) {
@@ -778,13 +760,6 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
     }
   }
   pdl_trigger();  // KM may be scheduled now; its pdl_wait still waits for this grid
-  if (qa.early) {  // every record of this CTA is published: count it for KF
-    __syncthreads();
-    if (threadIdx.x == 0) {
-      __threadfence();
-      atomicAdd(&dv.ctl->kq_cnt[*(volatile uint32_t*)&dv.ctl->epoch & 1u], 1u);
-    }
-  }
 }
 
 // KG decoupled hit copy (Fig 8b): KQ only indexes (slot per lookup); KG copies
@@ -1135,7 +1110,7 @@ template <bool BYTES, int D, int M>
 __device__ __forceinline__ void km_rows(const Dev& dv, float* __restrict__ out, const MissRec* __restrict__ mlist,
                                         uint32_t epoch, uint32_t nmiss, int lane, uint32_t gw, uint32_t nw,
                                         unsigned& ins, unsigned& ev, unsigned& byp, long long& docc,
-                                        unsigned long long& hostb, float4* wsm, bool early) {
+                                        unsigned long long& hostb, float4* wsm) {
 #ifdef FLECHE_EXPERIMENTS
   if (dv.exp_buf && lane == 0) {
     unsigned long long t;
@@ -1150,8 +1125,7 @@ __device__ __forceinline__ void km_rows(const Dev& dv, float* __restrict__ out, 
     const float* src = nullptr;
     if (has) {
       const TableInfo* ti = dv.tables + m.t;
-      src = early ? out + m.off                                 // KF fetched it during KQ
-                  : ti->host + (size_t)(m.fk - ti->base) * D;  // unified index: computed host address
+      src = ti->host + (size_t)(m.fk - ti->base) * D;  // unified index: computed host address
     }
 #ifdef FLECHE_EXPERIMENTS
     if (dv.exp_mode == 2) src = nullptr;  // timing experiment: no host loads
@@ -1164,7 +1138,7 @@ __device__ __forceinline__ void km_rows(const Dev& dv, float* __restrict__ out, 
     if (has) {
       admit = dv.admit_all ||
               splitmix64(dv.admit_seed ^ (uint64_t)m.fk ^ ((uint64_t)(epoch - 1u) << 32)) < dv.admit_thr;
-      if (!early) hostb += 4ull * D;
+      hostb += 4ull * D;
     }
     if constexpr (!BYTES) {
       // A7 while the loads are in flight: victim claim (L2 round trips only); the first
@@ -1203,7 +1177,7 @@ __device__ __forceinline__ void km_rows(const Dev& dv, float* __restrict__ out, 
         }
         if (slot == kClaimRetry && pending) __nanosleep(100);
       }
-      if (!early) rb.store(has ? out + m.off : nullptr, lane);  // the owner's output row
+      rb.store(has ? out + m.off : nullptr, lane);  // the owner's output row
 #ifdef FLECHE_EXPERIMENTS
       if (dv.exp_buf && lane == 0 && first_chunk) {
         unsigned long long t;
@@ -1354,8 +1328,7 @@ __global__ void __launch_bounds__(128, 4) km_kernel(const __grid_constant__ Dev 
   if (use_ha)                                                                                                 \
     km_ha<BYTES, D>(dv, ka.out, ml, epoch, nmiss, lane, gw, nw, ins, ev, byp, docc, hostb, hsm, wsm, harows, hato, kcut); \
   else                                                                                                        \
-    km_rows<BYTES, D, KmM<BYTES, D>::value>(dv, ka.out, ml, epoch, nmiss, lane, gw, nw, ins, ev, byp, docc, hostb, wsm, \
-                                            !BYTES && ka.early)
+    km_rows<BYTES, D, KmM<BYTES, D>::value>(dv, ka.out, ml, epoch, nmiss, lane, gw, nw, ins, ev, byp, docc, hostb, wsm)
     if constexpr (DU > 0) {
       FL_KM(DU);
     } else {
@@ -1401,99 +1374,11 @@ __global__ void __launch_bounds__(128, 4) km_kernel(const __grid_constant__ Dev 
 #pragma unroll
       for (int c = 0; c < 8; ++c) dv.ctl->counts[par ^ 1][c] = 0;
       dv.ctl->ha_f[par ^ 1] = 0;
-      dv.ctl->kq_cnt[par ^ 1] = 0;
       dv.ctl->done = 0;
       __threadfence();
       *(volatile uint32_t*)&dv.ctl->epoch = epoch + 1u;
     }
   }
-}
-
-// KF early miss fetch (uniform layout): runs on a side stream CONCURRENTLY with KQ and
-// starts each unique miss's host-row read as soon as KQ publishes its miss record, so
-// the host-link latency of the batch's misses (a ~60-90 us burst on this platform,
-// profiles/km_timeline_cfg2_r01c.txt) overlaps the index probe instead of following it.
-// Only the fetch moves: the inserts still follow every probe of the batch (reading R9)
-// in KM, which then reads the rows from `out` in HBM.  Lane = one miss record; its row
-// goes host -> shared memory with cp.async (no registers held while in flight), then to
-// the owner's `out` row.  One CTA per SM and <= 32 registers (launch bounds) leave room for
-// five KQ CTAs per SM next to it.
-constexpr int kKfWarps = 4;
-// rounds of 32 rows per warp in flight: 64 KB of staging per CTA (D <= 128)
-template <int D> struct KfRounds { static constexpr int value = (128 / D) < 4 ? (128 / D) : 4; };
-
-struct KFArgs {
-  float* out;
-  uint32_t kq_blocks;  // KQ grid size: KQ is complete once kq_cnt reaches it
-  int32_t dim;
-};
-
-__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
-  const unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(sa), "l"(gmem) : "memory");
-}
-
-template <int D>
-__global__ void __launch_bounds__(kKfWarps * 32, 16) kf_kernel(const __grid_constant__ Dev dv,
-                                                              const __grid_constant__ KFArgs fa) {
-  extern __shared__ float4 kf_sm[];  // [warps][rounds][32 rows][D/4]
-  constexpr int VEC = D / 4;
-  constexpr int kKfRounds = KfRounds<D>::value;
-  const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
-  const uint32_t epoch = *(volatile uint32_t*)&dv.ctl->epoch;
-  const int par = epoch & 1u;
-  const uint32_t gw = wib * gridDim.x + blockIdx.x;  // block-interleaved: spread over SMs
-  const uint32_t nw = gridDim.x * kKfWarps;
-  unsigned long long hostb = 0;
-  float4* wsm = kf_sm + (size_t)wib * kKfRounds * 32 * VEC;
-  bool done = false;
-  for (uint32_t base = gw * 32; !done; ) {
-    int64_t off[kKfRounds];
-    int nr = 0;
-#pragma unroll
-    for (int r = 0; r < kKfRounds; ++r) {
-      off[r] = -1;
-      if (done) continue;
-      const uint32_t i = base + lane;
-      bool mine = false;
-      while (true) {  // wait until record i is published, or KQ is complete and i is past the end
-        if (ld_cv_u32(dv.mready + i) == epoch) { mine = true; break; }
-        if (*(volatile uint32_t*)&dv.ctl->kq_cnt[par] >= fa.kq_blocks) {
-          __threadfence();
-          mine = i < *(volatile uint32_t*)&dv.ctl->counts[par][0];
-          break;
-        }
-        __nanosleep(256);
-      }
-      if (mine) {
-        __threadfence();
-        const MissRec m = dv.miss[i];
-        const TableInfo* ti = dv.tables + m.t;
-        const float* src = ti->host + (size_t)(m.fk - ti->base) * D;
-        float4* dst = wsm + ((size_t)r * 32 + lane) * VEC;
-#pragma unroll
-        for (int c = 0; c < VEC; ++c) cp_async16(dst + c, src + 4 * c);
-        off[r] = m.off;
-        hostb += 4ull * D;
-      }
-      asm volatile("cp.async.commit_group;" ::: "memory");
-      ++nr;
-      if (!__any_sync(kFull, mine)) done = true;  // records are dense: nothing beyond this round
-      base += nw * 32;
-    }
-    asm volatile("cp.async.wait_all;" ::: "memory");
-#pragma unroll
-    for (int r = 0; r < kKfRounds; ++r) {
-      if (off[r] < 0) continue;
-      const float4* srow = wsm + ((size_t)r * 32 + lane) * VEC;
-#pragma unroll 4
-      for (int c = 0; c < VEC; ++c) st_v4(fa.out + off[r] + 4 * c, srow[c]);
-    }
-    (void)nr;
-  }
-#pragma unroll
-  for (int o = 16; o; o >>= 1) hostb += __shfl_xor_sync(kFull, hostb, o);
-  if (lane == 0 && hostb) atomicAdd(dv.stats + (blockIdx.x % kStripes) * kNumCtr + C_HOSTBYTES, hostb);
 }
 
 // KD restore: every duplicate occurrence of a missed key copies its owner's

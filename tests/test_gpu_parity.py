@@ -159,11 +159,8 @@ def test_host_buffer_entry_point_matches_device_path():
         assert H.bits_equal(out, orc.query(bt.ids))
 
 
-@pytest.mark.parametrize("early", ["0", "1"])
-def test_cuda_graph_replay_advances_epoch(monkeypatch, early):
+def test_cuda_graph_replay_advances_epoch():
     # the epoch lives on the device, so a captured query replays with fresh semantics
-    # (early=1: the KF fork/join on the side stream is captured too)
-    monkeypatch.setenv("FLECHE_EARLY_FETCH", early)
     w = configs.get("cfg0")
     tabs = _tables(w)
     gpu, orc = H.make_pair(w, tabs)
@@ -323,43 +320,6 @@ def test_short_keys_parity(B):
     with pytest.raises(fl.binding.FlecheError):  # the key-sharded mode needs exact codes
         gpu.route([torch.zeros(1, dtype=torch.int64, device="cuda")] * w.n, 2, 1,
                   torch.empty(8, dtype=torch.int32, device="cuda"), torch.empty(2, dtype=torch.int64, device="cuda"))
-
-
-@pytest.mark.parametrize("case", ["cfg0", "churn", "p03"])
-def test_early_fetch_exact(monkeypatch, case):
-    """FLECHE_EARLY_FETCH: KF fetches the missed rows concurrently with KQ; KM inserts from
-    `out`.  Values and every counter stay exactly the set oracle's."""
-    monkeypatch.setenv("FLECHE_EARLY_FETCH", "1")
-    kw = {}
-    if case == "cfg0":
-        w = configs.get("cfg0").with_(cache_frac=0.25, invalid_ppm=2000)
-    elif case == "churn":
-        w = configs.get("cfg0").with_(cache_frac=0.01, invalid_ppm=3000, skews=[0.6] * 7, batch_size=400)
-    else:
-        w = configs.get("cfg0").with_(cache_frac=0.25)
-        kw = dict(admit_p=0.3, admit_seed=gen.seeds()["admit"])
-    gpu, orc = _run(w, _tables(w), 30, **kw)
-    st = gpu.stats()
-    assert st["kernels_launched"] == 4 * 30  # KF + KQ + KM + KD
-    assert st["host_bytes_fetched"] == st["unique_misses"] * 4 * w.dims[0]
-
-
-def test_early_fetch_cfg2_full_size(monkeypatch):
-    monkeypatch.setenv("FLECHE_EARLY_FETCH", "1")
-    w = configs.get("cfg2")
-    tabs = _tables(w)
-    gpu, seta = H.make_pair(w, tabs, O.MODE_SETASSOC)
-    for b in range(40):
-        bt = w.batch(b)
-        g0, o0 = gpu.stats(), seta.stats()
-        got = H.run_batch_gpu(gpu, bt.ids, torch)
-        ref = seta.query(bt.ids)
-        assert H.bits_equal(got, ref), b
-        dg, do = H.delta(g0, gpu.stats()), H.delta(o0, seta.stats())
-        if do["bypassed"] == 0:
-            for k in H.STAT_KEYS_EXACT:
-                assert dg[k] == do[k], (b, k)
-
 
 
 def test_host_buffer_calls_pipelined_back_to_back():
