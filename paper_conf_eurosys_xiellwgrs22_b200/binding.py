@@ -166,6 +166,43 @@ def _stream_handle(stream) -> int:
     return int(stream.cuda_stream)
 
 
+def _check_ids(ids, n: int, device, what: str):
+    """int64, contiguous, on `device` (None: host memory) -- for tensors and numpy arrays;
+    raw pointers (ints) are passed through unchecked."""
+    if len(ids) != n:
+        raise ValueError(f"{what}: {len(ids)} ID arrays for {n} tables")
+    for t, x in enumerate(ids):
+        if isinstance(x, int) or x is None:
+            continue
+        if isinstance(x, np.ndarray):
+            if device is not None:
+                raise ValueError(f"{what}: table {t} IDs are a host array, a device tensor is needed")
+            if x.dtype != np.int64 or not x.flags.c_contiguous:
+                raise ValueError(f"{what}: table {t} IDs must be contiguous int64")
+            continue
+        if str(x.dtype) != "torch.int64" or not x.is_contiguous():
+            raise ValueError(f"{what}: table {t} IDs must be contiguous int64 (got {x.dtype})")
+        dev = x.device.index if x.is_cuda else None
+        if (device is None) != (not x.is_cuda) or (device is not None and dev != device):
+            raise ValueError(f"{what}: table {t} IDs on {x.device}, expected "
+                             f"{'host memory' if device is None else f'cuda:{device}'}")
+
+
+def _check_out(out, floats: int, device, what: str):
+    """fp32, contiguous, >= floats elements, on `device` (None: host memory)."""
+    if isinstance(out, int) or out is None:
+        return
+    if isinstance(out, np.ndarray):
+        ok = device is None and out.dtype == np.float32 and out.flags.c_contiguous and out.size >= floats
+    else:
+        ok = (str(out.dtype) == "torch.float32" and out.is_contiguous() and out.numel() >= floats and
+              (out.device.index == device if device is not None else not out.is_cuda) and
+              (device is None or out.is_cuda))
+    if not ok:
+        raise ValueError(f"{what}: out must be a contiguous float32 buffer of >= {floats} elements in "
+                         f"{'host memory' if device is None else f'cuda:{device}'}")
+
+
 class FlatCache:
     """One flat GPU cache over the given host tables (fleche_create / fleche_query / fleche_stats)."""
 
@@ -207,14 +244,30 @@ class FlatCache:
 
     def query(self, ids, out, stream=None, lengths=None):
         """ids: list of n device int64 tensors (or pointers with `lengths`); out: device fp32 buffer."""
+        _check_ids(ids, self.n, self.device, "query")
         if lengths is None:
             lengths = [int(x.numel()) for x in ids]
+        _check_out(out, self.out_floats(lengths), self.device, "query")
         lp = (_i64 * self.n)(*lengths)
         ip = (_vp * self.n)(*[_ptr(x) for x in ids])
         _check(fleche_query(self.h, ip, lp, _ptr(out), _stream_handle(stream)), "fleche_query")
 
+    def prepare(self, ids, lengths=None):
+        """Validate and marshal a batch's ID arrays once (the caller keeps them alive and
+        unchanged); `query_prepared` then only checks `out`."""
+        _check_ids(ids, self.n, self.device, "prepare")
+        if lengths is None:
+            lengths = [int(x.numel()) for x in ids]
+        return ((_vp * self.n)(*[_ptr(x) for x in ids]), (_i64 * self.n)(*lengths), self.out_floats(lengths))
+
+    def query_prepared(self, prep, out, stream=None):
+        ip, lp, floats = prep
+        _check_out(out, floats, self.device, "query")
+        _check(fleche_query(self.h, ip, lp, _ptr(out), _stream_handle(stream)), "fleche_query")
+
     def prefill(self, ids, stream=None, lengths=None):
         """Warm start: one batch of lookups through the cache, rows discarded."""
+        _check_ids(ids, self.n, self.device, "prefill")
         if lengths is None:
             lengths = [int(x.numel()) for x in ids]
         lp = (_i64 * self.n)(*lengths)
@@ -226,10 +279,13 @@ class FlatCache:
 
     def query_pooled(self, ids, offsets, out, stream=None, bags=None, nnz=None):
         """ids/offsets: lists of n device int64 tensors (CSR per table); out: device fp32 buffer."""
+        _check_ids(ids, self.n, self.device, "query_pooled")
+        _check_ids(offsets, self.n, self.device, "query_pooled offsets")
         if bags is None:
             bags = [int(o.numel()) - 1 for o in offsets]
         if nnz is None:
             nnz = [int(x.numel()) for x in ids]
+        _check_out(out, self.pooled_floats(bags), self.device, "query_pooled")
         bp = (_i64 * self.n)(*bags)
         npp = (_i64 * self.n)(*nnz)
         ip = (_vp * self.n)(*[_ptr(x) for x in ids])
@@ -290,8 +346,10 @@ class FlatCache:
 
     def query_host(self, ids, out, stream=None, lengths=None):
         """ids: list of n host int64 arrays (ideally pinned); out: host fp32 buffer."""
+        _check_ids(ids, self.n, None, "query_host")
         if lengths is None:
             lengths = [int(x.size if isinstance(x, np.ndarray) else x.numel()) for x in ids]
+        _check_out(out, self.out_floats(lengths), None, "query_host")
         lp = (_i64 * self.n)(*lengths)
         ip = (_vp * self.n)(*[_ptr(x) for x in ids])
         _check(fleche_query_host(self.h, ip, lp, _ptr(out), _stream_handle(stream)), "fleche_query_host")

@@ -44,6 +44,7 @@ struct HostAssist {
   float* stage = nullptr;              // [2][stage_floats]
   uint32_t req_cap = 0, blk_cap = 0;
   bool nt_stores = true;  // FLECHE_HA_NT=0: plain memcpy into the staging buffer (A/B)
+  uint64_t delay_ns = 0;  // FLECHE_HA_DELAY_US: fault injection (tests): each block is gathered this late
   uint64_t stage_floats = 0;
   // the tables as the host threads see them
   std::vector<const float*> host;
@@ -79,9 +80,8 @@ struct fleche_ctx {
   TableInfo* d_tables = nullptr;
   int km_blocks = 0;
   int km_bps = 4;  // KM CTAs per SM
-  int kd_blocks = 0;
   bool per_table_launch = false;
-  // decoupled hit copy (uniform layout): KG on a side stream, forked after KQ, joined after KD
+  // decoupled hit copy (uniform layout): KG on a side stream, forked after KQ, joined after KM
   bool decoupled = false;
   cudaStream_t side = nullptr;
   cudaEvent_t fork_ev = nullptr, join_ev = nullptr;
@@ -353,6 +353,10 @@ void ha_worker(HostAssist* h, int me) {
     const uint64_t kb0 = lo_all / kHaBlock, kb1 = (hi_all - 1) / kHaBlock;
     for (uint64_t kb = kb0; kb <= kb1 && kb < kcut; ++kb) {
       if (kb % (uint64_t)h->nthreads != (uint64_t)me) continue;
+      if (h->delay_ns) {  // a stalled host thread (tests): its blocks time out on the GPU
+        struct timespec ts = {(time_t)(h->delay_ns / 1000000000ull), (long)(h->delay_ns % 1000000000ull)};
+        nanosleep(&ts, nullptr);
+      }
       bool any = false;
       for (int c = 0; c < 8; ++c) {  // the rows of every class region that overlaps block kb
         if (!d.cnt[c]) continue;
@@ -467,10 +471,10 @@ fleche_status prof_event(fleche_ctx* c, cudaStream_t s, bool first, int kinds) {
 
 // Launch with programmatic stream serialization (PDL): the kernel's launch and prologue
 // overlap its predecessor's tail; the kernel's pdl_wait() orders its dependent work.
-// Per-kernel PDL mask (bit 0 KQ, 1 KM, 2 KD, 3 KP).  KM is launched without it by default:
-// its blocks would be placed early, during KQ's tail, which measured slower for the
-// address-ordered miss fetch (profiles/README.md).
-enum { kPdlKQ = 0, kPdlKM = 1, kPdlKD = 2, kPdlKP = 3, kPdlNone = 30 };
+// Per-kernel PDL mask (bit 0 KQ, 2 the watermark scan, 3 KP).  KM is a cooperative launch
+// (never PDL): its grid barrier needs every CTA resident, and its early placement during
+// KQ's tail measured slower for the address-ordered miss fetch anyway (profiles/README.md).
+enum { kPdlKQ = 0, kPdlKM = 1, kPdlKD = 2, kPdlKP = 3, kPdlNone = 30, kPdlCoop = 31 };
 int pdl_mask() {
   static const int m = getenv("FLECHE_NO_PDL") ? 0 : (getenv("FLECHE_PDL_MASK") ? atoi(getenv("FLECHE_PDL_MASK")) : 0xD);
   return m;
@@ -478,21 +482,34 @@ int pdl_mask() {
 template <typename... KArgs, typename... Args>
 cudaError_t launch_k(int which, void (*kern)(KArgs...), unsigned grid, unsigned block, size_t smem, cudaStream_t s,
                      Args&&... args) {
-  const bool g_pdl = (pdl_mask() >> which) & 1;
+  const bool g_pdl = which != kPdlCoop && ((pdl_mask() >> which) & 1);
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(grid);
   cfg.blockDim = dim3(block);
   cfg.dynamicSmemBytes = smem;
   cfg.stream = s;
   cudaLaunchAttribute attr[1];
-  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  if (which == kPdlCoop) {  // every CTA resident at once (KM2's grid barrier)
+    attr[0].id = cudaLaunchAttributeCooperative;
+    attr[0].val.cooperative = 1;
+  } else {
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+  }
   cfg.attrs = attr;
-  cfg.numAttrs = g_pdl ? 1 : 0;
+  cfg.numAttrs = (g_pdl || which == kPdlCoop) ? 1 : 0;
   return cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
 }
 
-// Watermark scan after a batch's KD (fleche_set_watermarks): KE1 + KE2, both exit at
+// The miss side of one batch: KM (fetch + insert + restore), a cooperative launch (its grid
+// barrier before the restore needs every CTA resident; km_blocks never exceeds that).
+void launch_miss(fleche_ctx* c, cudaStream_t s, const KMArgs& ka) {
+  launch_k(kPdlCoop, km_fn(c->dv.bytes != 0, c->cls_dim.size() == 1 ? c->max_dim : 0), c->km_blocks, 128, c->km_smem, s,
+           c->dv, ka);
+  c->kernels += 1;
+}
+
+// Watermark scan after a batch's KM (fleche_set_watermarks): KE1 + KE2, both exit at
 // once when the cached bytes are <= hi.
 void launch_scan(fleche_ctx* c, cudaStream_t s) {
   if (!c->wm_on) return;
@@ -566,10 +583,8 @@ fleche_status launch_query(fleche_ctx* c, const int64_t* const* ids, const int64
     }
   }
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
-  launch_k(kPdlKM, km_fn(c->dv.bytes != 0, c->cls_dim.size() == 1 ? c->max_dim : 0), c->km_blocks, 128, c->km_smem, s, c->dv, ka);
-  if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
-  launch_k(kPdlKD, kd_fn(), c->kd_blocks, 128, 0, s, c->dv, out);
-  c->kernels += 2;
+  launch_miss(c, s, ka);
+  if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;  // (the former KD's slot: empty)
   if (decouple) FL_CUDA(c, cudaStreamWaitEvent(s, c->join_ev, 0));  // join: out complete on s
   launch_scan(c, s);
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
@@ -825,20 +840,26 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
     if (const char* e = getenv("FLECHE_ORDER_MIN_SPAN")) min_span = strtoull(e, nullptr, 10);
     dv.ordered = (!bytes && !part && span > (uint64_t)scr_n && span >= min_span && getenv("FLECHE_NO_ORDER") == nullptr)
                      ? 1 : 0;
+    dv.bands = getenv("FLECHE_KM_BANDS") ? atoi(getenv("FLECHE_KM_BANDS")) : 2;  // 1-2 measured best at cfg2, 8 at cfg5 (profiles/km_bands_r02.txt)
     dv.host_lo = lo;
     dv.host_mul = dv.ordered ? (uint64_t)(((unsigned __int128)scr_n << 64) / span) : 0;
   }
   if (cudaEventCreateWithFlags(&c->chain_ev, cudaEventDisableTiming) != cudaSuccess) return fail(FLECHE_ECUDA);
-  // KM: enough warps for the expected unique misses, km_bps CTAs of 4 warps per SM
-  c->km_blocks = (int)std::min<int64_t>((int64_t)c->km_bps * c->sm_count,
-                                        std::max<int64_t>(1, (cfg->max_lookups + 255) / 256));
+  // KM: enough warps for the expected unique misses, km_bps CTAs of 4 warps per SM, and no
+  // more CTAs than fit at once (cooperative launch: its grid barrier needs them all resident)
   c->km_smem = (size_t)kKmWarps * ((bytes ? kKmSmemF4 : 0) + ((cfg->flags & FLECHE_FLAG_HOST_ASSIST) ? kHaSmemF4 : 0)) *
                sizeof(float4);
-  if (c->km_smem > 48 * 1024 &&
-      cudaFuncSetAttribute((const void*)km_fn(bytes, c->cls_dim.size() == 1 ? c->max_dim : 0),
-                           cudaFuncAttributeMaxDynamicSharedMemorySize, (int)c->km_smem) != cudaSuccess)
-    return fail(FLECHE_ECUDA);
-  c->kd_blocks = std::max(1, std::min(c->km_blocks, c->sm_count));  // one wave: duplicates are few
+  {
+    const void* km = (const void*)km_fn(bytes, c->cls_dim.size() == 1 ? c->max_dim : 0);
+    if (c->km_smem > 48 * 1024 &&
+        cudaFuncSetAttribute(km, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)c->km_smem) != cudaSuccess)
+      return fail(FLECHE_ECUDA);
+    int per_sm = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, km, 128, c->km_smem) != cudaSuccess || per_sm < 1)
+      return fail(FLECHE_ECUDA);
+    c->km_blocks = (int)std::min<int64_t>((int64_t)std::min(c->km_bps, per_sm) * c->sm_count,
+                                          std::max<int64_t>(1, (cfg->max_lookups + 255) / 256));
+  }
   // decoupled hit copy: uniform layout only (the bytes layout compacts set regions in KM,
   // which may move rows a concurrent copy reads; epoch protection covers the uniform slots)
   c->decoupled = !bytes && !(cfg->flags & FLECHE_FLAG_FUSED_HIT_COPY) && getenv("FLECHE_FUSED_GATHER") == nullptr;
@@ -901,6 +922,7 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
       dv.ha_min_rows = (uint32_t)env_u("FLECHE_HA_MIN_ROWS", 32768);
     }
     h->nt_stores = env_u("FLECHE_HA_NT", 1) != 0 && __builtin_cpu_supports("avx2");
+    h->delay_ns = env_u("FLECHE_HA_DELAY_US", 0) * 1000ull;
     h->host.assign(cfg->host_tables, cfg->host_tables + n);
     h->card = c->card;
     h->dims = c->dims;
@@ -1020,10 +1042,15 @@ fleche_status fleche_query_host(fleche_ctx* c, const int64_t* const* ids, const 
   st = order_on(c, s);
   if (st != FLECHE_OK) return st;
   std::vector<const int64_t*> dids(c->n);
-  // one copy when the per-table host arrays are consecutive in memory, else one per table
+  // one copy when the non-empty per-table host arrays are consecutive in memory, else one
+  // per table (empty tables are skipped: their pointers may be anything)
   bool contiguous = true;
-  for (int t = 0; t + 1 < c->n; ++t)
-    if (lengths[t] > 0 && ids[t] + lengths[t] != ids[t + 1]) contiguous = false;
+  const int64_t* expect = nullptr;
+  for (int t = 0; t < c->n; ++t) {
+    if (lengths[t] == 0) continue;
+    if (expect && ids[t] != expect) contiguous = false;
+    expect = ids[t] + lengths[t];
+  }
   int64_t acc = 0;
   const int64_t* first = nullptr;
   for (int t = 0; t < c->n; ++t) {
@@ -1203,7 +1230,7 @@ fleche_status fleche_kernel_times_ex(fleche_ctx* c, double* ms4, uint64_t* queri
   if (c->poisoned) return FLECHE_ESTATE;
   double acc[4] = {0, 0, 0, 0};
   size_t i = 0;
-  for (int k : c->ev_kinds) {  // events: [start, after KQ, after KM, after KD (, after KP)]
+  for (int k : c->ev_kinds) {  // events: [start, after KQ, after KM (incl. restore), same again (, after KP)]
     FL_CUDA(c, cudaEventSynchronize(c->ev_pool[i + k - 1]));
     for (int j = 0; j + 1 < k; ++j) {
       float x = 0;
@@ -1303,10 +1330,8 @@ fleche_status launch_keys(fleche_ctx* c, const uint32_t* keys, int64_t count, fl
     c->kernels++;
   }
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
-  launch_k(kPdlKM, km_fn(false, c->cls_dim.size() == 1 ? c->max_dim : 0), c->km_blocks, 128, c->km_smem, s, c->dv, ka);
+  launch_miss(c, s, ka);
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
-  launch_k(kPdlKD, kd_fn(), c->kd_blocks, 128, 0, s, c->dv, rows);
-  c->kernels += 2;
   launch_scan(c, s);
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;
   cudaError_t e = cudaGetLastError();

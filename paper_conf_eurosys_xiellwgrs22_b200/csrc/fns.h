@@ -17,7 +17,6 @@ template <int MAXT> using KpFn = void (*)(PArgs<MAXT>, const TableInfo*);
 template <int MAXT> using KrFn = void (*)(RArgs<MAXT>, RouteDev, const TableInfo*);
 template <int MAXT> using KrsFn = void (*)(RArgs<MAXT>, RouteDev, const float*, const uint8_t*, float*, PeerArgs);
 using KmFn = void (*)(Dev, KMArgs);
-using KdFn = void (*)(Dev, float*);
 using ProbeFn = void (*)(const float*, uint64_t, int64_t, uint64_t, float*);
 using KpkFn = void (*)(RouteDev, uint32_t*, int64_t*, PeerKeys);
 using KeFn = void (*)(Dev, KEArgs);
@@ -25,8 +24,7 @@ using KeFn = void (*)(Dev, KEArgs);
 template <int MAXT> KqFn<MAXT> kq_fn();   // fused query (k_query.cu)
 template <int MAXT> KqFn<MAXT> kg_fn();   // decoupled hit copy (k_query.cu)
 template <int MAXT> KpFn<MAXT> kp_fn();   // pooling (k_query.cu)
-KmFn km_fn(bool bytes, int dim);          // miss kernel: bytes layout / uniform width dim / 0 = per class (k_miss.cu)
-KdFn kd_fn();                             // duplicate restore (k_misc.cu)
+KmFn km_fn(bool bytes, int dim);          // miss kernel + restore (cooperative): bytes layout / uniform width dim / 0 = per class (k_miss.cu)
 KeFn ke_hist_fn();                        // watermark scan: age histogram (k_misc.cu)
 KeFn ke_evict_fn();                       // watermark scan: threshold + evict (k_misc.cu)
 ProbeFn probe_fn(int dim);                // host-link probe (k_misc.cu)

@@ -1,11 +1,10 @@
-// k_misc.cu — instantiates the restore kernel (KD), the host-link probe and the
+// k_misc.cu — instantiates the watermark scan kernels, the host-link probe and the
 // key-sharded route / pack / restore kernels.
 #include "fleche.h"
 #include "fns.h"
 
 namespace fl {
 
-KdFn kd_fn() { return kd_kernel<0>; }
 KeFn ke_hist_fn() { return ke_hist_kernel<0>; }
 KeFn ke_evict_fn() { return ke_evict_kernel<0>; }
 

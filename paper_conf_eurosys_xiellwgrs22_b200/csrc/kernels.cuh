@@ -119,14 +119,15 @@ struct DupRec {  // a later occurrence of a missed key in the same batch
 
 struct Ctl {
   uint32_t epoch;  // current batch epoch (1-based); advanced by the last KM CTA
-  uint32_t done;   // KM CTA arrival counter
+  uint32_t done;   // KM grid barrier arrivals (before the restore)
+  uint32_t done2;  // KM CTA arrivals at the end (the last one closes the batch)
   uint32_t err_invalid;
   uint32_t ha_rung;  // host-assisted: epoch whose doorbell KM has rung (warps poll host flags after it)
   uint32_t counts[2][8];  // [epoch & 1][class 0..5: unique misses; 7: duplicate misses]
-  unsigned long long ha_f[2];  // [epoch & 1] host-assisted staging floats allocated
   long long occ_bytes;    // row bytes currently cached
   uint32_t ke_done;       // watermark eviction: KE2 CTA arrival counter
-  uint32_t ke_pad;
+  uint32_t km_bar;        // KM grid barrier: epoch whose owner rows are all in `out`
+  long long ke_occ;       // watermark eviction: occ_bytes as KE1 saw it (KE2's one snapshot per scan)
 };
 
 // Host-assisted miss fetch (FLECHE_FLAG_HOST_ASSIST).  The owner lane of each unique
@@ -168,7 +169,7 @@ struct Dev {
   unsigned long long* stats;  // [kStripes][kNumCtr]
   const TableInfo* tables;    // [n]
   uint32_t sets, rows, scr_mask, hash_seed;
-  int32_t dim, admit_all;     // dim: row width of the uniform layout
+  int32_t dim, admit_all;     // dim: row width of the uniform layout (bytes layout: the widest row)
   uint64_t admit_thr, admit_seed;
   int32_t bytes;     // 0 = uniform layout, 1 = bytes layout
   uint32_t set_units;  // bytes layout: region of a set in 32 B units (<= 256)
@@ -179,7 +180,7 @@ struct Dev {
   // monotone in its host-row address, slot0 = ((addr - host_lo) * host_mul) >> 64, so KM
   // can hand each warp a contiguous address window (host-link reads in address order)
   int32_t ordered;
-  int32_t pad2;
+  int32_t bands;     // ordered: band-major sweep, ~bands misses per warp per band (0: M; < 0: off)
   uint64_t host_lo, host_mul;
   // host-assisted miss fetch (mapped pinned host memory; see HaReq)
   int32_t ha;                  // 1 = host-assisted miss fetch on
@@ -698,27 +699,14 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
       if (kind == 1 && lane == leader) b = atomicAdd(&dv.ctl->counts[par][cls], (uint32_t)__popc(grp));
       b = __shfl_sync(kFull, b, leader);
       uint64_t hst = kNoStage;
-      if (dv.ha && dv.bytes) {  // host-assisted, mixed widths: a staging slot (warp-aggregated)
-        const int myd = kind == 1 ? d : 0;
-        int incl = myd;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-          const int y = __shfl_up_sync(kFull, incl, o);
-          if (lane >= o) incl += y;
-        }
-        const int tot = __shfl_sync(kFull, incl, 31);
-        unsigned long long f0 = 0;
-        if (lane == 0) f0 = atomicAdd(&dv.ctl->ha_f[par], (unsigned long long)tot);
-        f0 = __shfl_sync(kFull, f0, 0);
-        const uint64_t so = f0 + (uint64_t)(incl - myd);
-        if (kind == 1 && so + (uint64_t)d <= dv.ha_stage_floats) hst = so;
-      }
       if (kind == 1) {
         const uint32_t r = b + __popc(grp & lt);
         const int64_t li = qa.cls_off[cls] + r;  // miss-list index = request index
-        // uniform rows: the slot follows the list index (class regions are disjoint at
-        // ascending widths), so a block's staged rows are contiguous
-        if (dv.ha && !dv.bytes && (uint64_t)(li + 1) * (uint64_t)d <= dv.ha_stage_floats) hst = (uint64_t)li * d;
+        // host-assisted staging slot = the list index times the widest row: every staging
+        // block (kHaBlock list indices) owns a fixed region, written only by the host
+        // thread that owns the block, batch after batch (no slot of a timed-out block can
+        // be handed to another thread's block); rows past the buffer are read zero-copy
+        if (dv.ha && (uint64_t)(li + 1) * (uint64_t)dv.dim <= dv.ha_stage_floats) hst = (uint64_t)li * dv.dim;
         dv.miss[li] = MissRec{off, fk, scr, qa.t0 + t, 0, hst};
         dv.owner_off[scr] = off;
 #ifdef FLECHE_EXPERIMENTS
@@ -824,26 +812,28 @@ __device__ __forceinline__ int64_t claim_victim(const Dev& dv, const TableInfo* 
   unsigned long long* ip = dv.ipos + (size_t)s * 32u;
   const unsigned long long mine = ((unsigned long long)epoch << 32) | ((unsigned long long)pos << 1) | 1ull;
   while (true) {
-    uint32_t kk[32], tt[32];
+    // argmin (ts, key) over the ways not touched in this batch; the 32 keys and stamps
+    // arrive as 16 B vectors and are scanned with compile-time indices (no local memory)
+    unsigned long long best = ~0ull;
+    int bw = -1;
+    uint32_t bkey = kEmpty;
 #pragma unroll
     for (int q = 0; q < 8; ++q) {
       const uint4 a = ld_cg_v4u(kp + 4 * q), b = ld_cg_v4u(tp + 4 * q);
-      kk[4 * q] = a.x; kk[4 * q + 1] = a.y; kk[4 * q + 2] = a.z; kk[4 * q + 3] = a.w;
-      tt[4 * q] = b.x; tt[4 * q + 1] = b.y; tt[4 * q + 2] = b.z; tt[4 * q + 3] = b.w;
-    }
-    unsigned long long best = ~0ull;
-    int bw = -1;
+      const uint32_t ka[4] = {a.x, a.y, a.z, a.w}, ta[4] = {b.x, b.y, b.z, b.w};
 #pragma unroll
-    for (int w = 0; w < 32; ++w) {
-      const unsigned long long r = ((unsigned long long)tt[w] << 32) | kk[w];
-      if (w < nways && tt[w] < epoch && r < best) { best = r; bw = w; }
+      for (int j = 0; j < 4; ++j) {
+        const int w = 4 * q + j;
+        const unsigned long long r = ((unsigned long long)ta[j] << 32) | ka[j];
+        if (w < nways && ta[j] < epoch && r < best) { best = r; bw = w; bkey = ka[j]; }
+      }
     }
     if (bw >= 0) {
       const unsigned long long cur = ld_cg_u64(ip + bw);
       if ((uint32_t)(cur >> 32) == epoch) continue;  // claimed an instant ago; its ts is on the way
       if (atomicCAS(ip + bw, cur, mine) != cur) continue;
       tp[bw] = epoch;
-      *old_key = kk[bw];
+      *old_key = bkey;
       *took_over = false;
       return (int64_t)s * 32 + bw;
     }
@@ -858,7 +848,7 @@ __device__ __forceinline__ int64_t claim_victim(const Dev& dv, const TableInfo* 
     if (ww < 0 || ((worst >> 1) & 0x7FFFFFFFull) <= pos) return kClaimBypass;
     if (worst & 1ull) return kClaimRetry;  // still being written by its claimer
     if (atomicCAS(ip + ww, worst, mine) != worst) continue;
-    *old_key = kk[ww];
+    *old_key = ld_cg_u32(kp + ww);  // published before its claimer cleared BUSY (fenced)
     *took_over = true;
     return (int64_t)s * 32 + ww;
   }
@@ -1214,11 +1204,17 @@ __device__ __forceinline__ void km_rows(const Dev& dv, float* __restrict__ out, 
       chunk(has, m);
     }
   } else {
-    // address-ordered scratch: warp gw owns a contiguous slot window = a contiguous window
-    // of host addresses, so the GPU's host-link reads go out in (near) address order
+    // address-ordered scratch (slot ~ host address).  Band-major sweep: the slot space is cut
+    // into B bands of about M misses per warp each, and band b is cut into nw sub-windows, so
+    // round b of every warp reads rows of band b: the batch's host reads sweep the host tier
+    // once in address order and the reads in flight at any time share a narrow address band
+    // (translation locality: a sorted burst of 8K rows ran 92 vs 115 us unsorted,
+    // profiles/burst_cold_r02.json).  dv.bands < 0: one contiguous window per warp.
     const uint32_t nslots = dv.scr_mask + 1u;
-    const uint32_t per = (nslots + nw - 1) / nw;
-    const uint32_t lo = min(nslots, gw * per), hi = min(nslots, lo + per);
+    const uint32_t bw = dv.bands > 0 ? (uint32_t)dv.bands : (uint32_t)M;  // misses per warp per band
+    const uint32_t B = dv.bands >= 0 ? max(1u, (nmiss + nw * bw - 1) / (nw * bw)) : 1u;
+    const uint32_t band = (nslots + B - 1) / B;
+    const uint32_t per = (band + nw - 1) / nw;
     uint32_t my_slot = 0;
     int P = 0;  // misses collected so far (lanes 0..P-1 hold their slots)
     auto flush = [&]() {
@@ -1239,6 +1235,8 @@ __device__ __forceinline__ void km_rows(const Dev& dv, float* __restrict__ out, 
       chunk(has, m);
       P = 0;
     };
+    for (uint32_t b = 0; b < B; ++b) {
+    const uint32_t lo = min(nslots, b * band + gw * per), hi = min(min(nslots, (b + 1) * band), lo + per);
     for (uint32_t s1 = lo; s1 < hi; s1 += 256) {  // 8 tag loads per lane in flight, then in order
       unsigned long long tags[8];
 #pragma unroll
@@ -1259,6 +1257,7 @@ __device__ __forceinline__ void km_rows(const Dev& dv, float* __restrict__ out, 
         }
       }
     }
+    }
     if (__any_sync(kFull, P > 0)) flush();
   }
 #ifdef FLECHE_EXPERIMENTS
@@ -1276,6 +1275,16 @@ template <bool BYTES, int D>
 struct KmM {
   static constexpr int value = D >= 256 ? 4 : (BYTES || D >= 64 ? 8 : 16);
 };
+
+// Grid barrier helpers (KM is a cooperative launch: every CTA is resident at once).
+__device__ __forceinline__ uint32_t ld_acquire_gpu_u32(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_gpu_u32(uint32_t* p, uint32_t v) {
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
 
 // DU > 0: uniform layout of width DU (one class); DU = 0: every width class in turn.
 template <bool BYTES, int DU>
@@ -1366,39 +1375,43 @@ __global__ void __launch_bounds__(128, 4) km_kernel(const __grid_constant__ Dev 
   __syncthreads();
   if (threadIdx.x < kNumCtr && s_ctr[threadIdx.x])
     atomicAdd(dv.stats + (blockIdx.x % kStripes) * kNumCtr + threadIdx.x, s_ctr[threadIdx.x]);
+
+  // A8 restore, the former third kernel (KD) of a batch: every later
+  // occurrence of a missed key copies its owner's row once every owner row is in `out`.
+  // Grid barrier first (the launch is cooperative, so every CTA is resident); skipped by
+  // every CTA alike when the batch has no duplicate misses (the count is final: KQ wrote it).
+  const uint32_t ndup = *(volatile uint32_t*)&dv.ctl->counts[par][kDupSlot];
+  if (ndup) {
+    if (threadIdx.x == 0) {
+      __threadfence();
+      const uint32_t prev = atomicAdd(&dv.ctl->done, 1u);
+      if (prev == gridDim.x - 1) {
+        dv.ctl->done = 0;
+        st_release_gpu_u32(&dv.ctl->km_bar, epoch);
+      } else {
+        while (ld_acquire_gpu_u32(&dv.ctl->km_bar) != epoch) __nanosleep(64);
+      }
+    }
+    __syncthreads();
+    for (uint32_t i = gw; i < ndup; i += nw) {  // owner rows were written by other SMs: read via L2
+      const DupRec r = dv.dup[i];
+      const float* src = ka.out + dv.owner_off[r.scr];
+      for (int c = lane; c < r.dim / 4; c += 32) st_v4(ka.out + r.off + 4 * c, ld_cg_v4(src + 4 * c));
+    }
+  }
   pdl_trigger();
+  __syncthreads();
   if (threadIdx.x == 0) {
     __threadfence();
-    const uint32_t prev = atomicAdd(&dv.ctl->done, 1u);
+    const uint32_t prev = atomicAdd(&dv.ctl->done2, 1u);
     if (prev == gridDim.x - 1) {  // last CTA closes the batch: next batch's counters, epoch + 1
 #pragma unroll
       for (int c = 0; c < 8; ++c) dv.ctl->counts[par ^ 1][c] = 0;
-      dv.ctl->ha_f[par ^ 1] = 0;
-      dv.ctl->done = 0;
+      dv.ctl->done2 = 0;
       __threadfence();
       *(volatile uint32_t*)&dv.ctl->epoch = epoch + 1u;
     }
   }
-}
-
-// KD restore: every duplicate occurrence of a missed key copies its owner's
-// row (written by KM) in parallel.
-template <int = 0>
-__global__ void __launch_bounds__(128) kd_kernel(const __grid_constant__ Dev dv, float* __restrict__ out) {
-  pdl_wait();
-  // KM's last CTA already advanced the epoch: this batch is epoch - 1
-  const uint32_t epoch = *(volatile uint32_t*)&dv.ctl->epoch - 1u;
-  const int par = epoch & 1u;
-  const uint32_t ndup = *(volatile uint32_t*)&dv.ctl->counts[par][kDupSlot];
-  const int lane = threadIdx.x & 31;
-  const uint32_t gw = (threadIdx.x >> 5) * gridDim.x + blockIdx.x;
-  const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
-  for (uint32_t k = gw; k < ndup; k += nw) {
-    const DupRec r = dv.dup[k];
-    const float* src = out + dv.owner_off[r.scr];
-    for (int c = lane; c < r.dim / 4; c += 32) st_v4(out + r.off + 4 * c, ld_cg_v4(src + 4 * c));
-  }
-  pdl_trigger();
 }
 
 // Pooling: one thread per (bag, 4-float column); sums the bag's staged
@@ -1464,7 +1477,11 @@ __global__ void __launch_bounds__(256) ke_hist_kernel(const __grid_constant__ De
   __syncthreads();
   pdl_wait();
   const uint32_t epoch = *(volatile uint32_t*)&dv.ctl->epoch - 1u;  // KM advanced it
+  // nothing changes occ_bytes while KE1 runs (KM has completed, KE2 has not started), so
+  // every CTA reads the same value; CTA 0 records it as the scan's one snapshot for KE2,
+  // whose CTAs lower occ_bytes while others may not have started yet
   const long long occ = *(volatile long long*)&dv.ctl->occ_bytes;
+  if (blockIdx.x == 0 && threadIdx.x == 0) dv.ctl->ke_occ = occ;
   if (occ <= ea.hi) {
     pdl_trigger();
     return;
@@ -1505,8 +1522,8 @@ __global__ void __launch_bounds__(256) ke_evict_kernel(const __grid_constant__ D
   __shared__ int s_last;
   pdl_wait();
   const uint32_t epoch = *(volatile uint32_t*)&dv.ctl->epoch - 1u;
-  const long long occ = *(volatile long long*)&dv.ctl->occ_bytes;
-  if (occ <= ea.hi) {
+  const long long occ = *(volatile long long*)&dv.ctl->ke_occ;  // KE1's snapshot: the same in every CTA
+  if (occ <= ea.hi) {  // every CTA takes this exit together (no histogram was built)
     pdl_trigger();
     return;
   }

@@ -114,6 +114,39 @@ def test_assisted_mixed_widths_pooled():
     assert st["assist_timeouts"] == 0 and st["assisted_rows"] == st["unique_misses"]
 
 
+@pytest.mark.parametrize("pooled", [False, True])
+def test_assisted_mixed_widths_stalled_threads(monkeypatch, pooled):
+    # fault injection: every host thread gathers each block 300 us late while KM waits at
+    # most 40 us, so blocks time out and KM reads those rows itself; the stalled threads'
+    # late stores must never land in a slot another block of a later batch already
+    # published (each list index owns a fixed staging slot, and only one thread ever
+    # writes a given block).  Mixed widths: the bytes layout
+    monkeypatch.setenv("FLECHE_HA_DELAY_US", "300")
+    monkeypatch.setenv("FLECHE_HA_TIMEOUT_US", "40")
+    w = configs.get("cfg4")
+    w = w.with_(cards=[max(3, c // 64) for c in w.cards], batch_size=96, invalid_ppm=2000, skews=[0.7] * w.n)
+    tabs = _tables(w)
+    gpu, glob = H.make_pair(w, tabs, O.MODE_GLOBAL, max_lookups=w.batch(0).lookups * 2, flags=HA)
+    for b in range(16):
+        bt = w.batch(b)
+        ids = [torch.from_numpy(x).cuda() for x in bt.ids]
+        if pooled:
+            offs = [torch.from_numpy(o).cuda() for o in bt.offsets]
+            n_out = gpu.pooled_floats([o.size - 1 for o in bt.offsets])
+            out = torch.full((max(n_out, 1),), float("nan"), device="cuda")
+            gpu.query_pooled(ids, offs, out)
+            ref = glob.query_pooled(bt.ids, bt.offsets)
+        else:
+            n_out = gpu.out_floats([x.size for x in bt.ids])
+            out = torch.full((max(n_out, 1),), float("nan"), device="cuda")
+            gpu.query(ids, out)
+            ref = glob.query(bt.ids)
+        torch.cuda.synchronize()
+        assert H.bits_equal(out[:n_out].cpu().numpy(), ref), b
+    st = gpu.stats()
+    assert st["assist_timeouts"] > 0, st
+
+
 def test_assisted_cuda_graph_replay():
     # requests, doorbell and ready flags are epoch-tagged on the device: graph replays work
     w = configs.get("cfg0")

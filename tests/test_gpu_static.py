@@ -74,7 +74,7 @@ def test_static_per_table_values_and_hit_ratio(flags, div, tol):
     st = gpu.stats()
     assert st["occupancy_bytes"] <= st["capacity_bytes"]
     if flags & PER_TABLE:
-        assert st["kernels_launched"] > 2 * st["batches"]
+        assert st["kernels_launched"] > 1 * st["batches"]
 
 
 def test_per_table_launch_matches_fused_exactly():
@@ -91,8 +91,8 @@ def test_per_table_launch_matches_fused_exactly():
     assert sa["bypassed"] == 0
     for k in H.STAT_KEYS_EXACT:
         assert sa[k] == sc[k], k
-    # per-table: n x KQ + KM + KD; fused: KQ + KM + KD (+ KG when the hit copy is decoupled)
-    assert sc["kernels_launched"] == 15 * (w.n + 2) and sa["kernels_launched"] in (45, 60)
+    # per-table: n x KQ + KM; fused: KQ + KM (+ KG when the hit copy is decoupled)
+    assert sc["kernels_launched"] == 15 * (w.n + 1) and sa["kernels_launched"] in (30, 45)
 
 
 def test_flat_beats_static_on_skewed_table_sizes():

@@ -67,13 +67,13 @@ int main() {
   cudaEventCreate(&j);
   const uint64_t all_rows = span / 256;
   auto timeit = [&](auto&& body) {
-    body(0x777);  // warm-up
+    body(0xABCDEF1234567ull);  // warm-up
     cudaDeviceSynchronize();
     float tot = 0;
     for (int it = 0; it < 8; ++it) {
       cudaEventRecord(a, s1);
       cudaStreamWaitEvent(s2, a, 0);
-      body(1000 + it * 77);
+      body((uint64_t)(it + 1) * 0x9E3779B97F4A7C15ull);
       cudaEventRecord(j, s2);
       cudaStreamWaitEvent(s1, j, 0);
       cudaEventRecord(b, s1);

@@ -72,8 +72,8 @@ class Workload:
         d.update(kw)
         return Workload(**d)
 
-    def make_tables(self, nthreads: int = 0):
-        return gen.make_tables(self.cards, self.dims, self.value_mode, nthreads)
+    def make_tables(self, nthreads: int = 0, buf=None):
+        return gen.make_tables(self.cards, self.dims, self.value_mode, nthreads, buf)
 
     def batch(self, b: int, rank: int = 0, nthreads: int = 0) -> Batch:
         """Batch b; rank r takes samples [r*B, (r+1)*B) of the global batch (SURVEY d-2 cfg5)."""

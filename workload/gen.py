@@ -91,11 +91,16 @@ def fill_table(dst: np.ndarray, t: int, mode: int = 0, row0: int = 0, nthreads: 
     lib().flg_fill_table(seeds()["val"], t, row0, rows, d, d, mode, dst.ctypes.data, nthreads)
 
 
-def make_tables(cards, dims, mode: int = 0, nthreads: int = 0):
-    """One contiguous float32 buffer holding every table row-major; returns (buf, [views])."""
+def make_tables(cards, dims, mode: int = 0, nthreads: int = 0, buf: np.ndarray | None = None):
+    """One contiguous float32 buffer holding every table row-major; returns (buf, [views]).
+    `buf` (optional): a caller-provided float32 buffer of at least sum(c_t * d_t) elements
+    (e.g. driver-allocated pinned memory) to generate into."""
     sizes = [int(c) * int(d) for c, d in zip(cards, dims)]
     total = sum(sizes)
-    buf = np.empty(total, dtype=np.float32)
+    if buf is None:
+        buf = np.empty(total, dtype=np.float32)
+    assert buf.dtype == np.float32 and buf.flags["C_CONTIGUOUS"] and buf.size >= total
+    buf = buf[:total]
     views = []
     off = 0
     for t, (c, d) in enumerate(zip(cards, dims)):
