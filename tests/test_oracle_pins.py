@@ -567,3 +567,123 @@ def test_paper_synthetic_hit_rates_loose(frac, paper):
     s = o.stats()
     uh = (s["unique_hits"] - s0["unique_hits"]) / (s["unique_keys"] - s0["unique_keys"])
     assert abs(uh - paper) < 0.03, (uh, paper)
+
+
+# ------------------------------------------- policy: byte-budgeted sets (MODE_SETBYTES)
+def _fmix32(h: int) -> int:
+    """murmur3 fmix32 (the set hash of reading R12), written out here independently."""
+    h ^= h >> 16
+    h = (h * 0x85EBCA6B) & 0xFFFFFFFF
+    h ^= h >> 13
+    h = (h * 0xC2B2AE35) & 0xFFFFFFFF
+    h ^= h >> 16
+    return h
+
+
+def test_setbytes_hand_worked_example():
+    """MODE_SETBYTES (reading R22) against a hand-worked run: a way-limit eviction, a
+    byte-limit eviction and a bypass with every candidate touched."""
+    g = json.load(open(os.path.join(GOLD, "setbytes_example.json")))
+    base = [0, 64, 128]  # reading R3 for three tables of c = 64 (f = 6), ties by index
+    assert O.encode(g["cards"])[1].tolist() == base
+    S = g["cache_bytes"] // g["set_bytes"]
+    for sname, keys in g["sets"].items():
+        for t, i in keys:
+            assert (_fmix32((base[t] + i) ^ g["hash_seed"]) * S) >> 32 == int(sname), (t, i)
+    tabs = _tiny_tables(g["cards"], g["dims"])
+    o = O.Oracle(g["cards"], g["dims"], tabs, g["cache_bytes"], O.MODE_SETBYTES, hash_seed=g["hash_seed"],
+                 ways=g["ways"], set_bytes=g["set_bytes"])
+    prev = set()
+    for bt in g["batches"]:
+        s0 = o.stats()
+        o.query([np.array(x, np.int64) for x in bt["ids"]])
+        s1 = o.stats()
+        for k in ("hits", "inserted", "bypassed"):
+            assert s1[k] - s0[k] == bt[k], (bt, k)
+        assert s1["occupancy_bytes"] == bt["occupancy"]
+        now = set(map(tuple, o.cached_keys()))
+        assert prev - now == set(map(tuple, bt["evicted"])), bt
+        assert s1["evicted"] - s0["evicted"] == len(bt["evicted"])
+        prev = now
+    s = o.stats()
+    assert s["hits"] == g["total_hits"] and s["lookups"] == g["total_lookups"]
+    assert prev == set(map(tuple, g["final_cached"]))
+    assert s["bypass_full"] == 1
+
+
+def test_setbytes_equal_widths_is_setassoc():
+    """With one row width and set_bytes = 32 rows, the byte budget binds exactly when the 32
+    ways do, so MODE_SETBYTES must reproduce MODE_SETASSOC batch by batch (counters and the
+    cached keys); a dropped byte check, a wrong victim or a stale set-bytes counter would
+    diverge under this churn (low skew, tiny cache, invalid IDs)."""
+    d = 8
+    w = configs.get("cfg0").with_(dims=[d] * 7, skews=[0.6] * 7, invalid_ppm=3000, batch_size=500)
+    tabs = _tiny_tables(w.cards, w.dims)
+    S = 5
+    cap = S * 32 * 4 * d
+    a = O.Oracle(w.cards, w.dims, tabs, cap, O.MODE_SETASSOC, hash_seed=0x9E3779B9)
+    b = O.Oracle(w.cards, w.dims, tabs, cap, O.MODE_SETBYTES, hash_seed=0x9E3779B9, ways=32, set_bytes=32 * 4 * d)
+    for bi in range(60):
+        ids = w.batch(bi).ids
+        assert np.array_equal(a.query(ids).view(np.uint32), b.query(ids).view(np.uint32))
+        sa, sb = a.stats(), b.stats()
+        for k in ("hits", "misses", "invalid", "unique_hits", "unique_misses", "inserted", "evicted", "bypassed",
+                  "bypass_full", "occupancy_bytes"):
+            assert sa[k] == sb[k], (bi, k, sa[k], sb[k])
+        assert sorted(a.cached_keys()) == sorted(b.cached_keys()), bi
+    assert a.stats()["evicted"] > 1000
+
+
+def test_setbytes_invariants_under_churn():
+    """Mixed widths under churn: every set holds <= `ways` rows whose bytes sum to <=
+    set_bytes (sets recomputed here with the hash of reading R12); the live row bytes sum to
+    the reported occupancy <= S * set_bytes; no key is cached twice; every cached key is a
+    valid row; inserted - evicted = cached rows."""
+    w = configs.get("cfg0").with_(dims=[8, 16, 32, 64, 128, 8, 32], skews=[0.5] * 7, invalid_ppm=3000,
+                                  batch_size=400)
+    tabs = _tiny_tables(w.cards, w.dims)
+    ways, sb, seed = 8, 1024, 77
+    cap = 13 * sb + 100  # 13 sets; the remainder is not usable
+    o = O.Oracle(w.cards, w.dims, tabs, cap, O.MODE_SETBYTES, hash_seed=seed, ways=ways, set_bytes=sb)
+    _, base, _ = O.encode(w.cards)
+    S = cap // sb
+    for bi in range(50):
+        o.query(w.batch(bi).ids)
+        s = o.stats()
+        keys = o.cached_keys()
+        assert len(keys) == len(set(keys))
+        assert all(0 <= i < w.cards[t] for t, i in keys)
+        per_set, rows = {}, {}
+        for t, i in keys:
+            st = (_fmix32((int(base[t]) + i) ^ seed) * S) >> 32
+            per_set[st] = per_set.get(st, 0) + 4 * w.dims[t]
+            rows[st] = rows.get(st, 0) + 1
+        assert all(v <= sb for v in per_set.values()) and all(v <= ways for v in rows.values())
+        assert s["occupancy_bytes"] == sum(per_set.values()) <= S * sb == s["capacity_bytes"]
+        assert s["inserted"] - s["evicted"] == len(keys)
+    assert s["evicted"] > 0 and s["bypassed"] > 0
+
+
+@pytest.mark.slow
+def test_setbytes_near_global_on_cfg4_shape():
+    """DESIGN reading R22: one byte budget over 32-way, 4 KiB sets stays close to the global
+    byte-LRU (MODE_GLOBAL) on a cfg4-shaped workload (100 tables, widths 8-128 floats,
+    skews 0.8-1.2, multi-hot bags): 0.30 pp below it at this 1/64 scale, 0.24 pp at 1/16
+    (profiles/setbytes_vs_global_r02.txt), far inside the 1 pp parity bar, while a static
+    per-width split would cost ~3.4 pp (SURVEY c-6)."""
+    w = configs.get("cfg4")
+    w = w.with_(cards=[max(3, c // 64) for c in w.cards], batch_size=256)
+    tabs = w.make_tables()[1]
+    hits = {}
+    for mode in (O.MODE_GLOBAL, O.MODE_SETBYTES):
+        o = O.Oracle(w.cards, w.dims, tabs, w.cache_bytes, mode, hash_seed=0x9E3779B9, ways=32, set_bytes=4096)
+        for b in range(40):
+            bt = w.batch(b)
+            o.query_pooled(bt.ids, bt.offsets)
+        s0 = o.stats()
+        for b in range(40, 100):
+            bt = w.batch(b)
+            o.query_pooled(bt.ids, bt.offsets)
+        s1 = o.stats()
+        hits[mode] = (s1["hits"] - s0["hits"]) / ((s1["hits"] + s1["misses"]) - (s0["hits"] + s0["misses"]))
+    assert 0 <= hits[O.MODE_GLOBAL] - hits[O.MODE_SETBYTES] < 0.005, hits
