@@ -169,7 +169,11 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out);
  * IDs outside [0, c_t) (reading R15) yield a zero row, count as `invalid`, are never
  * cached, and make the next fleche_stats return FLECHE_ERANGE.  Caller owns ids and
  * out; they must stay valid until the stream has passed this call.  Enqueues 2
- * kernels and never blocks the host. */
+ * kernels on `stream` -- the query kernel (KQ: probe, hit gather, miss dedup) and the
+ * miss kernel (KM, a cooperative launch: miss fetch, insert, restore of duplicate
+ * misses) -- plus, from 512K lookups per batch, the decoupled hit copy (KG) on a
+ * ctx-owned side stream that `stream` joins; with watermarks set (fleche_set_watermarks)
+ * 2 scan kernels follow.  Never blocks the host. */
 fleche_status fleche_query(fleche_ctx* ctx, const int64_t* const* ids, const int64_t* lengths, float* out,
                            fleche_stream stream);
 
@@ -191,7 +195,7 @@ fleche_status fleche_prefill(fleche_ctx* ctx, const int64_t* const* ids, const i
  *                bag order (reading R16: the oracle's order, so results are bit-identical);
  *                an empty bag gives a zero row; invalid IDs contribute nothing.
  * Every ID is a lookup for the cache (hit/miss/insert as in fleche_query).  Enqueues
- * 3 kernels (query, miss, pooling); the per-ID rows are staged in a ctx-owned buffer
+ * 3 kernels (query, miss + restore, pooling); the per-ID rows are staged in a ctx-owned buffer
  * (max_lookups x max d floats, allocated at the first pooled call). */
 fleche_status fleche_query_pooled(fleche_ctx* ctx, const int64_t* const* ids, const int64_t* const* offsets,
                                   const int64_t* bags, const int64_t* nnz, float* out, fleche_stream stream);
@@ -247,6 +251,18 @@ const char* fleche_strerror(fleche_status status);
  * fleche_debug_locations: bytes layout only: loc[S*32] = (size << 8) | offset of each
  *   way's row inside its set's region, both in 32-byte units. */
 fleche_status fleche_get_encoding(fleche_ctx* ctx, uint64_t* base, int32_t* fbits, int32_t* key_bits);
+
+/* The flat-key code fleche_create would build for these cardinalities, without a ctx or a
+ * GPU (host-only; P:L640-652 size-aware coding, readings R3 and R24).
+ *   cards[n] (host, c_t >= 1); key_bits = the config's key_bits (0 = exact code);
+ *   out: base[n] (first flat key of table t), fbits[n] (feature bits f_t, or g_t for a
+ *   hashed table), hashed[n] (1 = the table's feature IDs are hashed; may be NULL),
+ *   *key_bits_out = the code's key width (B_min for the exact code).
+ * Errors: FLECHE_EINVAL on null pointers, n outside [1, FLECHE_MAX_TABLES], c_t < 1,
+ *   key_bits outside [0, 32], or a code that does not fit (exact code wider than 32 bits
+ *   with key_bits = 0).  Caller owns every buffer. */
+fleche_status fleche_encode(int32_t n, const int64_t* cards, int32_t key_bits, uint64_t* base, int32_t* fbits,
+                            int32_t* hashed, int32_t* key_bits_out);
 fleche_status fleche_get_geometry(fleche_ctx* ctx, int64_t* sets, int64_t* rows, int32_t* row_floats);
 fleche_status fleche_debug_snapshot(fleche_ctx* ctx, uint32_t* keys, uint32_t* ts, size_t ways_cap, float* slab,
                                     size_t slab_floats_cap);
@@ -261,7 +277,7 @@ fleche_status fleche_debug_locations(fleche_ctx* ctx, uint16_t* loc, size_t ways
  *      flat keys, DEVICE) with per-owner counts (send_counts[G], int64, DEVICE).
  *   2. the caller exchanges counts and keys with an all-to-all (NCCL over NVLink);
  *   3. fleche_query_keys(recv_keys, R, rows, flags): the owner answers R flat keys
- *      (its share of every rank's batch) with the ordinary query/miss/restore kernels:
+ *      (its share of every rank's batch) with the ordinary query and miss kernels:
  *      rows[R x d] fp32 (DEVICE, row g answers key g), hit_flags[R] (DEVICE, 1 = hit;
  *      may be NULL); this is one batch (epoch) of the owner's cache;
  *   4. the caller returns rows (and flags) with an all-to-all, owners in rank order,
@@ -324,8 +340,9 @@ fleche_status fleche_ipc_close(void* dptr);
  * fleche_set_profiling: when enabled, every later query records CUDA events on its
  *   stream around each of its kernels (adds ~3 event records per call).
  * fleche_kernel_times: blocking; summed device time (ms) of the query kernel (KQ) and
- *   the insert kernel (KI) over the profiled queries since the last call, and their
- *   count; resets the accumulation.
+ *   of everything after it (*ki_ms: the miss kernel KM, which also restores duplicate
+ *   misses, and the pooling kernel) over the profiled queries since the last call, and
+ *   their count; resets the accumulation.
  * fleche_probe_host_read: measures random-row zero-copy read bandwidth of the host
  *   link: a kernel with the KQ miss-fetch access pattern reads `rows` rows of
  *   `row_bytes` (multiple of 16, <= 4096) at seeded random row indices of the mapped
@@ -333,8 +350,9 @@ fleche_status fleche_ipc_close(void* dptr);
  *   with CUDA events on `stream`; *gbps = rows * row_bytes / time.  Blocking. */
 fleche_status fleche_set_profiling(fleche_ctx* ctx, int enable);
 fleche_status fleche_kernel_times(fleche_ctx* ctx, double* kq_ms, double* ki_ms, uint64_t* queries);
-/* Same accumulation split per kernel: ms4 = {query (KQ), miss (KM), restore (KD),
- * pooling (KP; 0 for one-hot)} summed over the profiled queries; resets. */
+/* Same accumulation split per kernel: ms4 = {query (KQ), miss + restore (KM), 0 (the
+ * former separate restore kernel, now inside KM), pooling (KP; 0 for one-hot)} summed
+ * over the profiled queries; resets. */
 fleche_status fleche_kernel_times_ex(fleche_ctx* ctx, double* ms4, uint64_t* queries);
 /* Tools only: copy the device control block (sizeof = bytes >= its size) to host on a
  * private non-blocking stream, so it can be read while the ctx's streams are stuck. */

@@ -56,6 +56,7 @@ fleche_reset_stats = _sig("fleche_reset_stats", ctypes.c_int, [_vp])
 fleche_destroy = _sig("fleche_destroy", ctypes.c_int, [_vp])
 fleche_strerror = _sig("fleche_strerror", ctypes.c_char_p, [ctypes.c_int])
 fleche_get_encoding = _sig("fleche_get_encoding", ctypes.c_int, [_vp, _vp, _vp, ctypes.POINTER(_i32)])
+fleche_encode = _sig("fleche_encode", ctypes.c_int, [_i32, _vp, _i32, _vp, _vp, _vp, ctypes.POINTER(_i32)])
 fleche_get_geometry = _sig("fleche_get_geometry", ctypes.c_int,
                            [_vp, ctypes.POINTER(_i64), ctypes.POINTER(_i64), ctypes.POINTER(_i32)])
 fleche_debug_snapshot = _sig("fleche_debug_snapshot", ctypes.c_int, [_vp, _vp, _vp, ctypes.c_size_t, _vp,
@@ -93,7 +94,20 @@ EXPORTED = ["fleche_create", "fleche_query", "fleche_query_pooled", "fleche_quer
             "fleche_probe_host_read", "fleche_route", "fleche_query_keys", "fleche_restore", "fleche_shard_stats",
             "fleche_kernel_times_ex", "fleche_set_watermarks", "fleche_prefill", "fleche_debug_ctl",
             "fleche_restore_p2p", "fleche_ipc_handle", "fleche_ipc_open", "fleche_ipc_close", "fleche_ipc_alloc",
-            "fleche_ipc_free", "fleche_route_p2p", "fleche_query_keys_seg"]
+            "fleche_ipc_free", "fleche_route_p2p", "fleche_query_keys_seg", "fleche_encode"]
+
+
+def encode(cards, key_bits: int = 0):
+    """The flat-key code fleche_create builds (host-only, no GPU): (key_bits, base[n], fbits[n], hashed[n])."""
+    c = np.ascontiguousarray(cards, dtype=np.int64)
+    n = len(c)
+    base = np.zeros(n, dtype=np.uint64)
+    fb = np.zeros(n, dtype=np.int32)
+    h = np.zeros(n, dtype=np.int32)
+    kb = _i32()
+    _check(fleche_encode(n, c.ctypes.data, int(key_bits), base.ctypes.data, fb.ctypes.data, h.ctypes.data,
+                         ctypes.byref(kb)), "fleche_encode")
+    return int(kb.value), base, fb, h
 
 
 def ipc_alloc(nbytes: int) -> int:

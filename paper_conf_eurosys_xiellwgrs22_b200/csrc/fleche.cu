@@ -1145,6 +1145,30 @@ fleche_status fleche_get_encoding(fleche_ctx* c, uint64_t* base, int32_t* fbits,
   return FLECHE_OK;
 }
 
+fleche_status fleche_encode(int32_t n, const int64_t* cards, int32_t key_bits, uint64_t* base, int32_t* fbits,
+                            int32_t* hashed, int32_t* key_bits_out) {
+  if (n < 1 || n > FLECHE_MAX_TABLES || !cards || !base || !fbits || !key_bits_out || key_bits < 0 || key_bits > 32)
+    return FLECHE_EINVAL;
+  std::vector<int64_t> card(cards, cards + n);
+  for (int64_t c : card)
+    if (c < 1) return FLECHE_EINVAL;
+  std::vector<uint64_t> b;
+  std::vector<int32_t> fb, h(n, 0);
+  int kb = size_aware_code(card, b, fb);  // same steps as fleche_create
+  if (key_bits > 0 && (kb < 0 || key_bits < kb)) {
+    if (short_code(card, key_bits, b, fb, h) < 0) return FLECHE_EINVAL;
+    kb = key_bits;
+  }
+  if (kb < 0) return FLECHE_EINVAL;
+  for (int t = 0; t < n; ++t) {
+    base[t] = b[t];
+    fbits[t] = fb[t];
+    if (hashed) hashed[t] = h[t];
+  }
+  *key_bits_out = kb;
+  return FLECHE_OK;
+}
+
 fleche_status fleche_get_geometry(fleche_ctx* c, int64_t* sets, int64_t* rows, int32_t* row_floats) {
   if (!c) return FLECHE_EINVAL;
   if (sets) *sets = c->dv.sets;

@@ -110,3 +110,32 @@ def test_p2p_two_processes_one_gpu(tmp_path):
     for r in res:
         assert 0 < r["req_hits"] <= r["req_lookups"] - r["invalid"], r
         assert r["owner_hits"] > 0
+    # hit ratio vs an oracle of G shard caches (SURVEY 8(e) tests): shard g is one cache
+    # of the per-GPU budget that sees, batch by batch, every valid lookup of every rank
+    # whose key it owns (same owner() as the route kernel, tests/shard_double.py); the
+    # requesters' per-lookup hits must match its hits within 1 pp (concurrent insert order)
+    from paper_conf_eurosys_xiellwgrs22_b200.sharded import DEFAULT_OWNER_SEED
+    G = 2
+    w = configs.get("cfg0").with_(invalid_ppm=3000, cache_frac=0.1)  # as in tests/p2p_worker.py
+    tabs = _tables(w)
+    _, base, _ = O.encode(w.cards)
+    orcs = [O.Oracle(w.cards, w.dims, tabs, w.cache_bytes, O.MODE_GLOBAL) for _ in range(G)]
+    for b in range(12):
+        bts = [w.batch(b, rank=r) for r in range(G)]
+        for g in range(G):
+            ids_g = []
+            for t in range(w.n):
+                parts = []
+                for r in range(G):
+                    x = bts[r].ids[t]
+                    ok = (x >= 0) & (x < w.cards[t])
+                    own = owner_of(int(base[t]) + np.where(ok, x, 0), DEFAULT_OWNER_SEED, G) == g
+                    parts.append(x[ok & own])
+                ids_g.append(np.concatenate(parts))
+            orcs[g].query(ids_g)
+    o_hits = sum(o.stats()["hits"] for o in orcs)
+    o_valid = sum(o.stats()["lookups"] for o in orcs)
+    req_hits = sum(r["req_hits"] for r in res)
+    req_valid = sum(r["req_lookups"] - r["invalid"] for r in res)
+    assert req_valid == o_valid, (req_valid, o_valid)
+    assert abs(req_hits - o_hits) <= 0.01 * o_valid, (req_hits, o_hits, o_valid)
