@@ -80,6 +80,8 @@ struct fleche_ctx {
   TableInfo* d_tables = nullptr;
   int km_blocks = 0;
   int km_bps = 4;  // KM CTAs per SM
+  int kq_tma = 0;      // KQ's hit gather by bulk copies through shared memory (row width 32 or 64; 0 = registers)
+  size_t kq_smem = 0;  // its dynamic shared memory (4 warps x 32 rows)
   bool per_table_launch = false;
   // decoupled hit copy (uniform layout): KG on a side stream, forked after KQ, joined after KM
   bool decoupled = false;
@@ -555,7 +557,7 @@ fleche_status launch_query(fleche_ctx* c, const int64_t* const* ids, const int64
   if (decouple) qa.slots = c->d_slots;
   if (total > 0 && !c->per_table_launch) {
     const int64_t blocks = (total + 127) / 128;
-    launch_k(kPdlKQ, kq_fn<MAXT>(), (unsigned)blocks, 128, 0, s, qa, c->dv);
+    launch_k(kPdlKQ, kq_fn<MAXT>(c->kq_tma), (unsigned)blocks, 128, c->kq_smem, s, qa, c->dv);
     c->kernels++;
     if (decouple) {  // fork: the hit copy runs on the side stream, concurrently with KM
       FL_CUDA(c, cudaEventRecord(c->fork_ev, s));
@@ -578,7 +580,7 @@ fleche_status launch_query(fleche_ctx* c, const int64_t* const* ids, const int64
       q1.scan[0] = 0;
       q1.scan[1] = lengths[t];
       q1.out_off[0] = qa.out_off[t];
-      launch_k(kPdlKQ, kq_fn<32>(), (unsigned)((lengths[t] + 127) / 128), 128, 0, s, q1, c->dv);
+      launch_k(kPdlKQ, kq_fn<32>(c->kq_tma), (unsigned)((lengths[t] + 127) / 128), 128, c->kq_smem, s, q1, c->dv);
       c->kernels++;
     }
   }
@@ -859,6 +861,14 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
       return fail(FLECHE_ECUDA);
     c->km_blocks = (int)std::min<int64_t>((int64_t)std::min(c->km_bps, per_sm) * c->sm_count,
                                           std::max<int64_t>(1, (cfg->max_lookups + 255) / 256));
+  }
+  {  // KQ hit gather through the TMA engine (FLECHE_KQ_TMA=0/1; uniform rows of 32 or 64 floats)
+    const char* e = getenv("FLECHE_KQ_TMA");
+    const bool want = e ? atoi(e) != 0 : false;
+    if (want && !bytes && c->cls_dim.size() == 1 && (c->max_dim == 32 || c->max_dim == 64)) {
+      c->kq_tma = c->max_dim;
+      c->kq_smem = (size_t)4 * 32 * c->max_dim * sizeof(float);
+    }
   }
   // decoupled hit copy: uniform layout only (the bytes layout compacts set regions in KM,
   // which may move rows a concurrent copy reads; epoch protection covers the uniform slots)
@@ -1350,7 +1360,7 @@ fleche_status launch_keys(fleche_ctx* c, const uint32_t* keys, int64_t count, fl
   fleche_status st = prof_event(c, s, true, 4);
   if (st != FLECHE_OK) return st;
   if (count > 0) {
-    launch_k(kPdlKQ, kq_fn<MAXT>(), (unsigned)((count + 127) / 128), 128, 0, s, qa, c->dv);
+    launch_k(kPdlKQ, kq_fn<MAXT>(c->kq_tma), (unsigned)((count + 127) / 128), 128, c->kq_smem, s, qa, c->dv);
     c->kernels++;
   }
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;

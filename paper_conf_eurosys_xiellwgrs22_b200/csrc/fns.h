@@ -21,7 +21,7 @@ using ProbeFn = void (*)(const float*, uint64_t, int64_t, uint64_t, float*);
 using KpkFn = void (*)(RouteDev, uint32_t*, int64_t*, PeerKeys);
 using KeFn = void (*)(Dev, KEArgs);
 
-template <int MAXT> KqFn<MAXT> kq_fn();   // fused query (k_query.cu)
+template <int MAXT> KqFn<MAXT> kq_fn(int tma_dim = 0);  // fused query; tma_dim 32/64: bulk-copy hit gather (k_query.cu)
 template <int MAXT> KqFn<MAXT> kg_fn();   // decoupled hit copy (k_query.cu)
 template <int MAXT> KpFn<MAXT> kp_fn();   // pooling (k_query.cu)
 KmFn km_fn(bool bytes, int dim);          // miss kernel + restore (cooperative): bytes layout / uniform width dim / 0 = per class (k_miss.cu)

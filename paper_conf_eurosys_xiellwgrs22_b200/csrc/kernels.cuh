@@ -540,11 +540,48 @@ struct RowBuf {
   }
 };
 
-template <int MAXT>
+// Bulk-copy (TMA engine) helpers for KQ's hit gather (TD > 0): rows land in shared memory
+// through cp.async.bulk with an mbarrier transaction count; the warp's contiguous output
+// block leaves with one bulk store.
+__device__ __forceinline__ void mbar_init(unsigned mb, unsigned count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(mb), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(unsigned mb, unsigned bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mb), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(unsigned mb, unsigned parity) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\tKQ_WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+      "@!p bra KQ_WAIT_%=;\n\t}" ::"r"(mb), "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* smem, const void* gmem, unsigned bytes, unsigned mb) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                   (unsigned)__cvta_generic_to_shared(smem)),
+               "l"(gmem), "r"(bytes), "r"(mb)
+               : "memory");
+}
+__device__ __forceinline__ void bulk_s2g(void* gmem, const void* smem, unsigned bytes) {
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(gmem),
+               "r"((unsigned)__cvta_generic_to_shared(smem)), "r"(bytes)
+               : "memory");
+  asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+}
+
+// TD > 0: hit rows gathered with bulk copies through TD-float shared-memory rows (one row
+// width for every table; dynamic shared memory = 4 warps x 32 rows x TD floats).
+template <int MAXT, int TD>
 __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_constant__ QArgs<MAXT> qa,
                                                                    const __grid_constant__ Dev dv) {
   __shared__ int64_t s_scan[MAXT + 1];
+  __shared__ __align__(8) unsigned long long s_mbar[4];
+  extern __shared__ __align__(128) float kq_dyn[];
   for (int i = threadIdx.x; i <= qa.n; i += blockDim.x) s_scan[i] = qa.scan[i];
+  if constexpr (TD > 0) {
+    if (threadIdx.x < 4) mbar_init((unsigned)__cvta_generic_to_shared(&s_mbar[threadIdx.x]), 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
   pdl_wait();  // the previous batch (or the caller's producer of ids) has completed
   __syncthreads();
 
@@ -647,8 +684,25 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
                      : scr_hash(fk) & dv.scr_mask;
       cur = ld_cg_u64(dv.scratch + h);
     }
+    float* wsm = nullptr;
+    if constexpr (TD > 0) wsm = kq_dyn + (size_t)(threadIdx.x >> 5) * 32 * TD;
+    const unsigned mb = TD > 0 ? (unsigned)__cvta_generic_to_shared(&s_mbar[threadIdx.x >> 5]) : 0u;
     if (!qa.slots) {
-      gather_dispatch(src, dst, d, active, lane);
+      if constexpr (TD > 0) {
+        // hit rows -> this warp's shared-memory block by bulk copies (no registers held while
+        // they fly; the timestamp and dedup atomics below overlap them); invalid IDs -> zero
+        // rows; miss rows are left for KM, which writes them after this grid
+        const unsigned hm0 = __ballot_sync(kFull, hit);
+        if (lane == 0) mbar_expect_tx(mb, (unsigned)__popc(hm0) * 4u * TD);
+        __syncwarp();
+        if (hit) bulk_g2s(wsm + lane * TD, src, 4u * TD, mb);
+        if (active && !valid) {
+#pragma unroll
+          for (int c = 0; c < TD / 4; ++c) reinterpret_cast<float4*>(wsm + lane * TD)[c] = make_float4(0.f, 0.f, 0.f, 0.f);
+        }
+      } else {
+        gather_dispatch(src, dst, d, active, lane);
+      }
     } else if (active) {  // decoupled: KG copies the hits on a side stream while KM fetches misses
       qa.slots[g] = hit ? slot : (miss ? kSlotMiss : kSlotZero);
     }
@@ -745,6 +799,19 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
       if (um) atomicAdd(row + C_UHITS, (unsigned long long)__popc(um));
       if (own_m) atomicAdd(row + C_UMISS, (unsigned long long)__popc(own_m));
       if (dup_m) atomicAdd(row + C_DUPS, (unsigned long long)__popc(dup_m));
+    }
+    if constexpr (TD > 0) {
+      if (!qa.slots) {  // the rows have landed: the warp's output rows leave as one contiguous block
+        mbar_wait(mb, 0);
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // the zero rows, for the bulk store
+        __syncwarp();
+        const unsigned na = (unsigned)__popc(__ballot_sync(kFull, active));  // a prefix of the warp
+        if (lane == 0) {
+          bulk_s2g(qa.out + off, wsm, na * 4u * TD);  // lane 0's row starts the block (uniform rows)
+          asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+        }
+        __syncwarp();
+      }
     }
   }
   pdl_trigger();  // KM may be scheduled now; its pdl_wait still waits for this grid
