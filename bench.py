@@ -52,7 +52,10 @@ def parse():
     p.add_argument("--cpu-seconds", type=float, default=15.0, help="oracle sample budget")
     p.add_argument("--flags", type=int, default=0, help="fleche_config.flags (ablations)")
     p.add_argument("--host-assist", action="store_true",
-                   help="FLECHE_FLAG_HOST_ASSIST: host threads stage the missed rows (paper Fig 8b CPU-DRAM layer)")
+                   help="FLECHE_FLAG_HOST_ASSIST: force the host-assisted miss fetch (paper Fig 8b CPU-DRAM layer); "
+                        "it is on by default for host tiers >= 1 GiB")
+    p.add_argument("--no-host-assist", action="store_true",
+                   help="FLECHE_FLAG_NO_HOST_ASSIST: unified-index zero-copy reads only")
     p.add_argument("--cache-frac", type=float, default=None, help="override the config's cache fraction (sweeps)")
     p.add_argument("--dim", type=int, default=None, help="override every table's row width (sensitivity sweeps)")
     p.add_argument("--batch", type=int, default=None, help="override the samples per table per batch (sweeps)")
@@ -638,6 +641,8 @@ def main():
     if args.prefill is None and args.config.startswith("cfg3"):
         P = PREFILL_CFG3.get(round(w.cache_frac, 2), 360)
     W, K = max(args.warmup, 0), max(args.steps, 1)
+    if args.no_host_assist:
+        args.flags |= 0x20
     if args.host_assist:
         args.flags |= 0x8
         if args.ha_frac is not None:
@@ -679,10 +684,12 @@ def main():
                                                           "restore kernels" if args.p2p else "NCCL all-to-all") + ")"
                              if r["sharded"] else (f"replicated x{world}" if world > 1 else "single GPU"))
         cf["admit_prob"] = args.admit_prob
-        cf["miss_fetch"] = (("host-assisted: %s host threads stage the missed rows (FLECHE_FLAG_HOST_ASSIST)"
-                             % os.environ.get("FLECHE_HA_THREADS", "12")) + ", share %s of the blocks"
-                            % os.environ.get("FLECHE_HA_FRAC", "0.5")) if args.flags & 0x8 else \
-            "unified index: zero-copy reads of the host rows, address-ordered"
+        cf["miss_fetch"] = (("host-assisted split: host threads stage a share of each batch's unique misses "
+                             "(%.0f of %.0f per step, share FLECHE_HA_FRAC=%s), the miss kernel reads the rest "
+                             "zero-copy (unified index)") % (r["assisted_rows_per_step"], r["unique_misses_per_step"],
+                                                            os.environ.get("FLECHE_HA_FRAC", "default"))
+                            if r["assisted_rows_per_step"] > 0 else
+                            "unified index: zero-copy reads of the host rows, address-ordered")
         cf["flags"] = args.flags
         cf["eviction"] = (f"full-scan between watermarks hi={r['wm'][0]} lo={r['wm'][1]} (reading R23)" if r["wm"]
                           else "on demand (canonical, reading R2)")

@@ -106,22 +106,28 @@ typedef struct {
 /* HOST_ASSIST: host-assisted miss fetch -- the paper's decoupled workflow with the
  * CPU-DRAM layer queried "ahead", as soon as the indexing kernel knows which keys miss,
  * in parallel with the GPU's hit copy (Fig 8b; CPU-DRAM layer P:L177-178).
- * The default path is the unified index (Fig 8c): the GPU reads each missed
- * row where it lies in the host tables.  On a host whose IOMMU translation caps scattered
- * zero-copy reads (measured on the graft B200 pool: ~80 M rows/s beyond a ~1 GiB span,
- * DESIGN.md §6) the ctx can instead run host threads that gather the batch's unique
- * missed rows into a contiguous pinned staging buffer, which the miss kernel then reads
- * over the link at its full rate.  Requests travel GPU -> host through pinned memory (no
- * host sync, no extra launch: the query path stays asynchronous and graph-capturable);
- * a block the threads have not staged within FLECHE_HA_TIMEOUT_US (default 2000) is read
- * zero-copy from the tables instead, so correctness never depends on the threads.  Env:
- * FLECHE_HA_THREADS (default 12), FLECHE_HA_STAGE_KB (staging per epoch parity, default
- * 131072; rows beyond it are read zero-copy), FLECHE_HA_FRAC (share of the batch's
- * staging blocks the host threads take, default 0.5, or 0.85 for host tiers over 32 GiB;
- * KM reads the rest zero-copy at the same time), FLECHE_HA_MIN_ROWS (batches with fewer unique misses stay all zero-copy,
- * default 32768: below it the round trip to the host threads is not hidden).  Not with PER_TABLE_LAUNCH (FLECHE_EINVAL).  `out`, hits and every cache decision are identical with and without
- * it; only where the missed rows are read from changes. */
+ * The unified index (Fig 8c) lets the GPU read each missed row where it
+ * lies in the host tables.  On this platform scattered zero-copy reads are capped by
+ * address translation (~80 M rows/s beyond a ~1 GiB span), while host cores
+ * gather scattered rows at ~60 GB/s, so by DEFAULT a ctx whose host tier spans >= 1 GiB
+ * (uniform row width, >= 8 host CPUs) runs host threads that gather a share of the batch's
+ * unique missed rows into a contiguous pinned staging buffer, which the miss kernel reads
+ * over the link at its full rate while it reads the rest zero-copy itself (two paths at
+ * once).  HOST_ASSIST forces it on (also for mixed widths or small tiers),
+ * NO_HOST_ASSIST off.  Requests travel GPU -> host through pinned memory, tagged with the
+ * batch epoch; the query kernel's last CTA rings the doorbell; ONE miss-kernel warp polls
+ * the threads' progress words and mirrors them into HBM for the others (no host sync, no
+ * extra launch: the path stays asynchronous and graph-capturable).  Blocks not staged
+ * within FLECHE_HA_TIMEOUT_US (default 2000) are read zero-copy from the tables, so
+ * correctness never depends on the threads.  Env: FLECHE_HA_THREADS (default
+ * min(12, CPUs - 4)), FLECHE_HA_STAGE_KB (staging per epoch parity, default 131072; rows
+ * beyond it are read zero-copy), FLECHE_HA_FRAC (share of the batch's staging blocks the
+ * host threads take, default 0.8, or 0.85 for host tiers over 32 GiB), FLECHE_HA_MIN_ROWS
+ * (batches with fewer unique misses stay all zero-copy, default 1024).  Not with
+ * PER_TABLE_LAUNCH (FLECHE_EINVAL).  `out`, hits and every cache decision are identical
+ * with and without it; only where the missed rows are read from changes. */
 #define FLECHE_FLAG_HOST_ASSIST 0x8u
+#define FLECHE_FLAG_NO_HOST_ASSIST 0x20u
 /* FUSED_HIT_COPY: the query kernel copies each hit row itself (probe and copy in one
  * kernel, the fused design) instead of the default for uniform layouts with >= 512K
  * lookups per batch: the decoupled copy (Fig 8b), where the query kernel only

@@ -20,6 +20,7 @@ _lib = ctypes.CDLL(LIB_PATH)
 
 OK, EINVAL, ENOMEM, ECUDA, ENCCL, ERANGE, ESTATE = 0, -1, -2, -3, -4, -5, -6
 FLAG_STATIC_PER_TABLE, FLAG_PER_TABLE_LAUNCH, FLAG_HOST_ASSIST, FLAG_FUSED_HIT_COPY = 0x2, 0x4, 0x8, 0x10
+FLAG_NO_HOST_ASSIST = 0x20
 MAX_TABLES = 512
 
 _vp, _i64, _i32, _u64, _u32 = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32, ctypes.c_uint64, ctypes.c_uint32

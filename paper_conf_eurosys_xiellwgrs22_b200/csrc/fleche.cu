@@ -40,9 +40,9 @@ struct HostAssist {
   HaReq* req = nullptr;                // [2][req_cap] (indexed like the miss list)
   HaDesc* desc = nullptr;              // [2]
   unsigned long long* bell = nullptr;  // doorbell (epoch)
-  uint32_t* ready = nullptr;           // [2][blk_cap]
+  unsigned long long* prog = nullptr;  // [2][kHaMaxThreads] progress words (epoch << 32 | blocks staged)
   float* stage = nullptr;              // [2][stage_floats]
-  uint32_t req_cap = 0, blk_cap = 0;
+  uint32_t req_cap = 0;
   bool nt_stores = true;  // FLECHE_HA_NT=0: plain memcpy into the staging buffer (A/B)
   uint64_t delay_ns = 0;  // FLECHE_HA_DELAY_US: fault injection (tests): each block is gathered this late
   uint64_t stage_floats = 0;
@@ -292,11 +292,13 @@ __attribute__((target("avx2"))) void stage_row(float* dst, const float* src, siz
     _mm256_stream_si256((__m256i*)((char*)dst + b), _mm256_loadu_si256((const __m256i*)((const char*)src + b)));
 }
 
-// One host-assist thread: wait for a doorbell, gather this thread's blocks of the
-// batch's requests (block k = miss-list indices [64k, 64k + 64), rows of every width class
-// in it), publish each block's ready flag.  Spins while batches keep coming; after ~2 ms
-// without one it polls every 50 us (an idle ctx burns no core).  No `pause` in the spin:
-// on a KVM guest it can trigger pause-loop exits that deschedule the vCPU.
+// One host-assist thread: wait for a doorbell, gather this thread's blocks of the batch's
+// requests (block k = miss-list indices [64k, 64k + 64), rows of every width class in
+// it, k % nthreads == me, in increasing k) into the staging buffer with non-temporal
+// stores, and publish the progress word (epoch << 32 | blocks done) after each block.
+// Spins while batches keep coming; after ~2 ms without one it polls every 50 us (an idle
+// ctx burns no core).  No `pause` in the spin: on a KVM guest it can trigger pause-loop
+// exits that deschedule the vCPU.
 void ha_worker(HostAssist* h, int me) {
   uint32_t last = 0;
   uint64_t spins = 0;
@@ -327,8 +329,22 @@ void ha_worker(HostAssist* h, int me) {
     if (me < 64) h->exp_t[(e % 64) * 128 + me] = rt();
 #endif
     const int par = e & 1u;
-    const HaDesc d = h->desc[par];
-    if (d.epoch != e) continue;  // the GPU is a full parity cycle ahead: this batch timed out anyway
+    // the descriptor was written without a system fence before the doorbell: re-read until
+    // both epoch fields carry this batch (and a second read agrees), at most ~1 ms
+    HaDesc d;
+    bool got = false;
+    for (uint64_t n = 0; !got; ++n) {
+      memcpy(&d, (const void*)(h->desc + par), sizeof d);
+      __atomic_thread_fence(__ATOMIC_ACQUIRE);
+      HaDesc d2;
+      memcpy(&d2, (const void*)(h->desc + par), sizeof d2);
+      got = d.epoch == e && d.epoch2 == e && !memcmp(&d, &d2, sizeof d);
+      if (!got && (n & 255) == 255 && now_ns() - t_last > 1000000ull) break;
+    }
+    if (!got) continue;  // the GPU moved on (a later batch's doorbell, or a parity cycle ahead)
+    unsigned long long* prog = h->prog + (size_t)par * kHaMaxThreads + me;
+    uint64_t done = 0;
+    __atomic_store_n(prog, ((unsigned long long)e << 32), __ATOMIC_RELEASE);  // this batch, nothing staged yet
     const HaReq* rq = h->req + (size_t)par * h->req_cap;
     float* st = h->stage + (size_t)par * h->stage_floats;
     uint64_t lo_all = ~0ull, hi_all = 0;
@@ -339,52 +355,81 @@ void ha_worker(HostAssist* h, int me) {
       }
     if (hi_all == 0 || hi_all > h->req_cap) continue;
     const uint64_t kcut = d.kcut;  // blocks >= kcut: KM reads them from the tables itself
-    auto src_of = [&](const HaReq& r, int32_t* dim) -> const float* {
-      const int t = (int)(r.tid >> 48);
-      const int64_t id = (int64_t)(r.tid & 0xFFFFFFFFFFFFull);
-      if (r.stage == kNoStage || t >= nt || id >= h->card[t]) return nullptr;  // no room / defensive
+    // a request of this batch (KQ wrote it without a system fence: wait until both halves
+    // carry this batch's tags, read twice so a torn read is never taken); false after ~1 ms
+    auto fetch = [&](uint64_t i, HaReq* out) -> bool {
+      const volatile HaReq* p = rq + i;
+      for (uint64_t n = 0;; ++n) {
+        HaReq a{p->tid, p->stage};
+        if (ha_req_current(a, e)) {
+          HaReq b{p->tid, p->stage};
+          if (b.tid == a.tid && b.stage == a.stage) {
+            *out = a;
+            return true;
+          }
+        }
+        if ((n & 255) == 255 && (h->stop.load(std::memory_order_relaxed) || now_ns() - t_last > 1000000ull))
+          return false;
+      }
+    };
+    bool lost = false;  // a request never arrived: stop publishing (KM times out and reads zero-copy)
+    auto src_of = [&](const HaReq& r, int32_t* dim, uint64_t* so) -> const float* {
+      const int t = (int)(r.tid >> 55);
+      const int64_t id = (int64_t)(r.tid & kReqLow40);
+      *so = r.stage & kReqLow40;
+      if (*so == kReqLow40 || t >= nt || id >= h->card[t]) return nullptr;  // no room / defensive
       *dim = h->dims[t];
-      if (r.stage + (uint64_t)*dim > h->stage_floats) return nullptr;
+      if (*so + (uint64_t)*dim > h->stage_floats) return nullptr;
       return h->host[t] + (size_t)id * (size_t)*dim;
     };
     auto prefetch = [&](uint64_t i) {
+      HaReq r;
       int32_t dd = 0;
-      if (const float* p = src_of(rq[i], &dd))
+      uint64_t so = 0;
+      if (lost || !fetch(i, &r)) {
+        lost = true;
+        return;
+      }
+      if (const float* p = src_of(r, &dd, &so))
         for (int b = 0; b < dd * 4; b += 64) __builtin_prefetch((const char*)p + b, 0, 0);
     };
     const uint64_t kb0 = lo_all / kHaBlock, kb1 = (hi_all - 1) / kHaBlock;
-    for (uint64_t kb = kb0; kb <= kb1 && kb < kcut; ++kb) {
+    for (uint64_t kb = kb0; kb <= kb1 && kb < kcut && !lost; ++kb) {
       if (kb % (uint64_t)h->nthreads != (uint64_t)me) continue;
       if (h->delay_ns) {  // a stalled host thread (tests): its blocks time out on the GPU
         struct timespec ts = {(time_t)(h->delay_ns / 1000000000ull), (long)(h->delay_ns % 1000000000ull)};
         nanosleep(&ts, nullptr);
       }
-      bool any = false;
       for (int c = 0; c < 8; ++c) {  // the rows of every class region that overlaps block kb
         if (!d.cnt[c]) continue;
         const uint64_t lo = std::max<uint64_t>(kb * kHaBlock, d.off[c]);
         const uint64_t hi = std::min<uint64_t>(kb * kHaBlock + kHaBlock, (uint64_t)d.off[c] + d.cnt[c]);
         if (lo >= hi) continue;
-        any = true;
-        constexpr uint64_t PF = 8;  // rows prefetched ahead
+        constexpr uint64_t PF = 12;  // rows prefetched ahead (~4 lines each: keeps the line fill buffers busy)
         for (uint64_t i = lo; i < std::min(hi, lo + PF); ++i) prefetch(i);
         for (uint64_t i = lo; i < hi; ++i) {
           if (i + PF < hi) prefetch(i + PF);
-          const HaReq r = rq[i];
+          HaReq r;
+          if (lost || !fetch(i, &r)) {  // never arrived: abandon the batch (KM's poller times out)
+            lost = true;
+            break;
+          }
           int32_t dd = 0;
-          if (const float* p = src_of(r, &dd)) {
+          uint64_t so = 0;
+          if (const float* p = src_of(r, &dd, &so)) {
 #ifdef FLECHE_EXPERIMENTS
             if (h->exp_nogather) continue;  // timing experiment: publish without gathering (wrong rows)
 #endif
-            if (h->nt_stores) stage_row(st + r.stage, p, (size_t)dd * 4u);
-            else memcpy(st + r.stage, p, (size_t)dd * 4u);
+            if (h->nt_stores) stage_row(st + so, p, (size_t)dd * 4u);
+            else memcpy(st + so, p, (size_t)dd * 4u);
           }
         }
       }
-      if (h->nt_stores) _mm_sfence();  // streaming stores are weakly ordered: drain them before the flag
-      if (any) __atomic_store_n(h->ready + (size_t)par * h->blk_cap + kb, e, __ATOMIC_RELEASE);
+      if (h->nt_stores) _mm_sfence();  // streaming stores are weakly ordered: drain them before the progress word
+      if (lost) break;
+      __atomic_store_n(prog, ((unsigned long long)e << 32) | ++done, __ATOMIC_RELEASE);
 #ifdef FLECHE_EXPERIMENTS
-      if (any && h->exp_pub) {
+      if (h->exp_pub) {
         struct timespec ts;
         clock_gettime(CLOCK_REALTIME, &ts);
         h->exp_pub[kb] = (uint64_t)ts.tv_sec * 1000000000ull + (uint64_t)ts.tv_nsec;
@@ -417,7 +462,7 @@ void free_all(fleche_ctx* c) {
                   c->dv.miss, c->dv.dup, c->dv.ctl, c->dv.stats, c->d_tables, c->d_ids_stage, c->d_out_stage,
                   c->d_pool_stage, c->d_kdec, c->rd.scratch, c->rd.slotval, c->rd.inv, c->rd.region, c->rd.cnt,
                   c->rd.prefix, c->rd.done, c->rd.stats, c->d_slots, c->d_age_hist, c->d_prefill_out,
-                  c->d_out_stage2};
+                  c->d_out_stage2, c->dv.ha_seen};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   for (auto& r : c->registered) cudaHostUnregister(r.first);
@@ -555,6 +600,11 @@ fleche_status launch_query(fleche_ctx* c, const int64_t* const* ids, const int64
   // small batches: the fork/join costs more than the overlap saves (cfg1 measured +5 %)
   const bool decouple = c->decoupled && total >= c->decouple_min && !c->per_table_launch;
   if (decouple) qa.slots = c->d_slots;
+  // host-assisted: KQ's last CTA rings the host threads' doorbell (FLECHE_HA_BELL=km: KM does)
+  static const bool bell_km = getenv("FLECHE_HA_BELL") && !strcmp(getenv("FLECHE_HA_BELL"), "km");
+  qa.ha_bell = c->dv.ha && !bell_km;
+  ka.bell = c->dv.ha && bell_km;
+  qa.ncls = ka.ncls;
   if (total > 0 && !c->per_table_launch) {
     const int64_t blocks = (total + 127) / 128;
     launch_k(kPdlKQ, kq_fn<MAXT>(c->kq_tma), (unsigned)blocks, 128, c->kq_smem, s, qa, c->dv);
@@ -672,10 +722,12 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   const int n = cfg->num_tables;
   if (n < 1 || n > FLECHE_MAX_TABLES || !cfg->cardinalities || !cfg->dims || !cfg->host_tables) return FLECHE_EINVAL;
   const uint32_t known = FLECHE_FLAG_STATIC_PER_TABLE | FLECHE_FLAG_PER_TABLE_LAUNCH |
-                         FLECHE_FLAG_HOST_ASSIST | FLECHE_FLAG_FUSED_HIT_COPY;
+                         FLECHE_FLAG_HOST_ASSIST | FLECHE_FLAG_FUSED_HIT_COPY | FLECHE_FLAG_NO_HOST_ASSIST;
   if (cfg->max_lookups < 1 || cfg->max_lookups > (int64_t(1) << 31) || (cfg->flags & ~known) || cfg->reserved)
     return FLECHE_EINVAL;
-  if ((cfg->flags & FLECHE_FLAG_HOST_ASSIST) && (cfg->flags & FLECHE_FLAG_PER_TABLE_LAUNCH)) return FLECHE_EINVAL;
+  if ((cfg->flags & FLECHE_FLAG_HOST_ASSIST) &&
+      (cfg->flags & (FLECHE_FLAG_PER_TABLE_LAUNCH | FLECHE_FLAG_NO_HOST_ASSIST)))
+    return FLECHE_EINVAL;
   for (int t = 0; t < n; ++t) {
     if (cfg->cardinalities[t] < 1 || !valid_dim(cfg->dims[t])) return FLECHE_EINVAL;
     if (!cfg->host_tables[t] || ((uintptr_t)cfg->host_tables[t] & 15u)) return FLECHE_EINVAL;
@@ -849,8 +901,15 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   if (cudaEventCreateWithFlags(&c->chain_ev, cudaEventDisableTiming) != cudaSuccess) return fail(FLECHE_ECUDA);
   // KM: enough warps for the expected unique misses, km_bps CTAs of 4 warps per SM, and no
   // more CTAs than fit at once (cooperative launch: its grid barrier needs them all resident)
-  c->km_smem = (size_t)kKmWarps * ((bytes ? kKmSmemF4 : 0) + ((cfg->flags & FLECHE_FLAG_HOST_ASSIST) ? kHaSmemF4 : 0)) *
-               sizeof(float4);
+  // host-assisted miss fetch: forced by the flag, else by default on a large host tier
+  // (the translation-bound regime of scattered zero-copy reads) with uniform rows
+  uint64_t tier_bytes = 0;
+  for (int t = 0; t < n; ++t) tier_bytes += (uint64_t)c->card[t] * (uint64_t)c->dims[t] * 4u;
+  const unsigned ncpu = std::thread::hardware_concurrency();
+  const bool use_ha = (cfg->flags & FLECHE_FLAG_HOST_ASSIST) ||
+                      (!(cfg->flags & FLECHE_FLAG_NO_HOST_ASSIST) && !bytes && !part && !c->per_table_launch &&
+                       tier_bytes >= (1ull << 30) && ncpu >= 8 && !(getenv("FLECHE_HA") && !atoi(getenv("FLECHE_HA"))));
+  c->km_smem = (size_t)kKmWarps * ((bytes ? kKmSmemF4 : 0) + (use_ha ? kHaSmemF4 : 0)) * sizeof(float4);
   {
     const void* km = (const void*)km_fn(bytes, c->cls_dim.size() == 1 ? c->max_dim : 0);
     if (c->km_smem > 48 * 1024 &&
@@ -881,19 +940,19 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
         cudaMalloc((void**)&c->d_slots, (size_t)cfg->max_lookups * 4) != cudaSuccess)
       return fail(FLECHE_ENOMEM);
   }
-  if (cfg->flags & FLECHE_FLAG_HOST_ASSIST) {
+  if (use_ha) {
     HostAssist* h = c->ha = new (std::nothrow) HostAssist();
     if (!h) return fail(FLECHE_ENOMEM);
     auto env_u = [](const char* k, uint64_t dflt) {
       const char* e = getenv(k);
       return e ? strtoull(e, nullptr, 10) : dflt;
     };
-    h->nthreads = (int)std::max<uint64_t>(1, std::min<uint64_t>(64, env_u("FLECHE_HA_THREADS", 12)));
+    h->nthreads = (int)std::max<uint64_t>(
+        1, std::min<uint64_t>(kHaMaxThreads, env_u("FLECHE_HA_THREADS", std::max(1u, std::min(12u, ncpu > 4 ? ncpu - 4 : 1)))));
     h->req_cap = (uint32_t)cfg->max_lookups;  // requests are indexed like the miss list
-    h->blk_cap = h->req_cap / kHaBlock + 2;
     h->stage_floats = std::max<uint64_t>(1024, env_u("FLECHE_HA_STAGE_KB", 131072) << 8);
     const size_t o_req = 0, o_desc = o_req + 2 * sizeof(HaReq) * (size_t)h->req_cap, o_bell = o_desc + 2 * sizeof(HaDesc),
-                 o_ready = (o_bell + 8 + 63) & ~size_t(63), o_stage = (o_ready + 8ull * h->blk_cap + 255) & ~size_t(255),
+                 o_prog = (o_bell + 8 + 127) & ~size_t(127), o_stage = (o_prog + 16ull * kHaMaxThreads + 255) & ~size_t(255),
                  total = o_stage + 2 * 4 * h->stage_floats;
     if (cudaHostAlloc(&h->mem, total, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess) {
       cudaGetLastError();
@@ -905,7 +964,7 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
     h->req = (HaReq*)(b + o_req);
     h->desc = (HaDesc*)(b + o_desc);
     h->bell = (unsigned long long*)(b + o_bell);
-    h->ready = (uint32_t*)(b + o_ready);
+    h->prog = (unsigned long long*)(b + o_prog);
     h->stage = (float*)(b + o_stage);
     void* dmem = nullptr;
     if (cudaHostGetDevicePointer(&dmem, h->mem, 0) != cudaSuccess) return fail(FLECHE_ECUDA);
@@ -914,22 +973,25 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
     dv.ha_req = (HaReq*)(db + o_req);
     dv.ha_desc = (HaDesc*)(db + o_desc);
     dv.ha_bell = (unsigned long long*)(db + o_bell);
-    dv.ha_ready = (uint32_t*)(db + o_ready);
+    dv.ha_prog = (unsigned long long*)(db + o_prog);
+    dv.ha_threads = (uint32_t)h->nthreads;
+    if (cudaMalloc((void**)&dv.ha_seen, 8 * kHaMaxThreads) != cudaSuccess ||
+        cudaMemset(dv.ha_seen, 0, 8 * kHaMaxThreads) != cudaSuccess)
+      return fail(FLECHE_ENOMEM);
     dv.ha_stage = (float*)(db + o_stage);
     dv.ha_req_cap = h->req_cap;
-    dv.ha_blk_cap = h->blk_cap;
     dv.ha_stage_floats = h->stage_floats;
     dv.ha_timeout_ns = env_u("FLECHE_HA_TIMEOUT_US", 2000) * 1000ull;
     {  // share of the staging blocks the host threads gather (the rest: KM's zero-copy reads)
       // default share: the host threads' share pays off more the larger the host tier (the
-      // GPU's translated reads slow down with the span): measured best ~0.5-0.6 at 8.6 GB
-      // (cfg5), >= 0.85 at 113 GB (cfg3h); profiles/bench_r01_*ha*.json
+      // GPU's translated reads slow down with the span): measured best 0.7-0.8 at 8.6 GB
+      // (cfg2, cfg5; profiles/bench_r02_ha_*.json), >= 0.85 at 113 GB (cfg3h, round 1)
       uint64_t span = 0;
       for (int t = 0; t < n; ++t) span += (uint64_t)c->card[t] * (uint64_t)c->dims[t] * 4u;
       const char* e = getenv("FLECHE_HA_FRAC");
-      const double f = e ? std::min(1.0, std::max(0.0, atof(e))) : (span > (32ull << 30) ? 0.85 : 0.5);
+      const double f = e ? std::min(1.0, std::max(0.0, atof(e))) : (span > (32ull << 30) ? 0.85 : 0.8);
       dv.ha_frac_q16 = (uint32_t)(f * 65536.0 + 0.5);
-      dv.ha_min_rows = (uint32_t)env_u("FLECHE_HA_MIN_ROWS", 32768);
+      dv.ha_min_rows = (uint32_t)env_u("FLECHE_HA_MIN_ROWS", 1024);
     }
     h->nt_stores = env_u("FLECHE_HA_NT", 1) != 0 && __builtin_cpu_supports("avx2");
     h->delay_ns = env_u("FLECHE_HA_DELAY_US", 0) * 1000ull;
@@ -943,9 +1005,9 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   cudaMemset(dv.exp_buf, 0, ((size_t)c->km_blocks * 4 * 4 + 8) * 8);
   dv.exp_slots = (uint32_t)c->km_blocks * 16;
   if (c->ha) {
-    if (cudaMalloc((void**)&dv.exp_blk, ((size_t)c->ha->blk_cap * 4) * 8) != cudaSuccess) return fail(FLECHE_ENOMEM);
-    cudaMemset(dv.exp_blk, 0, ((size_t)c->ha->blk_cap * 4) * 8);
-    c->ha->exp_pub = new uint64_t[c->ha->blk_cap]();
+    if (cudaMalloc((void**)&dv.exp_blk, ((size_t)(c->ha->req_cap / kHaBlock + 2) * 4) * 8) != cudaSuccess) return fail(FLECHE_ENOMEM);
+    cudaMemset(dv.exp_blk, 0, ((size_t)(c->ha->req_cap / kHaBlock + 2) * 4) * 8);
+    c->ha->exp_pub = new uint64_t[(c->ha->req_cap / kHaBlock + 2)]();
   }
 #endif
   if (cudaDeviceSynchronize() != cudaSuccess) return fail(FLECHE_ECUDA);
@@ -1688,7 +1750,7 @@ extern "C" __attribute__((visibility("default"))) fleche_status fleche_exp_ha_bl
                                                                                      size_t nblk) {
   if (!c || !host || !c->ha) return FLECHE_EINVAL;
   if (c->have_last) cudaStreamSynchronize(c->last_stream);
-  const size_t m = std::min(nblk, (size_t)c->ha->blk_cap);
+  const size_t m = std::min(nblk, (size_t)(c->ha->req_cap / kHaBlock + 2));
   std::vector<uint64_t> g(m * 4);
   if (cudaMemcpy(g.data(), c->dv.exp_blk, m * 4 * 8, cudaMemcpyDeviceToHost) != cudaSuccess) return FLECHE_ECUDA;
   for (size_t k = 0; k < m; ++k) {

@@ -58,7 +58,8 @@ constexpr uint32_t kSlotMiss = 0xFFFFFFFFu, kSlotZero = 0xFFFFFFFEu;  // KQ -> K
 constexpr int kKmWarps = 4;     // KM CTA = 4 warps
 constexpr int kKmStageF4 = 256; // bytes layout, per warp: staged rows of a chunk (<= 4 KB) ...
 constexpr int kKmSmemF4 = 512;  // ... + the compaction buffer of one set region (<= 4 KB)
-constexpr int kHaBlock = 64;    // host-assisted miss fetch: rows per staging block (one ready flag)
+constexpr int kHaBlock = 64;    // host-assisted miss fetch: rows per staging block
+constexpr int kHaMaxThreads = 16;  // host-assisted: at most this many host threads (one progress word each)
 constexpr int kHaSmemF4 = 512;  // host-assisted KM, per warp: 8 KB of rows landed from the host (4 KM CTAs per SM)
 
 enum Ctr : int {
@@ -122,35 +123,51 @@ struct Ctl {
   uint32_t done;   // KM grid barrier arrivals (before the restore)
   uint32_t done2;  // KM CTA arrivals at the end (the last one closes the batch)
   uint32_t err_invalid;
-  uint32_t ha_rung;  // host-assisted: epoch whose doorbell KM has rung (warps poll host flags after it)
+  uint32_t ha_rung;  // host-assisted: epoch whose doorbell KQ's last CTA has rung
   uint32_t counts[2][8];  // [epoch & 1][class 0..5: unique misses; 7: duplicate misses]
   long long occ_bytes;    // row bytes currently cached
   uint32_t ke_done;       // watermark eviction: KE2 CTA arrival counter
   uint32_t km_bar;        // KM grid barrier: epoch whose owner rows are all in `out`
-  long long ke_occ;       // watermark eviction: occ_bytes as KE1 saw it (KE2's one snapshot per scan)
+  long long ke_occ;
+  uint32_t kq_done;       // host-assisted: KQ CTA arrivals (the last one rings the doorbell)
+  uint32_t ha_abort;      // host-assisted: epoch whose staging the poller gave up on (timeout)       // watermark eviction: occ_bytes as KE1 saw it (KE2's one snapshot per scan)
 };
 
-// Host-assisted miss fetch (FLECHE_FLAG_HOST_ASSIST).  The owner lane of each unique
-// miss in KQ writes (table, row, staging slot) to the request list in pinned host memory
-// at the miss's own miss-list index; KM's first thread rings a doorbell with the batch's
-// per-width miss counts (KQ's writes are complete by then: stream order).  Host threads gather the
-// requested rows into the contiguous pinned staging buffer, kHaBlock list indices at a
-// time, and publish a ready flag (= epoch) per block.  KM then takes whole blocks, waits
-// for each block's flag once and reads its staged rows (contiguous zero-copy: no per-row
-// address translation on the host link, the limit of the plain unified index on this
-// platform) instead of the scattered table rows.  A block not ready within the timeout
-// is fetched zero-copy from the tables as in the plain path, so a missing or slow host
-// thread costs time, never correctness.  Every area is double-buffered by epoch parity.
-struct HaReq {             // one request: (table << 48 | row), float offset of its staging slot
-  unsigned long long tid;
-  unsigned long long stage;  // kNoStage: no staging room this batch (KM reads the table row)
+// Host-assisted miss fetch (FLECHE_FLAG_HOST_ASSIST): the CPU-DRAM layer's threads
+// gather missed rows (Fig 8b) -- host cores read scattered rows without the
+// GPU's address-translation limit on scattered zero-copy reads (profiles/), and the GPU
+// then reads their staging buffer contiguously.  The owner lane of each unique miss in KQ
+// writes (table, row, staging slot) to the request list in pinned host memory at its
+// miss-list index; KQ's last CTA rings a doorbell with the batch's per-width miss counts.
+// Host thread i gathers every staging block k (kHaBlock list indices) with k % T == i,
+// in increasing k, and after each block publishes its progress word (epoch << 32 |
+// blocks done; all T words share two cache lines).  ONE poller warp of KM reads those
+// words over the link and mirrors them into HBM; every other KM warp waits on the mirror
+// for its block (no per-block polls competing with the row reads for the link), then
+// reads the block's staged rows.  Past the timeout the poller gives up and the readers
+// fetch the rows zero-copy from the tables, so a missing or slow host thread costs time,
+// never correctness.  Every area is double-buffered by epoch parity.
+struct HaReq {  // one request, both halves tagged with the batch epoch (see ha_req_make)
+  unsigned long long tid;    // table (9 bits) << 55 | epoch (15 bits) << 40 | row (40 bits)
+  unsigned long long stage;  // epoch (24 bits) << 40 | float offset of its staging slot (40 bits; all ones: none)
 };
-struct HaDesc {            // written by KM's first thread, read by the host threads
+constexpr unsigned long long kReqLow40 = (1ull << 40) - 1;
+// KQ writes a request with one 16-byte store and no system fence: the host thread that
+// reads it after the doorbell re-reads until both halves carry the batch's epoch tags, so a
+// request still in flight over the link (or a torn read) is never taken for this batch's.
+__host__ __device__ __forceinline__ HaReq ha_req_make(int t, int64_t id, uint64_t stage, uint32_t epoch) {
+  return HaReq{((unsigned long long)t << 55) | ((unsigned long long)(epoch & 0x7FFFu) << 40) | ((uint64_t)id & kReqLow40),
+               ((unsigned long long)(epoch & 0xFFFFFFu) << 40) | (stage & kReqLow40)};
+}
+__host__ __device__ __forceinline__ bool ha_req_current(const HaReq& r, uint32_t epoch) {
+  return (uint32_t)((r.tid >> 40) & 0x7FFFu) == (epoch & 0x7FFFu) && (uint32_t)(r.stage >> 40) == (epoch & 0xFFFFFFu);
+}
+struct HaDesc {            // written by the doorbell ringer, read by the host threads
   uint32_t epoch;
   uint32_t cnt[8];         // unique misses of width class c (list indices off[c] .. off[c] + cnt[c])
   uint32_t off[8];
   uint32_t kcut;           // split: the host threads stage blocks < kcut, KM reads blocks >= kcut itself
-  uint32_t pad;
+  uint32_t epoch2;         // = epoch, written last: the host accepts the descriptor once both match
 };
 
 struct Dev {
@@ -188,9 +205,10 @@ struct Dev {
   HaReq* ha_req;               // [2][ha_req_cap]: indexed like the miss list
   HaDesc* ha_desc;             // [2]
   unsigned long long* ha_bell; // doorbell: epoch of the latest published descriptor
-  uint32_t* ha_ready;          // [2][ha_blk_cap] epoch of the block's staged rows
+  unsigned long long* ha_prog; // [2][kHaMaxThreads] (host memory) thread i's progress: epoch << 32 | blocks staged
+  unsigned long long* ha_seen; // [kHaMaxThreads] (HBM) the poller warp's mirror of ha_prog[epoch & 1]
   float* ha_stage;             // [2][ha_stage_floats]
-  uint32_t ha_req_cap, ha_blk_cap;
+  uint32_t ha_req_cap, ha_threads;
   uint64_t ha_stage_floats;
   uint64_t ha_timeout_ns;
   uint32_t ha_frac_q16;        // share of the batch's staging blocks given to the host threads (x 2^-16)
@@ -219,6 +237,8 @@ struct QArgs {
   int32_t n;
   int32_t t0;                // first table of this launch (per-table launches: t0 = t, n = 1)
   int32_t fkseg;             // key-sharded fused exchange: fkeys come in n segments (ids[], scan[])
+  int32_t ha_bell;           // host-assisted: the last CTA rings the host threads' doorbell
+  int32_t ncls;              //   (number of width classes of the miss list)
 };
 
 struct KMArgs {
@@ -226,6 +246,7 @@ struct KMArgs {
   int64_t cls_off[8];
   int32_t cls_dim[8];
   int32_t ncls;
+  int32_t bell;  // host-assisted: KM (not KQ's last CTA) rings the doorbell
 };
 
 template <int MAXT>
@@ -345,22 +366,98 @@ __device__ __forceinline__ uint32_t ld_cv_u32(const uint32_t* p) {
   asm volatile("ld.global.cv.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
   return v;
 }
-// Wait (one lane) until a staging block carries this batch's epoch; false after timeout_ns.
-// First waits (in device memory) for KM's doorbell, so no host poll is in flight while the
-// doorbell's system fence drains; then polls the host flag (.cv loads) and takes one
-// acquire load once it matches.
-__device__ __forceinline__ bool ha_wait_block(const uint32_t* flag, const uint32_t* rung, uint32_t epoch,
-                                              unsigned long long timeout_ns) {
+// Grid barrier helpers (KM is a cooperative launch: every CTA is resident at once).
+__device__ __forceinline__ uint32_t ld_acquire_gpu_u32(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_gpu_u32(uint32_t* p, uint32_t v) {
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+__device__ __forceinline__ unsigned long long ld_acquire_sys_u64(const unsigned long long* p) {
+  unsigned long long v;
+  asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ unsigned long long ld_cv_u64(const unsigned long long* p) {
+  unsigned long long v;
+  asm volatile("ld.global.cv.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ unsigned long long ld_acquire_gpu_u64(const unsigned long long* p) {
+  unsigned long long v;
+  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_gpu_u64(unsigned long long* p, unsigned long long v) {
+  asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+// Host-assisted geometry of a batch: staging blocks [kb0, kend) go to the host threads
+// (kend = the split point kcut, clipped to the batch's last block + 1).
+__device__ __forceinline__ void ha_range(const Dev& dv, const uint32_t* cnt, const int64_t* cls_off, int ncls,
+                                         uint32_t& kb0, uint32_t& kb1) {
+  uint32_t lo = 0xFFFFFFFFu, hi = 0;
+  for (int c = 0; c < ncls; ++c) {
+    if (!cnt[c]) continue;
+    lo = min(lo, (uint32_t)cls_off[c]);
+    hi = max(hi, (uint32_t)cls_off[c] + cnt[c]);
+  }
+  kb0 = hi ? lo / kHaBlock : 0u;
+  kb1 = hi ? (hi - 1) / kHaBlock : 0u;
+}
+
+// The poller warp (lane i < T: host thread i): mirror the host threads' progress words
+// into HBM until every thread has staged its share of [kb0, kend), or give up after the
+// timeout (ha_abort = epoch: the readers then fetch the rest zero-copy).
+__device__ __forceinline__ void ha_poll(const Dev& dv, uint32_t epoch, uint32_t kb0, uint32_t kend, int lane) {
+  const int T = (int)dv.ha_threads;
+  const unsigned long long* prog = dv.ha_prog + (size_t)(epoch & 1u) * kHaMaxThreads;
+  uint32_t quota = 0;
+  if (lane < T && kend > kb0) {
+    const uint32_t first = kb0 + (uint32_t)((lane - (int)(kb0 % (uint32_t)T) + T) % T);
+    quota = first < kend ? (kend - 1 - first) / (uint32_t)T + 1u : 0u;
+  }
+  unsigned long long last = 0;
   const unsigned long long t0 = globaltimer_ns();
-  while (*(const volatile uint32_t*)rung != epoch) {
-    __nanosleep(200);
-    if (globaltimer_ns() - t0 > timeout_ns) return false;
+  while (true) {
+    bool done = true;
+    if (lane < T) {
+      unsigned long long v = ld_cv_u64(prog + lane);
+      if ((uint32_t)(v >> 32) == epoch) {
+        if (v != last) {
+          v = ld_acquire_sys_u64(prog + lane);  // orders the staged rows before the mirror
+          st_release_gpu_u64(dv.ha_seen + lane, v);
+          last = v;
+        }
+        done = (uint32_t)v >= quota;
+      } else {
+        done = quota == 0;
+      }
+    }
+    if (__all_sync(kFull, done)) break;
+    if (globaltimer_ns() - t0 > dv.ha_timeout_ns) {
+      if (lane == 0) st_release_gpu_u32(&dv.ctl->ha_abort, epoch);
+      break;
+    }
   }
-  while (ld_cv_u32(flag) != epoch) {
-    __nanosleep(500);  // each poll is a host-link round trip: one poller per block
-    if (globaltimer_ns() - t0 > timeout_ns) return false;
+}
+
+// A reader warp's wait (one lane) for staging block kb; false: timed out / abandoned.
+__device__ __forceinline__ bool ha_wait_block(const Dev& dv, uint32_t epoch, uint32_t kb0, uint32_t kb) {
+  const uint32_t T = dv.ha_threads, i = kb % T;
+  const uint32_t first = kb0 + (i + T - kb0 % T) % T;
+  const uint32_t need = (kb - first) / T + 1u;
+  const unsigned long long t0 = globaltimer_ns();
+  while (true) {
+    const unsigned long long v = ld_acquire_gpu_u64(dv.ha_seen + i);
+    if ((uint32_t)(v >> 32) == epoch && (uint32_t)v >= need) return true;
+    if (*(volatile uint32_t*)&dv.ctl->ha_abort == epoch) return false;
+    if (globaltimer_ns() - t0 > dv.ha_timeout_ns + 20000ull) return false;  // safety net behind the poller's
+    __nanosleep(64);
   }
-  return ld_acquire_sys_u32(flag) == epoch;
 }
 
 // Host-assisted split: the batch's miss list spans staging blocks [kb0, kb1]; the host
@@ -767,8 +864,12 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
         if (dv.exp_mode != 4)
 #endif
         if (dv.ha)  // published by KM's doorbell (after this grid completes)
-          dv.ha_req[(size_t)par * dv.ha_req_cap + li] =
-              HaReq{((unsigned long long)(qa.t0 + t) << 48) | (unsigned long long)id, hst};
+        {
+          const HaReq rq = ha_req_make(qa.t0 + t, id, hst, epoch);
+          asm volatile("st.global.v2.u64 [%0], {%1, %2};" ::"l"(dv.ha_req + (size_t)par * dv.ha_req_cap + li),
+                       "l"(rq.tid), "l"(rq.stage)
+                       : "memory");
+        }
       }
     }
     if (dup_m) {
@@ -811,6 +912,42 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
           asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
         }
         __syncwarp();
+      }
+    }
+  }
+  if (qa.ha_bell) {
+    // host-assisted fetch: the last CTA rings the doorbell once every CTA has counted its
+    // misses (one KM launch earlier than KM could).  No system fence per CTA: the requests
+    // carry epoch tags and the host threads wait for them (ha_req_current).
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      __threadfence();
+      const uint32_t prev = atomicAdd(&dv.ctl->kq_done, 1u);
+      if (prev == gridDim.x - 1) {
+        __threadfence();
+        dv.ctl->kq_done = 0;
+        const uint32_t epoch = *(volatile uint32_t*)&dv.ctl->epoch;
+        const int par = epoch & 1u;
+        uint32_t cnt[8], total = 0;
+        for (int c = 0; c < 8; ++c) {
+          cnt[c] = c < qa.ncls ? *(volatile uint32_t*)&dv.ctl->counts[par][c] : 0u;
+          total += cnt[c];
+        }
+        if (dv.ha_frac_q16 && total >= dv.ha_min_rows) {  // KM's ha_active() takes the same decision
+          uint32_t kb0, kb1;
+          ha_range(dv, cnt, qa.cls_off, qa.ncls, kb0, kb1);
+          HaDesc hd;
+          hd.epoch = epoch;
+          for (int c = 0; c < 8; ++c) {
+            hd.cnt[c] = cnt[c];
+            hd.off[c] = c < qa.ncls ? (uint32_t)qa.cls_off[c] : 0u;
+          }
+          hd.kcut = kb0 + (uint32_t)(((unsigned long long)(kb1 - kb0 + 1u) * dv.ha_frac_q16 + 65535ull) >> 16);
+          hd.epoch2 = epoch;
+          dv.ha_desc[par] = hd;  // no system fence: the host re-reads until both epoch fields match
+          asm volatile("st.relaxed.sys.global.u64 [%0], %1;" ::"l"(dv.ha_bell), "l"((unsigned long long)epoch) : "memory");
+          *(volatile uint32_t*)&dv.ctl->ha_rung = epoch;
+        }
       }
     }
   }
@@ -1033,14 +1170,14 @@ template <bool BYTES, int D>
 __device__ __forceinline__ void km_ha(const Dev& dv, float* __restrict__ out, const MissRec* __restrict__ mlist,
                                       uint32_t epoch, uint32_t nmiss, int lane, uint32_t gw, uint32_t nw, unsigned& ins,
                                       unsigned& ev, unsigned& byp, long long& docc, unsigned long long& hostb,
-                                      float4* hsm, float4* cbuf, unsigned& harows, unsigned& hato, uint32_t kcut) {
+                                      float4* hsm, float4* cbuf, unsigned& harows, unsigned& hato, uint32_t kcut,
+                                      uint32_t bkb0) {
   constexpr int VEC = D / 4;
   constexpr int ROWS = (kHaSmemF4 / VEC) < kHaBlock ? (kHaSmemF4 / VEC) : kHaBlock;  // rows per piece
   constexpr int PER_LANE = ROWS * VEC / 32;  // float4 per lane per piece
   constexpr int INFL = PER_LANE < 16 ? PER_LANE : 16;
   const uint32_t off = (uint32_t)(mlist - dv.miss);
   const uint32_t kb0 = off / kHaBlock, kb1 = (off + nmiss - 1) / kHaBlock;
-  const uint32_t* flags = dv.ha_ready + (size_t)(epoch & 1u) * dv.ha_blk_cap;
   const float* stage = dv.ha_stage + (size_t)(epoch & 1u) * dv.ha_stage_floats;
   for (uint32_t kb = kb0 + gw; kb <= kb1; kb += nw) {
     int ok = 0;
@@ -1048,7 +1185,7 @@ __device__ __forceinline__ void km_ha(const Dev& dv, float* __restrict__ out, co
     if (dv.exp_blk && lane == 0) dv.exp_blk[kb * 4 + 0] = globaltimer_ns();
 #endif
     if (lane == 0 && kb < kcut) {  // the host threads' share; blocks >= kcut are read from the tables
-      ok = ha_wait_block(flags + kb, &dv.ctl->ha_rung, epoch, dv.ha_timeout_ns);
+      ok = ha_wait_block(dv, epoch, bkb0, kb);
       if (!ok) ++hato;
     }
 #ifdef FLECHE_EXPERIMENTS
@@ -1343,16 +1480,6 @@ struct KmM {
   static constexpr int value = D >= 256 ? 4 : (BYTES || D >= 64 ? 8 : 16);
 };
 
-// Grid barrier helpers (KM is a cooperative launch: every CTA is resident at once).
-__device__ __forceinline__ uint32_t ld_acquire_gpu_u32(const uint32_t* p) {
-  uint32_t v;
-  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-  return v;
-}
-__device__ __forceinline__ void st_release_gpu_u32(uint32_t* p, uint32_t v) {
-  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
-}
-
 // DU > 0: uniform layout of width DU (one class); DU = 0: every width class in turn.
 template <bool BYTES, int DU>
 __global__ void __launch_bounds__(128, 4) km_kernel(const __grid_constant__ Dev dv, const __grid_constant__ KMArgs ka) {
@@ -1364,30 +1491,30 @@ __global__ void __launch_bounds__(128, 4) km_kernel(const __grid_constant__ Dev 
   const uint32_t epoch = *(volatile uint32_t*)&dv.ctl->epoch;
   const int par = epoch & 1u;
   const int lane = threadIdx.x & 31;
-  const bool use_ha = ha_active(dv, ka, par);
-  if (use_ha && blockIdx.x == 0 && threadIdx.x == 0) {
-    // host-assisted: ring the doorbell.  KQ (the previous grid in stream order) wrote the
-    // requests; this fence orders them before the doorbell for the host threads.
+  const bool use_ha = ha_active(dv, ka, par);  // KQ's last CTA rang the doorbell (same test)
+  if (use_ha && ka.bell && blockIdx.x == 0 && threadIdx.x == 0) {
+    // doorbell from KM (ctx option): KQ's request writes completed with its grid
+    uint32_t cnt[8];
+    for (int c = 0; c < 8; ++c) cnt[c] = c < ka.ncls ? *(volatile uint32_t*)&dv.ctl->counts[par][c] : 0u;
+    uint32_t kb0, kb1;
+    ha_range(dv, cnt, ka.cls_off, ka.ncls, kb0, kb1);
     HaDesc hd;
     hd.epoch = epoch;
-#pragma unroll
     for (int c = 0; c < 8; ++c) {
-      hd.cnt[c] = c < ka.ncls ? *(volatile uint32_t*)&dv.ctl->counts[par][c] : 0u;
+      hd.cnt[c] = cnt[c];
       hd.off[c] = c < ka.ncls ? (uint32_t)ka.cls_off[c] : 0u;
     }
     hd.kcut = ha_kcut(dv, ka, par);
+    hd.epoch2 = epoch;
     dv.ha_desc[par] = hd;
-    __threadfence_system();  // before any warp polls the host (a system fence drains link traffic)
+    __threadfence_system();
     st_release_sys_u64(dv.ha_bell, (unsigned long long)epoch);
     *(volatile uint32_t*)&dv.ctl->ha_rung = epoch;
-#ifdef FLECHE_EXPERIMENTS
-    if (dv.exp_buf) dv.exp_buf[dv.exp_slots] = globaltimer_ns();
-#endif
   }
   // block-interleaved warp numbering: consecutive miss chunks land on different SMs,
   // so the host-link loads of a batch are spread over the whole GPU
-  const uint32_t gw = (threadIdx.x >> 5) * gridDim.x + blockIdx.x;
-  const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
+  uint32_t gw = (threadIdx.x >> 5) * gridDim.x + blockIdx.x;
+  uint32_t nw = (gridDim.x * blockDim.x) >> 5;
   // per warp: [kHaSmemF4 host-assisted rows][kKmSmemF4 bytes-layout staging + compaction]
   const int wsm_f4 = (dv.ha ? kHaSmemF4 : 0) + (BYTES ? kKmSmemF4 : 0);
   float4* hsm = s_dyn + (threadIdx.x >> 5) * wsm_f4;
@@ -1396,13 +1523,25 @@ __global__ void __launch_bounds__(128, 4) km_kernel(const __grid_constant__ Dev 
   long long docc = 0;
   const uint32_t kcut = use_ha ? ha_kcut(dv, ka, par) : 0u;
   unsigned long long hostb = 0;
-  for (int c = 0; c < ka.ncls; ++c) {
+  uint32_t bkb0 = 0, bkb1 = 0;
+  bool poller = false;
+  if (use_ha) {  // warp 0 of CTA 0 polls the host threads' progress; the other warps read blocks
+    uint32_t cnt[8];
+    for (int c = 0; c < 8; ++c) cnt[c] = c < ka.ncls ? *(volatile uint32_t*)&dv.ctl->counts[par][c] : 0u;
+    ha_range(dv, cnt, ka.cls_off, ka.ncls, bkb0, bkb1);
+    poller = gw == 0;
+    if (poller) ha_poll(dv, epoch, bkb0, min(kcut, bkb1 + 1u), lane);
+    gw -= 1;
+    nw -= 1;
+  }
+  for (int c = 0; c < ka.ncls && !poller; ++c) {
     const uint32_t nmiss = *(volatile uint32_t*)&dv.ctl->counts[par][c];
     if (!nmiss) continue;
     const MissRec* ml = dv.miss + ka.cls_off[c];
 #define FL_KM(D)                                                                                              \
   if (use_ha)                                                                                                 \
-    km_ha<BYTES, D>(dv, ka.out, ml, epoch, nmiss, lane, gw, nw, ins, ev, byp, docc, hostb, hsm, wsm, harows, hato, kcut); \
+    km_ha<BYTES, D>(dv, ka.out, ml, epoch, nmiss, lane, gw, nw, ins, ev, byp, docc, hostb, hsm, wsm, harows, hato, kcut, \
+                    bkb0);                                                                                  \
   else                                                                                                        \
     km_rows<BYTES, D, KmM<BYTES, D>::value>(dv, ka.out, ml, epoch, nmiss, lane, gw, nw, ins, ev, byp, docc, hostb, wsm)
     if constexpr (DU > 0) {

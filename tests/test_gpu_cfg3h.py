@@ -47,7 +47,8 @@ def test_cfg3h_terabyte_shape_both_miss_paths(monkeypatch):
     N = w.batch(0).lookups
     zc = ha = None
     try:
-        zc = fl.FlatCache(w.cards, w.dims, tabs, w.cache_bytes, N, 0, 1.0, 0, H.HASH_SEED)  # registers the tier
+        zc = fl.FlatCache(w.cards, w.dims, tabs, w.cache_bytes, N, 0, 1.0, 0, H.HASH_SEED,
+                          fl.binding.FLAG_NO_HOST_ASSIST)  # registers the tier
         monkeypatch.delenv("FLECHE_HA_FRAC", raising=False)  # the default share (0.85 above 32 GiB)
         ha = fl.FlatCache(w.cards, w.dims, tabs, w.cache_bytes, N, 0, 1.0, 0, H.HASH_SEED, fl.binding.FLAG_HOST_ASSIST)
         assert zc.encoding()[0] == 31

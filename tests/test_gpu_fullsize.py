@@ -29,9 +29,9 @@ def cfg5_tables():
     return [np.ascontiguousarray(t) for t in w.make_tables()[1]]
 
 
-@pytest.mark.parametrize("ha", ["off", "split"])
+@pytest.mark.parametrize("ha", ["off", "split", "default"])
 def test_cfg5_full_size(monkeypatch, cfg5_tables, ha):
-    flags = 0
+    flags = fl.binding.FLAG_NO_HOST_ASSIST if ha == "off" else 0
     if ha == "split":
         monkeypatch.setenv("FLECHE_HA_FRAC", "0.5")
         flags = fl.binding.FLAG_HOST_ASSIST
@@ -52,7 +52,7 @@ def test_cfg5_full_size(monkeypatch, cfg5_tables, ha):
     assert abs(hg - ho) < 0.01, (hg, ho)
     st = gpu.stats()
     assert st["occupancy_bytes"] <= st["capacity_bytes"]
-    if ha == "split":
+    if ha != "off":
         # the host threads idle (50 us polls) while the oracle runs between batches here, so
         # some staging blocks time out and are fetched zero-copy: allowed (values are checked
         # above), as long as the host threads still stage most of their share

@@ -218,13 +218,17 @@ def test_cfg1_parity_and_hit_ratio():
     assert dg["host_bytes_fetched"] == dg["unique_misses"] * 128
 
 
-def test_cfg2_full_size_parity():
+@pytest.mark.parametrize("miss_path", ["default", "zero_copy"])
+def test_cfg2_full_size_parity(miss_path):
     # BASELINE configs[1] at full size in the bench's launch configuration: 8.64 GB host
     # tier, 1,688,128-row cache, 212,992 lookups per batch; out bit-exact each batch,
-    # hit ratio within 1 pp of the oracle's global policy over the window
+    # hit ratio within 1 pp of the oracle's global policy over the window.  default: the
+    # host-assisted split (on by default for a >= 1 GiB host tier); zero_copy: unified
+    # index only (FLAG_NO_HOST_ASSIST)
     w = configs.get("cfg2")
     tabs = _tables(w)
-    gpu, glob = H.make_pair(w, tabs, O.MODE_GLOBAL)
+    gpu, glob = H.make_pair(w, tabs, O.MODE_GLOBAL,
+                            flags=fl.binding.FLAG_NO_HOST_ASSIST if miss_path == "zero_copy" else 0)
     warm, meas = 150, 30
     for b in range(warm + meas):
         if b == warm:
@@ -240,6 +244,10 @@ def test_cfg2_full_size_parity():
     assert abs(hg - ho) < 0.01, (hg, ho)
     st = gpu.stats()
     assert st["occupancy_bytes"] <= st["capacity_bytes"]
+    if miss_path == "default":
+        assert dg["assisted_rows"] > 0.5 * dg["unique_misses"], dg  # the host threads staged most rows
+    else:
+        assert st["assisted_rows"] == 0
 
 
 @pytest.mark.parametrize("ordered", ["0", "1"])
