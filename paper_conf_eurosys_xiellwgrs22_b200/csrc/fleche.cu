@@ -8,6 +8,7 @@
 #include <cuda_runtime.h>
 
 #include <immintrin.h>
+#include <sys/prctl.h>
 #include <time.h>
 
 #include <algorithm>
@@ -40,7 +41,8 @@ struct HostAssist {
   HaReq* req = nullptr;                // [2][req_cap] (indexed like the miss list)
   HaDesc* desc = nullptr;              // [2]
   unsigned long long* bell = nullptr;  // doorbell (epoch)
-  unsigned long long* prog = nullptr;  // [2][kHaMaxThreads] progress words (epoch << 32 | blocks staged)
+  uint32_t* ready = nullptr;           // [2][blk_cap] ready word of each staging block (= epoch once staged)
+  uint32_t blk_cap = 0;
   float* stage = nullptr;              // [2][stage_floats]
   uint32_t req_cap = 0;
   bool nt_stores = true;  // FLECHE_HA_NT=0: plain memcpy into the staging buffer (A/B)
@@ -295,11 +297,12 @@ __attribute__((target("avx2"))) void stage_row(float* dst, const float* src, siz
 // One host-assist thread: wait for a doorbell, gather this thread's blocks of the batch's
 // requests (block k = miss-list indices [64k, 64k + 64), rows of every width class in
 // it, k % nthreads == me, in increasing k) into the staging buffer with non-temporal
-// stores, and publish the progress word (epoch << 32 | blocks done) after each block.
-// Spins while batches keep coming; after ~2 ms without one it polls every 50 us (an idle
+// stores, and publish each block's ready word (= epoch) once its rows are in place.
+// Spins while batches keep coming; after ~20 ms without one it polls every 20 us (an idle
 // ctx burns no core).  No `pause` in the spin: on a KVM guest it can trigger pause-loop
 // exits that deschedule the vCPU.
 void ha_worker(HostAssist* h, int me) {
+  prctl(PR_SET_TIMERSLACK, 1000UL, 0, 0, 0);  // idle polls wake within ~20 us, not the default 50 us slack
   uint32_t last = 0;
   uint64_t spins = 0;
   auto now_ns = []() {
@@ -312,8 +315,8 @@ void ha_worker(HostAssist* h, int me) {
   while (!h->stop.load(std::memory_order_relaxed)) {
     const uint32_t e = (uint32_t)__atomic_load_n(h->bell, __ATOMIC_ACQUIRE);
     if (e == last) {
-      if ((++spins & 1023) == 0 && now_ns() - t_last > 2000000ull) {
-        struct timespec ts = {0, 50000};
+      if ((++spins & 1023) == 0 && now_ns() - t_last > 20000000ull) {
+        struct timespec ts = {0, 20000};
         nanosleep(&ts, nullptr);
       }
       continue;
@@ -342,9 +345,7 @@ void ha_worker(HostAssist* h, int me) {
       if (!got && (n & 255) == 255 && now_ns() - t_last > 1000000ull) break;
     }
     if (!got) continue;  // the GPU moved on (a later batch's doorbell, or a parity cycle ahead)
-    unsigned long long* prog = h->prog + (size_t)par * kHaMaxThreads + me;
-    uint64_t done = 0;
-    __atomic_store_n(prog, ((unsigned long long)e << 32), __ATOMIC_RELEASE);  // this batch, nothing staged yet
+    uint32_t* ready = h->ready + (size_t)par * h->blk_cap;
     const HaReq* rq = h->req + (size_t)par * h->req_cap;
     float* st = h->stage + (size_t)par * h->stage_floats;
     uint64_t lo_all = ~0ull, hi_all = 0;
@@ -394,7 +395,11 @@ void ha_worker(HostAssist* h, int me) {
         for (int b = 0; b < dd * 4; b += 64) __builtin_prefetch((const char*)p + b, 0, 0);
     };
     const uint64_t kb0 = lo_all / kHaBlock, kb1 = (hi_all - 1) / kHaBlock;
-    for (uint64_t kb = kb0; kb <= kb1 && kb < kcut && !lost; ++kb) {
+    const uint64_t kend = std::min<uint64_t>(kb1 + 1, kcut);
+    // static ownership (block k belongs to thread k % nthreads in every batch, taken in
+    // increasing k): a thread that stalls past the GPU's give-up can only ever overwrite
+    // slots of its own blocks, which it republishes only after rewriting them
+    for (uint64_t kb = kb0; kb < kend && !lost; ++kb) {
       if (kb % (uint64_t)h->nthreads != (uint64_t)me) continue;
       if (h->delay_ns) {  // a stalled host thread (tests): its blocks time out on the GPU
         struct timespec ts = {(time_t)(h->delay_ns / 1000000000ull), (long)(h->delay_ns % 1000000000ull)};
@@ -425,9 +430,9 @@ void ha_worker(HostAssist* h, int me) {
           }
         }
       }
-      if (h->nt_stores) _mm_sfence();  // streaming stores are weakly ordered: drain them before the progress word
+      if (h->nt_stores) _mm_sfence();  // streaming stores are weakly ordered: drain them before the ready word
       if (lost) break;
-      __atomic_store_n(prog, ((unsigned long long)e << 32) | ++done, __ATOMIC_RELEASE);
+      __atomic_store_n(ready + kb, e, __ATOMIC_RELEASE);
 #ifdef FLECHE_EXPERIMENTS
       if (h->exp_pub) {
         struct timespec ts;
@@ -551,7 +556,8 @@ cudaError_t launch_k(int which, void (*kern)(KArgs...), unsigned grid, unsigned 
 // The miss side of one batch: KM (fetch + insert + restore), a cooperative launch (its grid
 // barrier before the restore needs every CTA resident; km_blocks never exceeds that).
 void launch_miss(fleche_ctx* c, cudaStream_t s, const KMArgs& ka) {
-  launch_k(kPdlCoop, km_fn(c->dv.bytes != 0, c->cls_dim.size() == 1 ? c->max_dim : 0), c->km_blocks, 128, c->km_smem, s,
+  static const bool coop = !(getenv("FLECHE_KM_COOP") && !atoi(getenv("FLECHE_KM_COOP")));  // A/B of the launch cost only
+  launch_k(coop ? kPdlCoop : kPdlNone, km_fn(c->dv.bytes != 0, c->cls_dim.size() == 1 ? c->max_dim : 0), c->km_blocks, 128, c->km_smem, s,
            c->dv, ka);
   c->kernels += 1;
 }
@@ -950,9 +956,10 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
     h->nthreads = (int)std::max<uint64_t>(
         1, std::min<uint64_t>(kHaMaxThreads, env_u("FLECHE_HA_THREADS", std::max(1u, std::min(12u, ncpu > 4 ? ncpu - 4 : 1)))));
     h->req_cap = (uint32_t)cfg->max_lookups;  // requests are indexed like the miss list
+    h->blk_cap = h->req_cap / kHaBlock + 2;
     h->stage_floats = std::max<uint64_t>(1024, env_u("FLECHE_HA_STAGE_KB", 131072) << 8);
     const size_t o_req = 0, o_desc = o_req + 2 * sizeof(HaReq) * (size_t)h->req_cap, o_bell = o_desc + 2 * sizeof(HaDesc),
-                 o_prog = (o_bell + 8 + 127) & ~size_t(127), o_stage = (o_prog + 16ull * kHaMaxThreads + 255) & ~size_t(255),
+                 o_ready = (o_bell + 8 + 127) & ~size_t(127), o_stage = (o_ready + 8ull * h->blk_cap + 255) & ~size_t(255),
                  total = o_stage + 2 * 4 * h->stage_floats;
     if (cudaHostAlloc(&h->mem, total, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess) {
       cudaGetLastError();
@@ -964,7 +971,7 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
     h->req = (HaReq*)(b + o_req);
     h->desc = (HaDesc*)(b + o_desc);
     h->bell = (unsigned long long*)(b + o_bell);
-    h->prog = (unsigned long long*)(b + o_prog);
+    h->ready = (uint32_t*)(b + o_ready);
     h->stage = (float*)(b + o_stage);
     void* dmem = nullptr;
     if (cudaHostGetDevicePointer(&dmem, h->mem, 0) != cudaSuccess) return fail(FLECHE_ECUDA);
@@ -973,10 +980,10 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
     dv.ha_req = (HaReq*)(db + o_req);
     dv.ha_desc = (HaDesc*)(db + o_desc);
     dv.ha_bell = (unsigned long long*)(db + o_bell);
-    dv.ha_prog = (unsigned long long*)(db + o_prog);
-    dv.ha_threads = (uint32_t)h->nthreads;
-    if (cudaMalloc((void**)&dv.ha_seen, 8 * kHaMaxThreads) != cudaSuccess ||
-        cudaMemset(dv.ha_seen, 0, 8 * kHaMaxThreads) != cudaSuccess)
+    dv.ha_ready = (uint32_t*)(db + o_ready);
+    dv.ha_blk_cap = h->blk_cap;
+    if (cudaMalloc((void**)&dv.ha_seen, 4ull * h->blk_cap) != cudaSuccess ||
+        cudaMemset(dv.ha_seen, 0, 4ull * h->blk_cap) != cudaSuccess)
       return fail(FLECHE_ENOMEM);
     dv.ha_stage = (float*)(db + o_stage);
     dv.ha_req_cap = h->req_cap;
@@ -1005,9 +1012,9 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   cudaMemset(dv.exp_buf, 0, ((size_t)c->km_blocks * 4 * 4 + 8) * 8);
   dv.exp_slots = (uint32_t)c->km_blocks * 16;
   if (c->ha) {
-    if (cudaMalloc((void**)&dv.exp_blk, ((size_t)(c->ha->req_cap / kHaBlock + 2) * 4) * 8) != cudaSuccess) return fail(FLECHE_ENOMEM);
-    cudaMemset(dv.exp_blk, 0, ((size_t)(c->ha->req_cap / kHaBlock + 2) * 4) * 8);
-    c->ha->exp_pub = new uint64_t[(c->ha->req_cap / kHaBlock + 2)]();
+    if (cudaMalloc((void**)&dv.exp_blk, ((size_t)c->ha->blk_cap * 4) * 8) != cudaSuccess) return fail(FLECHE_ENOMEM);
+    cudaMemset(dv.exp_blk, 0, ((size_t)c->ha->blk_cap * 4) * 8);
+    c->ha->exp_pub = new uint64_t[c->ha->blk_cap]();
   }
 #endif
   if (cudaDeviceSynchronize() != cudaSuccess) return fail(FLECHE_ECUDA);
@@ -1750,7 +1757,7 @@ extern "C" __attribute__((visibility("default"))) fleche_status fleche_exp_ha_bl
                                                                                      size_t nblk) {
   if (!c || !host || !c->ha) return FLECHE_EINVAL;
   if (c->have_last) cudaStreamSynchronize(c->last_stream);
-  const size_t m = std::min(nblk, (size_t)(c->ha->req_cap / kHaBlock + 2));
+  const size_t m = std::min(nblk, (size_t)c->ha->blk_cap);
   std::vector<uint64_t> g(m * 4);
   if (cudaMemcpy(g.data(), c->dv.exp_blk, m * 4 * 8, cudaMemcpyDeviceToHost) != cudaSuccess) return FLECHE_ECUDA;
   for (size_t k = 0; k < m; ++k) {

@@ -59,7 +59,7 @@ constexpr int kKmWarps = 4;     // KM CTA = 4 warps
 constexpr int kKmStageF4 = 256; // bytes layout, per warp: staged rows of a chunk (<= 4 KB) ...
 constexpr int kKmSmemF4 = 512;  // ... + the compaction buffer of one set region (<= 4 KB)
 constexpr int kHaBlock = 64;    // host-assisted miss fetch: rows per staging block
-constexpr int kHaMaxThreads = 16;  // host-assisted: at most this many host threads (one progress word each)
+constexpr int kHaMaxThreads = 16;  // host-assisted: at most this many host threads
 constexpr int kHaSmemF4 = 512;  // host-assisted KM, per warp: 8 KB of rows landed from the host (4 KM CTAs per SM)
 
 enum Ctr : int {
@@ -138,15 +138,16 @@ struct Ctl {
 // GPU's address-translation limit on scattered zero-copy reads (profiles/), and the GPU
 // then reads their staging buffer contiguously.  The owner lane of each unique miss in KQ
 // writes (table, row, staging slot) to the request list in pinned host memory at its
-// miss-list index; KQ's last CTA rings a doorbell with the batch's per-width miss counts.
-// Host thread i gathers every staging block k (kHaBlock list indices) with k % T == i,
-// in increasing k, and after each block publishes its progress word (epoch << 32 |
-// blocks done; all T words share two cache lines).  ONE poller warp of KM reads those
-// words over the link and mirrors them into HBM; every other KM warp waits on the mirror
-// for its block (no per-block polls competing with the row reads for the link), then
-// reads the block's staged rows.  Past the timeout the poller gives up and the readers
-// fetch the rows zero-copy from the tables, so a missing or slow host thread costs time,
-// never correctness.  Every area is double-buffered by epoch parity.
+// miss-list index; KQ's last warp rings a doorbell with the batch's per-width miss counts.
+// Host thread i gathers every staging block k (kHaBlock list indices) with k % T == i, in
+// increasing k, and sets each block's ready word (= epoch) once staged.  ONE poller warp of KM reads the batch's
+// ready words over the link (32 per load instruction) and mirrors them into HBM; every
+// other KM warp waits on the mirror for its block (no per-block polls competing with the
+// row reads for the link), then reads the block's staged rows.  When no new block has
+// been staged for kHaStallNs (a host thread descheduled mid-batch) or past the timeout,
+// the poller gives up and the waiting readers fetch their rows zero-copy from the tables,
+// so a missing or slow host thread costs time, never correctness.  Every area is double-buffered by
+// epoch parity.
 struct HaReq {  // one request, both halves tagged with the batch epoch (see ha_req_make)
   unsigned long long tid;    // table (9 bits) << 55 | epoch (15 bits) << 40 | row (40 bits)
   unsigned long long stage;  // epoch (24 bits) << 40 | float offset of its staging slot (40 bits; all ones: none)
@@ -205,10 +206,10 @@ struct Dev {
   HaReq* ha_req;               // [2][ha_req_cap]: indexed like the miss list
   HaDesc* ha_desc;             // [2]
   unsigned long long* ha_bell; // doorbell: epoch of the latest published descriptor
-  unsigned long long* ha_prog; // [2][kHaMaxThreads] (host memory) thread i's progress: epoch << 32 | blocks staged
-  unsigned long long* ha_seen; // [kHaMaxThreads] (HBM) the poller warp's mirror of ha_prog[epoch & 1]
+  uint32_t* ha_ready;          // [2][ha_blk_cap] (host memory) epoch of each staging block once staged
+  uint32_t* ha_seen;           // [ha_blk_cap] (HBM) the poller warp's mirror of ha_ready[epoch & 1]
   float* ha_stage;             // [2][ha_stage_floats]
-  uint32_t ha_req_cap, ha_threads;
+  uint32_t ha_req_cap, ha_blk_cap;
   uint64_t ha_stage_floats;
   uint64_t ha_timeout_ns;
   uint32_t ha_frac_q16;        // share of the batch's staging blocks given to the host threads (x 2^-16)
@@ -409,36 +410,53 @@ __device__ __forceinline__ void ha_range(const Dev& dv, const uint32_t* cnt, con
   kb1 = hi ? (hi - 1) / kHaBlock : 0u;
 }
 
-// The poller warp (lane i < T: host thread i): mirror the host threads' progress words
-// into HBM until every thread has staged its share of [kb0, kend), or give up after the
-// timeout (ha_abort = epoch: the readers then fetch the rest zero-copy).
+// The poller warp: mirror the ready words of staging blocks [kb0, kend) into HBM until all
+// are staged, or give up (ha_abort = epoch: the readers still waiting go zero-copy) when
+// no new block became ready for kHaStallNs after one did (a host thread descheduled
+// mid-batch), or past the timeout.  Each round reads the ready words of every block not
+// mirrored yet (strong relaxed loads, 4 per lane in flight), then one system-scope fence
+// orders the staged rows of the newly ready blocks before their mirror words.
+constexpr unsigned long long kHaStallNs = 40000;
+__device__ __forceinline__ uint32_t ld_relaxed_sys_u32(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.relaxed.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
 __device__ __forceinline__ void ha_poll(const Dev& dv, uint32_t epoch, uint32_t kb0, uint32_t kend, int lane) {
-  const int T = (int)dv.ha_threads;
-  const unsigned long long* prog = dv.ha_prog + (size_t)(epoch & 1u) * kHaMaxThreads;
-  uint32_t quota = 0;
-  if (lane < T && kend > kb0) {
-    const uint32_t first = kb0 + (uint32_t)((lane - (int)(kb0 % (uint32_t)T) + T) % T);
-    quota = first < kend ? (kend - 1 - first) / (uint32_t)T + 1u : 0u;
-  }
-  unsigned long long last = 0;
+  const uint32_t* ready = dv.ha_ready + (size_t)(epoch & 1u) * dv.ha_blk_cap;
   const unsigned long long t0 = globaltimer_ns();
-  while (true) {
-    bool done = true;
-    if (lane < T) {
-      unsigned long long v = ld_cv_u64(prog + lane);
-      if ((uint32_t)(v >> 32) == epoch) {
-        if (v != last) {
-          v = ld_acquire_sys_u64(prog + lane);  // orders the staged rows before the mirror
-          st_release_gpu_u64(dv.ha_seen + lane, v);
-          last = v;
-        }
-        done = (uint32_t)v >= quota;
-      } else {
-        done = quota == 0;
+  unsigned long long t_progress = 0;  // last time a new block was seen ready (0: none yet)
+  uint32_t lo = kb0;                  // every block below lo has been mirrored
+  while (lo < kend) {
+    uint32_t first_missing = kend, fresh = 0;
+    for (uint32_t k0 = lo; k0 < kend; k0 += 32 * 4) {
+      uint32_t v[4];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const uint32_t k = k0 + 32 * q + lane;
+        v[q] = (k < kend && ld_acquire_gpu_u32(dv.ha_seen + k) != epoch) ? ld_relaxed_sys_u32(ready + k) : ~0u;
+      }
+      uint32_t newly = 0;
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const uint32_t k = k0 + 32 * q + lane;
+        if (v[q] == epoch) newly |= 1u << q;
+        const unsigned miss = __ballot_sync(kFull, k < kend && v[q] != ~0u && v[q] != epoch);
+        if (miss) first_missing = min(first_missing, k0 + 32 * q + (uint32_t)(__ffs(miss) - 1));
+      }
+      if (__any_sync(kFull, newly)) {
+        asm volatile("fence.acq_rel.sys;" ::: "memory");  // the rows staged before these ready words
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+          if (newly & (1u << q)) st_release_gpu_u32(dv.ha_seen + k0 + 32 * q + lane, epoch);
+        fresh += __popc(__ballot_sync(kFull, newly != 0));
       }
     }
-    if (__all_sync(kFull, done)) break;
-    if (globaltimer_ns() - t0 > dv.ha_timeout_ns) {
+    const unsigned long long now = globaltimer_ns();
+    if (fresh) t_progress = now;
+    lo = first_missing;
+    if (lo >= kend) break;
+    if (now - t0 > dv.ha_timeout_ns || (t_progress && now - t_progress > kHaStallNs)) {
       if (lane == 0) st_release_gpu_u32(&dv.ctl->ha_abort, epoch);
       break;
     }
@@ -446,14 +464,10 @@ __device__ __forceinline__ void ha_poll(const Dev& dv, uint32_t epoch, uint32_t 
 }
 
 // A reader warp's wait (one lane) for staging block kb; false: timed out / abandoned.
-__device__ __forceinline__ bool ha_wait_block(const Dev& dv, uint32_t epoch, uint32_t kb0, uint32_t kb) {
-  const uint32_t T = dv.ha_threads, i = kb % T;
-  const uint32_t first = kb0 + (i + T - kb0 % T) % T;
-  const uint32_t need = (kb - first) / T + 1u;
+__device__ __forceinline__ bool ha_wait_block(const Dev& dv, uint32_t epoch, uint32_t kb) {
   const unsigned long long t0 = globaltimer_ns();
   while (true) {
-    const unsigned long long v = ld_acquire_gpu_u64(dv.ha_seen + i);
-    if ((uint32_t)(v >> 32) == epoch && (uint32_t)v >= need) return true;
+    if (ld_acquire_gpu_u32(dv.ha_seen + kb) == epoch) return true;
     if (*(volatile uint32_t*)&dv.ctl->ha_abort == epoch) return false;
     if (globaltimer_ns() - t0 > dv.ha_timeout_ns + 20000ull) return false;  // safety net behind the poller's
     __nanosleep(64);
@@ -916,12 +930,13 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
     }
   }
   if (qa.ha_bell) {
-    // host-assisted fetch: the last CTA rings the doorbell once every CTA has counted its
-    // misses (one KM launch earlier than KM could).  No system fence per CTA: the requests
-    // carry epoch tags and the host threads wait for them (ha_req_current).
+    // host-assisted fetch: the last CTA to finish rings the doorbell once every CTA has
+    // counted its misses (earlier than KM could).  No system fence: the requests carry
+    // epoch tags and the host threads wait for them (ha_req_current); no fence before the
+    // arrival either: the warps' miss-count atomics returned their values, so they are
+    // performed (a fence would also wait for the request stores to cross the link).
     __syncthreads();
     if (threadIdx.x == 0) {
-      __threadfence();
       const uint32_t prev = atomicAdd(&dv.ctl->kq_done, 1u);
       if (prev == gridDim.x - 1) {
         __threadfence();
@@ -1185,7 +1200,7 @@ __device__ __forceinline__ void km_ha(const Dev& dv, float* __restrict__ out, co
     if (dv.exp_blk && lane == 0) dv.exp_blk[kb * 4 + 0] = globaltimer_ns();
 #endif
     if (lane == 0 && kb < kcut) {  // the host threads' share; blocks >= kcut are read from the tables
-      ok = ha_wait_block(dv, epoch, bkb0, kb);
+      ok = ha_wait_block(dv, epoch, kb);
       if (!ok) ++hato;
     }
 #ifdef FLECHE_EXPERIMENTS
