@@ -21,6 +21,10 @@ import argparse
 import faulthandler
 import json
 import os
+
+# the workload generator's OpenMP threads must not spin-wait after their parallel regions:
+# they would compete for cores with the ctx's host-assist threads (must be set before libgomp loads)
+os.environ.setdefault("OMP_WAIT_POLICY", "PASSIVE")
 import statistics
 import sys
 import threading
@@ -525,7 +529,8 @@ def run_config(args, w, P, W, K, world, rank, local, dist, primary: bool, extra_
                "l2": "inputs larger than L2: fresh ID batch per step, 4 rotating output buffers "
                      f"({4 * out_max * 4 / 1e6:.0f} MB), {w.cache_bytes / 1e6:.0f} MB slab"},
            "scans_per_step": dst["scans"] / steps_timed, "assisted_rows_per_step": dst["assisted_rows"] / steps_timed,
-           "assist_timeouts": dst["assist_timeouts"], "sharded": sharded, "wm": wm}
+           "assist_timeouts": dst["assist_timeouts"], "sharded": sharded, "wm": wm,
+           "ui_share": s1["ui_share_ppm"] / 1e6}
     if not primary:
         del outs, pre
         cache.close()
@@ -686,8 +691,11 @@ def main():
         cf["admit_prob"] = args.admit_prob
         cf["miss_fetch"] = (("host-assisted split: host threads stage a share of each batch's unique misses "
                              "(%.0f of %.0f per step, share FLECHE_HA_FRAC=%s), the miss kernel reads the rest "
-                             "zero-copy (unified index)") % (r["assisted_rows_per_step"], r["unique_misses_per_step"],
-                                                            os.environ.get("FLECHE_HA_FRAC", "default"))
+                             "zero-copy (unified index; its share of the blocks %.2f, %s)") % (
+                                r["assisted_rows_per_step"], r["unique_misses_per_step"],
+                                os.environ.get("FLECHE_HA_FRAC", "tuned"), r["ui_share"],
+                                "fixed by FLECHE_HA_FRAC" if os.environ.get("FLECHE_HA_FRAC") else
+                                "tuned online by the paper's loop, P:L861-872")
                             if r["assisted_rows_per_step"] > 0 else
                             "unified index: zero-copy reads of the host rows, address-ordered")
         cf["flags"] = args.flags

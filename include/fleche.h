@@ -157,6 +157,10 @@ typedef struct {
   uint64_t assisted_rows;      /* HOST_ASSIST: unique misses read from the host threads' staging    */
   uint64_t assist_timeouts;    /* HOST_ASSIST: staging blocks fetched zero-copy after the timeout   */
   uint64_t scans;              /* fleche_set_watermarks: batches whose full-table scan evicted      */
+  uint64_t ui_share_ppm;       /* host-assisted ctx: the unified index's current share of a batch's
+                                  staging blocks (GPU zero-copy reads; the host threads take the
+                                  rest), in parts per million, as tuned by the loop of P:L861-872;
+                                  0 without host assistance                                         */
 } fleche_stats_t;
 
 /* Create a cache for the tables in *cfg on cfg->device.  Allocates every device

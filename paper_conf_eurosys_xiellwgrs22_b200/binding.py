@@ -34,7 +34,7 @@ class fleche_config(ctypes.Structure):
 
 STAT_FIELDS = ["batches", "lookups", "hits", "misses", "invalid", "unique_keys", "unique_hits", "unique_misses",
                "inserted", "evicted", "bypassed", "occupancy_bytes", "capacity_bytes", "index_bytes",
-               "host_bytes_fetched", "kernels_launched", "assisted_rows", "assist_timeouts", "scans"]
+               "host_bytes_fetched", "kernels_launched", "assisted_rows", "assist_timeouts", "scans", "ui_share_ppm"]
 
 
 class fleche_stats_t(ctypes.Structure):

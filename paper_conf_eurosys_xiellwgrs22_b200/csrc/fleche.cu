@@ -876,6 +876,7 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   if (cudaMemset(dv.firstpos, 0xFF, (size_t)scr_n * 8) != cudaSuccess) return fail(FLECHE_ECUDA);
   Ctl ctl{};
   ctl.epoch = 1;
+  ctl.ha_frac_q16 = 0;  // set below once the host-assisted fetch is configured
   if (cudaMemcpy(dv.ctl, &ctl, sizeof(Ctl), cudaMemcpyHostToDevice) != cudaSuccess) return fail(FLECHE_ECUDA);
 
   std::vector<const float*> dptr;
@@ -990,14 +991,16 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
     dv.ha_stage_floats = h->stage_floats;
     dv.ha_timeout_ns = env_u("FLECHE_HA_TIMEOUT_US", 2000) * 1000ull;
     {  // share of the staging blocks the host threads gather (the rest: KM's zero-copy reads)
-      // default share: the host threads' share pays off more the larger the host tier (the
-      // GPU's translated reads slow down with the span): measured best 0.7-0.8 at 8.6 GB
-      // (cfg2, cfg5; profiles/bench_r02_ha_*.json), >= 0.85 at 113 GB (cfg3h, round 1)
-      uint64_t span = 0;
-      for (int t = 0; t < n; ++t) span += (uint64_t)c->card[t] * (uint64_t)c->dims[t] * 4u;
+      // (fixed shares measured: best 0.7-0.8 at 8.6 GB, cfg2 and cfg5, profiles/bench_r02_ha_*.json;
+      // >= 0.85 at 113 GB, cfg3h, round 1)
       const char* e = getenv("FLECHE_HA_FRAC");
-      const double f = e ? std::min(1.0, std::max(0.0, atof(e))) : (span > (32ull << 30) ? 0.85 : 0.8);
-      dv.ha_frac_q16 = (uint32_t)(f * 65536.0 + 0.5);
+      // FLECHE_HA_FRAC fixes the share; otherwise the unified-index tuning loop (ui_tune,
+      // P:L861-872) starts with the host threads taking every block and moves it by itself
+      const double f = e ? std::min(1.0, std::max(0.0, atof(e))) : 1.0;
+      const uint32_t frac_q16 = (uint32_t)(f * 65536.0 + 0.5);
+      dv.ha_frac_fixed = e ? 1u : 0u;
+      if (cudaMemcpy(&dv.ctl->ha_frac_q16, &frac_q16, 4, cudaMemcpyHostToDevice) != cudaSuccess)
+        return fail(FLECHE_ECUDA);
       dv.ha_min_rows = (uint32_t)env_u("FLECHE_HA_MIN_ROWS", 1024);
     }
     h->nt_stores = env_u("FLECHE_HA_NT", 1) != 0 && __builtin_cpu_supports("avx2");
@@ -1186,6 +1189,7 @@ fleche_status fleche_stats(fleche_ctx* c, fleche_stats_t* out) {
   out->assisted_rows = v[C_HAROWS];
   out->assist_timeouts = v[C_HATIMEOUT];
   out->scans = v[C_SCANS];
+  out->ui_share_ppm = c->ha ? (uint64_t)(65536u - std::min(65536u, ctl.ha_frac_q16)) * 1000000ull / 65536ull : 0;
   return ctl.err_invalid ? FLECHE_ERANGE : FLECHE_OK;
 }
 

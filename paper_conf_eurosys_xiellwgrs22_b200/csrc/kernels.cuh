@@ -130,7 +130,18 @@ struct Ctl {
   uint32_t km_bar;        // KM grid barrier: epoch whose owner rows are all in `out`
   long long ke_occ;
   uint32_t kq_done;       // host-assisted: KQ CTA arrivals (the last one rings the doorbell)
-  uint32_t ha_abort;      // host-assisted: epoch whose staging the poller gave up on (timeout)       // watermark eviction: occ_bytes as KE1 saw it (KE2's one snapshot per scan)
+  uint32_t ha_abort;      // host-assisted: epoch whose staging the poller gave up on (timeout)
+  // unified-index share tuning (see ui_tune): the host threads' share of a
+  // batch's staging blocks (x 2^-16; the GPU's zero-copy reads -- the unified index -- take
+  // the rest), and the loop's state
+  uint32_t ha_frac_q16;
+  uint32_t tune_phase;         // 0 = growing the unified-index share, 1 = paused at the peak
+  unsigned long long km_t0;    // globaltimer at this batch's KM start (CTA 0)
+  unsigned long long win_ns;   // current window: KM time summed
+  unsigned long long win_miss; //   unique misses summed
+  uint32_t win_n;              //   batches
+  uint32_t tune_pad;
+  double prev_cost;            // ns per unique miss of the previous window (growing) / at the peak (paused)       // watermark eviction: occ_bytes as KE1 saw it (KE2's one snapshot per scan)
 };
 
 // Host-assisted miss fetch (FLECHE_FLAG_HOST_ASSIST): the CPU-DRAM layer's threads
@@ -212,7 +223,7 @@ struct Dev {
   uint32_t ha_req_cap, ha_blk_cap;
   uint64_t ha_stage_floats;
   uint64_t ha_timeout_ns;
-  uint32_t ha_frac_q16;        // share of the batch's staging blocks given to the host threads (x 2^-16)
+  uint32_t ha_frac_fixed;      // 1 = FLECHE_HA_FRAC fixed the host threads' share (no tuning loop)
   uint32_t ha_min_rows;        // batches with fewer unique misses stay all zero-copy (the split loses there)
 #ifdef FLECHE_EXPERIMENTS
   int32_t exp_mode;  // timing experiments only (libfleche_exp.so); breaks semantics
@@ -416,7 +427,7 @@ __device__ __forceinline__ void ha_range(const Dev& dv, const uint32_t* cnt, con
 // mid-batch), or past the timeout.  Each round reads the ready words of every block not
 // mirrored yet (strong relaxed loads, 4 per lane in flight), then one system-scope fence
 // orders the staged rows of the newly ready blocks before their mirror words.
-constexpr unsigned long long kHaStallNs = 40000;
+constexpr unsigned long long kHaStallNs = 150000;
 __device__ __forceinline__ uint32_t ld_relaxed_sys_u32(const uint32_t* p) {
   uint32_t v;
   asm volatile("ld.relaxed.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
@@ -482,7 +493,7 @@ __device__ __forceinline__ bool ha_wait_block(const Dev& dv, uint32_t epoch, uin
 // a non-zero share.  Otherwise KM takes the plain (address-ordered) zero-copy path and the
 // host threads are not woken.
 __device__ __forceinline__ bool ha_active(const Dev& dv, const KMArgs& ka, int par) {
-  if (!dv.ha || !dv.ha_frac_q16) return false;
+  if (!dv.ha || !*(volatile uint32_t*)&dv.ctl->ha_frac_q16) return false;
   uint32_t total = 0;
   for (int c = 0; c < ka.ncls; ++c) total += *(volatile uint32_t*)&dv.ctl->counts[par][c];
   return total >= dv.ha_min_rows;
@@ -501,7 +512,7 @@ __device__ __forceinline__ uint32_t ha_kcut(const Dev& dv, const KMArgs& ka, int
   uint32_t total = 0;
   for (int c = 0; c < ka.ncls; ++c) total += *(volatile uint32_t*)&dv.ctl->counts[par][c];
   if (total < dv.ha_min_rows) return kb0;  // small batch: the round trip to the host threads is not hidden
-  return kb0 + (uint32_t)(((unsigned long long)nb * dv.ha_frac_q16 + 65535ull) >> 16);
+  return kb0 + (uint32_t)(((unsigned long long)nb * *(volatile uint32_t*)&dv.ctl->ha_frac_q16 + 65535ull) >> 16);
 }
 
 // Programmatic dependent launch (sm_90+): the batch's kernels are launched with
@@ -948,7 +959,8 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
           cnt[c] = c < qa.ncls ? *(volatile uint32_t*)&dv.ctl->counts[par][c] : 0u;
           total += cnt[c];
         }
-        if (dv.ha_frac_q16 && total >= dv.ha_min_rows) {  // KM's ha_active() takes the same decision
+        const uint32_t frac = *(volatile uint32_t*)&dv.ctl->ha_frac_q16;  // KM reads the same value
+        if (frac && total >= dv.ha_min_rows) {  // KM's ha_active() takes the same decision
           uint32_t kb0, kb1;
           ha_range(dv, cnt, qa.cls_off, qa.ncls, kb0, kb1);
           HaDesc hd;
@@ -957,7 +969,7 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
             hd.cnt[c] = cnt[c];
             hd.off[c] = c < qa.ncls ? (uint32_t)qa.cls_off[c] : 0u;
           }
-          hd.kcut = kb0 + (uint32_t)(((unsigned long long)(kb1 - kb0 + 1u) * dv.ha_frac_q16 + 65535ull) >> 16);
+          hd.kcut = kb0 + (uint32_t)(((unsigned long long)(kb1 - kb0 + 1u) * frac + 65535ull) >> 16);
           hd.epoch2 = epoch;
           dv.ha_desc[par] = hd;  // no system fence: the host re-reads until both epoch fields match
           asm volatile("st.relaxed.sys.global.u64 [%0], %1;" ::"l"(dv.ha_bell), "l"((unsigned long long)epoch) : "memory");
@@ -1495,6 +1507,52 @@ struct KmM {
   static constexpr int value = D >= 256 ? 4 : (BYTES || D >= 64 ? 8 : 16);
 };
 
+// The paper's unified-index capacity loop: "We start with an empty unified
+// index, and keep gradually increasing its capacity ... We pause increasing until the
+// performance peak is reached.  If a significant performance decline is detected (which
+// means that workload changes), we clear the unified index and repeat."  Here the unified
+// index costs no HBM (computed host addresses, R11); what it trades against is the
+// CPU-DRAM layer: every staging block the GPU fetches itself (zero-copy) is one the host
+// threads do not gather.  So the tuned quantity is the unified index's share of a batch's
+// blocks, 1 - ha_frac: it starts at 0 (the host threads take every block), grows by
+// kTuneStep per window of kTuneWin batches while the miss kernel's time per unique miss
+// improves, pauses one step back at the peak, and restarts from 0 when a paused window is
+// kTuneDecline slower than the peak.  Run by KM's last CTA; it changes where rows are read
+// from only, never a result.
+constexpr uint32_t kTuneWin = 16;
+constexpr uint32_t kTuneStep = 6554;  // 0.1 of the blocks (x 2^-16)
+constexpr double kTuneDecline = 1.15;
+__device__ __forceinline__ void ui_tune(const Dev& dv, uint32_t nmiss) {
+  Ctl* c = dv.ctl;
+  const unsigned long long t = globaltimer_ns() - c->km_t0;
+  if (dv.ha_frac_fixed || nmiss < dv.ha_min_rows || t > 1000000000ull) return;
+  c->win_ns += t;
+  c->win_miss += nmiss;
+  if (++c->win_n < kTuneWin) return;
+  const double cost = (double)c->win_ns / (double)max(1ull, c->win_miss);
+  c->win_ns = c->win_miss = 0;
+  c->win_n = 0;
+  uint32_t f = c->ha_frac_q16;
+  if (c->tune_phase == 0) {  // growing the unified-index share
+    if (c->prev_cost == 0.0 || cost < c->prev_cost) {
+      c->prev_cost = cost;
+      if (f > kTuneStep) {
+        f -= kTuneStep;
+      } else {
+        c->tune_phase = 1;  // the unified index has every block: that is the peak
+      }
+    } else {
+      f = min(65536u, f + kTuneStep);  // one step back: the previous share was the peak
+      c->tune_phase = 1;
+    }
+  } else if (cost > c->prev_cost * kTuneDecline) {  // the workload changed: clear and repeat
+    f = 65536u;
+    c->tune_phase = 0;
+    c->prev_cost = 0.0;
+  }
+  c->ha_frac_q16 = f;
+}
+
 // DU > 0: uniform layout of width DU (one class); DU = 0: every width class in turn.
 template <bool BYTES, int DU>
 __global__ void __launch_bounds__(128, 4) km_kernel(const __grid_constant__ Dev dv, const __grid_constant__ KMArgs ka) {
@@ -1506,6 +1564,7 @@ __global__ void __launch_bounds__(128, 4) km_kernel(const __grid_constant__ Dev 
   const uint32_t epoch = *(volatile uint32_t*)&dv.ctl->epoch;
   const int par = epoch & 1u;
   const int lane = threadIdx.x & 31;
+  if (dv.ha && blockIdx.x == 0 && threadIdx.x == 0) dv.ctl->km_t0 = globaltimer_ns();  // (ui_tune)
   const bool use_ha = ha_active(dv, ka, par);  // KQ's last CTA rang the doorbell (same test)
   if (use_ha && ka.bell && blockIdx.x == 0 && threadIdx.x == 0) {
     // doorbell from KM (ctx option): KQ's request writes completed with its grid
@@ -1626,6 +1685,11 @@ __global__ void __launch_bounds__(128, 4) km_kernel(const __grid_constant__ Dev 
     __threadfence();
     const uint32_t prev = atomicAdd(&dv.ctl->done2, 1u);
     if (prev == gridDim.x - 1) {  // last CTA closes the batch: next batch's counters, epoch + 1
+      if (dv.ha) {
+        uint32_t nm = 0;
+        for (int c = 0; c < ka.ncls; ++c) nm += *(volatile uint32_t*)&dv.ctl->counts[par][c];
+        ui_tune(dv, nm);
+      }
 #pragma unroll
       for (int c = 0; c < 8; ++c) dv.ctl->counts[par ^ 1][c] = 0;
       dv.ctl->done2 = 0;

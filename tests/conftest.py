@@ -1,4 +1,8 @@
 import os
+
+# the workload generator's OpenMP threads must not spin-wait after their parallel regions:
+# they would compete for cores with the ctx's host-assist threads (must be set before libgomp loads)
+os.environ.setdefault("OMP_WAIT_POLICY", "PASSIVE")
 import subprocess
 import sys
 
