@@ -129,11 +129,12 @@ typedef struct {
 #define FLECHE_FLAG_HOST_ASSIST 0x8u
 #define FLECHE_FLAG_NO_HOST_ASSIST 0x20u
 /* FUSED_HIT_COPY: the query kernel copies each hit row itself (probe and copy in one
- * kernel, the fused design) instead of the default for uniform layouts with >= 512K
- * lookups per batch: the decoupled copy (Fig 8b), where the query kernel only
- * indexes and a copy kernel on a side stream moves the hit rows while the miss kernel
- * fetches the misses.  The paper's decoupling on/off comparison (Exp #7).
- * `out` and every counter are identical either way. */
+ * kernel, the fused design; the default since round 2, measured faster with the
+ * host-assisted miss fetch) even when FLECHE_DECOUPLE_MIN (lookups per batch, env) asks for
+ * the decoupled copy (Fig 8b), where the query kernel only indexes and a copy
+ * kernel on a side stream moves the hit rows while the miss kernel fetches the misses.
+ * The paper's decoupling on/off comparison (Exp #7).  `out` and every
+ * counter are identical either way. */
 #define FLECHE_FLAG_FUSED_HIT_COPY 0x10u
 
 typedef struct {

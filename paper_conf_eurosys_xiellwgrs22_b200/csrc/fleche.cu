@@ -90,7 +90,10 @@ struct fleche_ctx {
   cudaStream_t side = nullptr;
   cudaEvent_t fork_ev = nullptr, join_ev = nullptr;
   uint32_t* d_slots = nullptr;
-  int64_t decouple_min = 524288;  // lookups per batch from which the hit copy is decoupled (cfg2: equal, cfg5: +5 %)
+  // lookups per batch from which the hit copy is decoupled (FLECHE_DECOUPLE_MIN): never by
+  // default -- with the host-assisted miss fetch the fused copy measured faster at cfg2 (1780
+  // vs 1728 Mkeys/s) and cfg5 (2604 vs 2551; profiles/bench_r02_decouple_*.json)
+  int64_t decouple_min = INT64_MAX;
   size_t km_smem = 0;
   // host-side counters
   uint64_t batches = 0, lookups = 0, kernels = 0;
