@@ -409,11 +409,12 @@ __device__ __forceinline__ void st_release_gpu_u64(unsigned long long* p, unsign
 
 // Host-assisted geometry of a batch: staging blocks [kb0, kend) go to the host threads
 // (kend = the split point kcut, clipped to the batch's last block + 1).
-__device__ __forceinline__ void ha_range(const Dev& dv, const uint32_t* cnt, const int64_t* cls_off, int ncls,
+__device__ __forceinline__ void ha_range(const Dev& dv, const uint32_t (&cnt)[8], const int64_t* cls_off, int ncls,
                                          uint32_t& kb0, uint32_t& kb1) {
   uint32_t lo = 0xFFFFFFFFu, hi = 0;
-  for (int c = 0; c < ncls; ++c) {
-    if (!cnt[c]) continue;
+#pragma unroll
+  for (int c = 0; c < 8; ++c) {  // compile-time indices: cnt stays in registers
+    if (c >= ncls || !cnt[c]) continue;
     lo = min(lo, (uint32_t)cls_off[c]);
     hi = max(hi, (uint32_t)cls_off[c] + cnt[c]);
   }
