@@ -1005,6 +1005,7 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
       if (cudaMemcpy(&dv.ctl->ha_frac_q16, &frac_q16, 4, cudaMemcpyHostToDevice) != cudaSuccess)
         return fail(FLECHE_ECUDA);
       dv.ha_min_rows = (uint32_t)env_u("FLECHE_HA_MIN_ROWS", 1024);
+      dv.ha_unit_pieces = (uint32_t)env_u("FLECHE_HA_UNIT_PIECES", 0);  // 0: adaptive (km_ha)
     }
     h->nt_stores = env_u("FLECHE_HA_NT", 1) != 0 && __builtin_cpu_supports("avx2");
     h->delay_ns = env_u("FLECHE_HA_DELAY_US", 0) * 1000ull;

@@ -225,6 +225,8 @@ struct Dev {
   uint64_t ha_timeout_ns;
   uint32_t ha_frac_fixed;      // 1 = FLECHE_HA_FRAC fixed the host threads' share (no tuning loop)
   uint32_t ha_min_rows;        // batches with fewer unique misses stay all zero-copy (the split loses there)
+  uint32_t ha_unit_pieces;     // KM work unit = this many 16-row pieces (0: adaptive to the batch)
+  uint32_t ha_pad2;
 #ifdef FLECHE_EXPERIMENTS
   int32_t exp_mode;  // timing experiments only (libfleche_exp.so); breaks semantics
   int32_t exp_pad;
@@ -1201,27 +1203,43 @@ __device__ __forceinline__ void km_ha(const Dev& dv, float* __restrict__ out, co
                                       float4* hsm, float4* cbuf, unsigned& harows, unsigned& hato, uint32_t kcut,
                                       uint32_t bkb0) {
   constexpr int VEC = D / 4;
-  constexpr int ROWS = (kHaSmemF4 / VEC) < kHaBlock ? (kHaSmemF4 / VEC) : kHaBlock;  // rows per piece
-  constexpr int PER_LANE = ROWS * VEC / 32;  // float4 per lane per piece
+  constexpr int ROWS0 = (kHaSmemF4 / VEC) < kHaBlock ? (kHaSmemF4 / VEC) : kHaBlock;  // rows that fit the warp's smem
+  constexpr int ROWS = ROWS0 < 16 ? ROWS0 : 16;  // rows per piece: one warp per piece, pieces of a block in parallel
+  constexpr int PPB = kHaBlock / ROWS;           // pieces per staging block
+  constexpr int PER_LANE = ROWS * VEC / 32;      // float4 per lane per piece
   constexpr int INFL = PER_LANE < 16 ? PER_LANE : 16;
   const uint32_t off = (uint32_t)(mlist - dv.miss);
   const uint32_t kb0 = off / kHaBlock, kb1 = (off + nmiss - 1) / kHaBlock;
   const float* stage = dv.ha_stage + (size_t)(epoch & 1u) * dv.ha_stage_floats;
-  for (uint32_t kb = kb0 + gw; kb <= kb1; kb += nw) {
+  // work unit = one piece of one block: every piece of the batch has a warp of its own
+  // (a staged piece starts as soon as its block is ready; the zero-copy blocks >= kcut
+  // get the whole grid's memory-level parallelism, not one warp per 64 rows)
+  // pieces per warp unit: as fine as the grid allows (one piece per warp while there are
+  // enough warps, cfg2 +8 %), coarser for big batches (consecutive pieces of a block in one
+  // warp, cfg5 +8 %); FLECHE_HA_UNIT_PIECES fixes it (A/B)
+  const uint32_t npieces = (kb1 - kb0 + 1) * PPB;
+  const uint32_t ppu = dv.ha_unit_pieces ? min((uint32_t)PPB, dv.ha_unit_pieces)
+                                         : min((uint32_t)PPB, max(1u, (npieces + nw - 1) / nw));
+  for (uint32_t u0 = gw * ppu; u0 < (kb1 - kb0 + 1) * PPB; u0 += nw * ppu)
+  for (uint32_t u = u0; u < min(u0 + ppu, (kb1 - kb0 + 1) * PPB); ++u) {
+    const uint32_t kb = kb0 + u / PPB, pc = u % PPB;
+    const uint32_t plo_abs = kb * kHaBlock + pc * ROWS;  // the piece's list indices [plo_abs, plo_abs + ROWS)
+    const uint32_t lo_abs = max(plo_abs, off), hi_abs = min(plo_abs + (uint32_t)ROWS, off + nmiss);
+    if (lo_abs >= hi_abs) continue;  // the piece lies outside this width's region
+    const uint32_t blo = lo_abs - off, bhi = hi_abs - off;
     int ok = 0;
 #ifdef FLECHE_EXPERIMENTS
-    if (dv.exp_blk && lane == 0) dv.exp_blk[kb * 4 + 0] = globaltimer_ns();
+    if (dv.exp_blk && lane == 0 && pc == 0) dv.exp_blk[kb * 4 + 0] = globaltimer_ns();
 #endif
     if (lane == 0 && kb < kcut) {  // the host threads' share; blocks >= kcut are read from the tables
       ok = ha_wait_block(dv, epoch, kb);
-      if (!ok) ++hato;
+      if (!ok && pc == 0) ++hato;
     }
 #ifdef FLECHE_EXPERIMENTS
-    if (dv.exp_blk && lane == 0) dv.exp_blk[kb * 4 + 1] = globaltimer_ns();
+    if (dv.exp_blk && lane == 0 && pc == 0) dv.exp_blk[kb * 4 + 1] = globaltimer_ns();
 #endif
     ok = __shfl_sync(kFull, ok, 0);
-    const uint32_t blo = max(kb * kHaBlock, off) - off, bhi = min(kb * kHaBlock + kHaBlock, off + nmiss) - off;
-    for (uint32_t plo = blo; plo < bhi; plo += ROWS) {
+    for (uint32_t plo = blo; plo < bhi; plo += ROWS) {  // one iteration: the piece
       const uint32_t n = min((uint32_t)ROWS, bhi - plo);
       // the piece's miss records (row r on lane r % 32) and row sources
       MissRec m[(ROWS + 31) / 32];
