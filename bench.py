@@ -308,11 +308,21 @@ def run_config(args, w, P, W, K, world, rank, local, dist, primary: bool, extra_
     log(w.name, "host tier")
     t_gen = time.time()
     shm_cleanup = None
-    if dist:  # one copy per node in /dev/shm, mapped by every local rank
+    numa = None
+    if dist:  # one copy per NUMA node in /dev/shm, mapped by every local rank on that node
         from workload import shm
+        node = shm.gpu_numa_node(local)
+
+        def all_gather_object(x):
+            out = [None] * world
+            dist.all_gather_object(out, x)
+            return out
+
+        creator = shm.creator_ranks(local, node, all_gather_object)
         hostbuf, tabs, shm_cleanup = shm.shared_tables(
             f"fleche_{w.name}_{os.environ.get('MASTER_PORT', '0')}", w.cards, w.dims, w.value_mode, local,
-            dist.barrier)
+            dist.barrier, node=node, creator=creator)
+        numa = {"node": node, "nodes": shm.numa_nodes(), "copy_creator": creator}
     else:
         hostbuf, tabs = w.make_tables()
     t_gen = time.time() - t_gen
@@ -530,7 +540,7 @@ def run_config(args, w, P, W, K, world, rank, local, dist, primary: bool, extra_
                      f"({4 * out_max * 4 / 1e6:.0f} MB), {w.cache_bytes / 1e6:.0f} MB slab"},
            "scans_per_step": dst["scans"] / steps_timed, "assisted_rows_per_step": dst["assisted_rows"] / steps_timed,
            "assist_timeouts": dst["assist_timeouts"], "sharded": sharded, "wm": wm,
-           "ui_share": s1["ui_share_ppm"] / 1e6}
+           "ui_share": s1["ui_share_ppm"] / 1e6, "numa": numa}
     if not primary:
         del outs, pre
         cache.close()
@@ -702,6 +712,9 @@ def main():
         cf["eviction"] = (f"full-scan between watermarks hi={r['wm'][0]} lo={r['wm'][1]} (reading R23)" if r["wm"]
                           else "on demand (canonical, reading R2)")
         cf["timing"] = f"median of {args.reps} timed regions of {K} steps (CUDA events on the launching stream)"
+        if r["numa"]:
+            cf["host_tier"] = ("one /dev/shm copy per NUMA node (%d nodes), pages bound to the node of the GPUs "
+                               "that map it; rank 0's GPU on node %d" % (r["numa"]["nodes"], r["numa"]["node"]))
         line = {
             "metric": "embedding lookups/s", "value": r["value"], "unit": "Mkeys/s", "n_gpus": world, "steps": K,
             "warmup": W, "ms_per_step": r["ms_per_step"], "higher_is_better": True, "scaling": "weak",

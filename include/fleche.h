@@ -338,6 +338,21 @@ fleche_status fleche_route_p2p(fleche_ctx* ctx, const int64_t* const* ids, const
  * their concatenation.  One batch of the owner's cache. */
 fleche_status fleche_query_keys_seg(fleche_ctx* ctx, const uint32_t* const* segs, const int64_t* counts, int32_t nseg,
                                     float* rows, uint8_t* hit_flags, fleche_stream stream);
+/* Sync-free fused exchange (no host read of any count per batch): the G x G matrix
+ * counts_dev[src * G + owner] (int64, DEVICE, row-major) holds every rank's send_counts of
+ * this batch, e.g. the stream-ordered all-gather of them (NCCL), and me = this rank.
+ * fleche_query_keys_seg_dev answers segment src (counts_dev[src * G + me] keys at segs[src])
+ * with a grid sized for the ctx's max_lookups that strides over the device-side total;
+ * fleche_restore_p2p_dev computes this rank's offset in every owner's order on the device
+ * (the sum of counts_dev[src * G + o] over src < me).  Otherwise as fleche_query_keys_seg /
+ * fleche_restore_p2p; the owner's fleche_stats lookup count is not advanced (use
+ * fleche_shard_stats).  FLECHE_EINVAL for bad pointers, world or me. */
+fleche_status fleche_query_keys_seg_dev(fleche_ctx* ctx, const uint32_t* const* segs, const int64_t* counts_dev,
+                                        int32_t world, int32_t me, float* rows, uint8_t* hit_flags,
+                                        fleche_stream stream);
+fleche_status fleche_restore_p2p_dev(fleche_ctx* ctx, int32_t world, const float* const* peer_rows,
+                                     const uint8_t* const* peer_flags, const int64_t* counts_dev, int32_t me,
+                                     float* out, fleche_stream stream);
 /* CUDA IPC helpers for the fused exchange: export a device allocation (the base pointer
  * of a cudaMalloc allocation) as a 64-byte handle, map a peer process's handle into this
  * process (peer access enabled lazily), unmap it.  FLECHE_ECUDA on failure. */

@@ -82,6 +82,8 @@ fleche_set_watermarks = _sig("fleche_set_watermarks", ctypes.c_int, [_vp, ctypes
 fleche_route_p2p = _sig("fleche_route_p2p", ctypes.c_int, [_vp, _vp, _vp, _i32, _u32, _vp, _vp, _vp])
 fleche_query_keys_seg = _sig("fleche_query_keys_seg", ctypes.c_int, [_vp, _vp, _vp, _i32, _vp, _vp, _vp])
 fleche_restore_p2p = _sig("fleche_restore_p2p", ctypes.c_int, [_vp, _i32, _vp, _vp, _vp, _vp, _vp])
+fleche_query_keys_seg_dev = _sig("fleche_query_keys_seg_dev", ctypes.c_int, [_vp, _vp, _vp, _i32, _i32, _vp, _vp, _vp])
+fleche_restore_p2p_dev = _sig("fleche_restore_p2p_dev", ctypes.c_int, [_vp, _i32, _vp, _vp, _vp, _i32, _vp, _vp])
 fleche_ipc_alloc = _sig("fleche_ipc_alloc", ctypes.c_int, [ctypes.c_size_t, ctypes.POINTER(_vp)])
 fleche_ipc_free = _sig("fleche_ipc_free", ctypes.c_int, [_vp])
 fleche_ipc_handle = _sig("fleche_ipc_handle", ctypes.c_int, [_vp, _vp])
@@ -95,7 +97,8 @@ EXPORTED = ["fleche_create", "fleche_query", "fleche_query_pooled", "fleche_quer
             "fleche_probe_host_read", "fleche_route", "fleche_query_keys", "fleche_restore", "fleche_shard_stats",
             "fleche_kernel_times_ex", "fleche_set_watermarks", "fleche_prefill", "fleche_debug_ctl",
             "fleche_restore_p2p", "fleche_ipc_handle", "fleche_ipc_open", "fleche_ipc_close", "fleche_ipc_alloc",
-            "fleche_ipc_free", "fleche_route_p2p", "fleche_query_keys_seg", "fleche_encode"]
+            "fleche_ipc_free", "fleche_route_p2p", "fleche_query_keys_seg", "fleche_encode",
+            "fleche_query_keys_seg_dev", "fleche_restore_p2p_dev"]
 
 
 def encode(cards, key_bits: int = 0):
@@ -335,6 +338,21 @@ class FlatCache:
         cp = (_i64 * G)(*[int(x) for x in counts])
         _check(fleche_query_keys_seg(self.h, sp, cp, G, _ptr(rows), _ptr(hit_flags), _stream_handle(stream)),
                "fleche_query_keys_seg")
+
+    def query_keys_seg_dev(self, segs, counts_dev, me, rows, hit_flags=None, stream=None):
+        """Sync-free owner query: counts_dev = the G x G routed-count matrix (device int64)."""
+        G = len(segs)
+        sp = (_vp * G)(*[int(p) for p in segs])
+        _check(fleche_query_keys_seg_dev(self.h, sp, _ptr(counts_dev), G, int(me), _ptr(rows), _ptr(hit_flags),
+                                         _stream_handle(stream)), "fleche_query_keys_seg_dev")
+
+    def restore_p2p_dev(self, peer_rows, peer_flags, counts_dev, me, out, stream=None):
+        """Sync-free fused restore: offsets into the owners' answers from the device count matrix."""
+        W = len(peer_rows)
+        rp = (_vp * W)(*[int(p) for p in peer_rows])
+        fp = (_vp * W)(*[int(p) for p in peer_flags]) if peer_flags is not None else None
+        _check(fleche_restore_p2p_dev(self.h, W, rp, fp, _ptr(counts_dev), int(me), _ptr(out), _stream_handle(stream)),
+               "fleche_restore_p2p_dev")
 
     def restore_p2p(self, peer_rows, peer_flags, peer_off, out, stream=None):
         """Fused exchange: restore from every owner's rows in place (peer pointers, ints)."""

@@ -1409,7 +1409,7 @@ namespace {
 template <int MAXT>
 fleche_status launch_keys(fleche_ctx* c, const uint32_t* keys, int64_t count, float* rows, uint8_t* flags,
                           cudaStream_t s, const uint32_t* const* segs = nullptr, const int64_t* seg_counts = nullptr,
-                          int nseg = 0) {
+                          int nseg = 0, const int64_t* dcnt = nullptr, int me = 0) {
   QArgs<MAXT> qa;
   memset(&qa, 0, sizeof(qa));  // out_off[t] = 0: row g of `rows` answers keys[g]
   qa.n = 1;
@@ -1424,10 +1424,12 @@ fleche_status launch_keys(fleche_ctx* c, const uint32_t* keys, int64_t count, fl
     for (int i = 0; i < nseg; ++i) {
       qa.ids[i] = (const int64_t*)segs[i];
       qa.scan[i] = acc;
-      acc += seg_counts[i];
+      acc += seg_counts ? seg_counts[i] : 0;
     }
     qa.scan[nseg] = acc;
     qa.fkeys = segs[0];  // non-null: the flat-key path
+    qa.dcnt = dcnt;      // sync-free: the counts are read on the device; the grid strides over them
+    qa.dme = me;
   }
   KMArgs ka;
   memset(&ka, 0, sizeof(ka));
@@ -1436,7 +1438,11 @@ fleche_status launch_keys(fleche_ctx* c, const uint32_t* keys, int64_t count, fl
   ka.cls_dim[0] = c->max_dim;
   fleche_status st = prof_event(c, s, true, 4);
   if (st != FLECHE_OK) return st;
-  if (count > 0) {
+  if (dcnt) {  // count unknown on the host: a capacity-sized, grid-strided launch (TD = 0: no TMA variant)
+    const int64_t blocks = std::min<int64_t>((c->max_lookups + 127) / 128, (int64_t)FL_KQ_MIN_BLOCKS * c->sm_count);
+    launch_k(kPdlKQ, kq_fn<MAXT>(0), (unsigned)std::max<int64_t>(1, blocks), 128, 0, s, qa, c->dv);
+    c->kernels++;
+  } else if (count > 0) {
     launch_k(kPdlKQ, kq_fn<MAXT>(c->kq_tma), (unsigned)((count + 127) / 128), 128, c->kq_smem, s, qa, c->dv);
     c->kernels++;
   }
@@ -1615,6 +1621,53 @@ fleche_status fleche_query_keys_seg(fleche_ctx* c, const uint32_t* const* segs, 
     c->lookups += (uint64_t)count;
   }
   return st;
+}
+
+fleche_status fleche_query_keys_seg_dev(fleche_ctx* c, const uint32_t* const* segs, const int64_t* counts_dev,
+                                        int32_t world, int32_t me, float* rows, uint8_t* hit_flags,
+                                        fleche_stream stream) {
+  if (!c || !segs || !counts_dev || world < 1 || world > kMaxWorld || me < 0 || me >= world || !rows ||
+      ((uintptr_t)rows & 15u))
+    return FLECHE_EINVAL;
+  if (c->poisoned) return FLECHE_ESTATE;
+  if (!uniform_dims(c) || c->dv.part) return FLECHE_EINVAL;
+  for (int i = 0; i < world; ++i)
+    if (!segs[i]) return FLECHE_EINVAL;
+  fleche_status st = ensure_device(c);
+  if (st != FLECHE_OK) return st;
+  cudaStream_t s = (cudaStream_t)stream;
+  st = order_on(c, s);
+  if (st != FLECHE_OK) return st;
+  st = launch_keys<128>(c, segs[0], 0, rows, hit_flags, s, segs, nullptr, world, counts_dev, me);
+  if (st == FLECHE_OK) c->batches++;  // (the lookup count stays on the device: fleche_shard_stats)
+  return st;
+}
+
+fleche_status fleche_restore_p2p_dev(fleche_ctx* c, int32_t world, const float* const* peer_rows,
+                                     const uint8_t* const* peer_flags, const int64_t* counts_dev, int32_t me,
+                                     float* out, fleche_stream stream) {
+  if (!c || !out || ((uintptr_t)out & 15u) || !peer_rows || !counts_dev) return FLECHE_EINVAL;
+  if (c->poisoned) return FLECHE_ESTATE;
+  if (!c->rd_ready || world < 1 || world > kMaxWorld || world != c->rd.world || me < 0 || me >= world)
+    return FLECHE_EINVAL;
+  PeerArgs pa;
+  memset(&pa, 0, sizeof(pa));
+  pa.p2p = 1;
+  pa.me = me;
+  pa.dcnt = counts_dev;
+  for (int o = 0; o < world; ++o) {
+    if (!peer_rows[o]) return FLECHE_EINVAL;
+    pa.rows[o] = peer_rows[o];
+    pa.flags[o] = peer_flags ? peer_flags[o] : nullptr;
+  }
+  fleche_status st = ensure_device(c);
+  if (st != FLECHE_OK) return st;
+  cudaStream_t s = (cudaStream_t)stream;
+  st = order_on(c, s);
+  if (st != FLECHE_OK) return st;
+  if (c->n <= 32) return launch_restore<32>(c, nullptr, nullptr, out, s, pa);
+  if (c->n <= 128) return launch_restore<128>(c, nullptr, nullptr, out, s, pa);
+  return launch_restore<FLECHE_MAX_TABLES>(c, nullptr, nullptr, out, s, pa);
 }
 
 fleche_status fleche_route_p2p(fleche_ctx* c, const int64_t* const* ids, const int64_t* lengths, int32_t world,

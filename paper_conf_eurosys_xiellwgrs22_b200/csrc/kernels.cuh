@@ -253,6 +253,9 @@ struct QArgs {
   int32_t fkseg;             // key-sharded fused exchange: fkeys come in n segments (ids[], scan[])
   int32_t ha_bell;           // host-assisted: the last CTA rings the host threads' doorbell
   int32_t ncls;              //   (number of width classes of the miss list)
+  const int64_t* dcnt;       // key-sharded sync-free: [n][n] routed-count matrix in device memory
+  int32_t dme;               //   this rank (segment i's count = dcnt[i * n + dme])
+  int32_t pad3;
 };
 
 struct KMArgs {
@@ -702,17 +705,30 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
   __shared__ int64_t s_scan[MAXT + 1];
   __shared__ __align__(8) unsigned long long s_mbar[4];
   extern __shared__ __align__(128) float kq_dyn[];
-  for (int i = threadIdx.x; i <= qa.n; i += blockDim.x) s_scan[i] = qa.scan[i];
+  if (!qa.dcnt)
+    for (int i = threadIdx.x; i <= qa.n; i += blockDim.x) s_scan[i] = qa.scan[i];
   if constexpr (TD > 0) {
     if (threadIdx.x < 4) mbar_init((unsigned)__cvta_generic_to_shared(&s_mbar[threadIdx.x]), 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   pdl_wait();  // the previous batch (or the caller's producer of ids) has completed
+  if (qa.dcnt && threadIdx.x == 0) {
+    // key-sharded, sync-free: segment i's count is C[i][me] of the routed-count matrix in
+    // device memory (written by the collective the stream ran before this launch)
+    int64_t acc = 0;
+    for (int i = 0; i < qa.n; ++i) {
+      s_scan[i] = acc;
+      acc += qa.dcnt[(size_t)i * qa.n + qa.dme];
+    }
+    s_scan[qa.n] = acc;
+  }
   __syncthreads();
 
   const int lane = threadIdx.x & 31;
   const int64_t N = s_scan[qa.n];
-  const int64_t g = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  uint32_t it = 0;  // grid-stride iterations (one unless the grid was sized for a capacity, not N)
+  for (int64_t g0 = (int64_t)blockIdx.x * blockDim.x; g0 < N; g0 += (int64_t)gridDim.x * blockDim.x, ++it) {
+  const int64_t g = g0 + threadIdx.x;
   if (g - lane < N) {  // warp-uniform
     const uint32_t epoch = *(volatile uint32_t*)&dv.ctl->epoch;
     const bool active = g < N;
@@ -931,7 +947,7 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
     }
     if constexpr (TD > 0) {
       if (!qa.slots) {  // the rows have landed: the warp's output rows leave as one contiguous block
-        mbar_wait(mb, 0);
+        mbar_wait(mb, it & 1u);
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // the zero rows, for the bulk store
         __syncwarp();
         const unsigned na = (unsigned)__popc(__ballot_sync(kFull, active));  // a prefix of the warp
@@ -943,6 +959,7 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
       }
     }
   }
+  }  // grid-stride loop
   if (qa.ha_bell) {
     // host-assisted fetch: the last CTA to finish rings the doorbell once every CTA has
     // counted its misses (earlier than KM could).  No system fence: the requests carry

@@ -41,7 +41,8 @@ struct PeerArgs {
   const uint8_t* flags[kMaxWorld];
   int64_t off[kMaxWorld];
   int32_t p2p;
-  int32_t pad;
+  int32_t me;             // sync-free variant: this rank, and
+  const int64_t* dcnt;    // the [world][world] routed-count matrix in device memory (off[] unused)
 };
 
 // Fused exchange, key side (fleche_route_p2p): dst[o] = this rank's slot in owner o's
@@ -189,9 +190,20 @@ __global__ void __launch_bounds__(128) krs_kernel(const __grid_constant__ RArgs<
                                                   const float* __restrict__ rows, const uint8_t* __restrict__ flags,
                                                   float* __restrict__ out, const __grid_constant__ PeerArgs pa) {
   __shared__ int64_t s_scan[MAXT + 1];
+  __shared__ int64_t s_off[kMaxWorld];
   __shared__ unsigned long long s_hits;
   for (int i = threadIdx.x; i <= ra.n; i += blockDim.x) s_scan[i] = ra.scan[i];
   if (threadIdx.x == 0) s_hits = 0;
+  if (pa.p2p) {  // where this rank's keys start in each owner's received order
+    for (int o = threadIdx.x; o < rd.world; o += blockDim.x) {
+      int64_t acc = pa.off[o];
+      if (pa.dcnt) {  // sync-free: sum of the counts owner o received from ranks < me
+        acc = 0;
+        for (int src = 0; src < pa.me; ++src) acc += pa.dcnt[(size_t)src * rd.world + o];
+      }
+      s_off[o] = acc;
+    }
+  }
   __syncthreads();
   const int lane = threadIdx.x & 31;
   const int64_t N = s_scan[ra.n];
@@ -213,7 +225,7 @@ __global__ void __launch_bounds__(128) krs_kernel(const __grid_constant__ RArgs<
           if (flags) hit = flags[pos] != 0;
         } else {  // fused exchange: read the owner's answer row where it lies (peer HBM over NVLink)
           const int o = (int)(v >> 32);
-          const int64_t at = pa.off[o] + (int64_t)(v & 0xFFFFFFFFull);
+          const int64_t at = s_off[o] + (int64_t)(v & 0xFFFFFFFFull);
           src = pa.rows[o] + at * D;
           if (pa.flags[o]) hit = pa.flags[o][at] != 0;
         }

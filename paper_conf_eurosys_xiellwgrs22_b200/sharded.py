@@ -14,12 +14,14 @@ collective.  Every rank maps every owner's receive and answer buffers (CUDA IPC,
 access over NVLink).  The route's pack kernel stores each unique key straight into its
 owner's slot for this rank (fleche_route_p2p); a G x G counts all-gather (stream-ordered
 behind every rank's route, so it is also the "keys are in place" barrier) sizes the
-owner query over its per-source segments (fleche_query_keys_seg) and gives each rank its
-offset in every owner's answer order; after a one-element all-reduce (a stream-ordered
-barrier: every owner's answers are written; answers are double-buffered by batch parity)
-each requester's restore kernel (fleche_restore_p2p) reads its rows in place from the
-owners' HBM.  With the gloo backend (CPU / one-GPU tests) the small collectives go
-through host copies.
+owner query over its per-source segments (fleche_query_keys_seg_dev, reading the G x G
+counts matrix in device memory with a grid-strided launch) and gives each rank its
+offset in every owner's answer order, computed by the restore kernel on the device;
+after a one-element all-reduce (a stream-ordered barrier: every owner's answers are
+written; answers are double-buffered by batch parity) each requester's restore kernel
+(fleche_restore_p2p_dev) reads its rows in place from the owners' HBM.  With NCCL no step
+reads anything back to the host; with the gloo backend (CPU / one-GPU tests) the small
+collectives go through host copies.
 """
 from __future__ import annotations
 
@@ -92,6 +94,7 @@ class ShardedCache:
             self.peer_slots.append(base + me * n * 4)
         self.own_segs = [self.own_recv + src * n * 4 for src in range(W)]
         self.bar = torch.zeros(1, dtype=torch.int32, device="cpu" if self.cpu_coll else self.send_counts.device)
+        self.dC = torch.zeros(W * W, dtype=torch.int64, device=self.send_counts.device)  # routed counts [src][owner]
 
     def close(self):
         if getattr(self, "p2p", False) and getattr(self, "own_rows", None):
@@ -130,24 +133,25 @@ class ShardedCache:
         dist.all_reduce(self.bar, group=self.group)
 
     def query_p2p(self, ids, out, lengths=None):
-        """One batch through the fused exchange (see the module docstring)."""
+        """One batch through the fused exchange (see the module docstring).  With NCCL the
+        host never waits: the counts matrix is all-gathered into device memory and read there
+        by the owner query and the restore (fleche_*_dev); gloo (CPU tests) gathers through
+        host memory."""
         c, W, me = self.cache, self.world, self.rank
         par = self.batch & 1
         self.batch += 1
         # keys: the route's pack kernel stores them straight into the owners' slots (peer HBM)
         c.route_p2p(ids, W, self.seed, self.peer_slots, self.send_counts, lengths=lengths)
         # counts: all-gather (stream-ordered behind every rank's route: the keys are in place)
-        C = self._all_gather_counts()  # C[src][owner]
-        S = [int(x) for x in C[me]]
-        R = [int(x) for x in C[:, me]]
-        off = [int(C[:me, o].sum()) for o in range(W)]
-        ns, nr = sum(S), sum(R)
-        c.query_keys_seg(self.own_segs, R, self.own_rows[par], self.own_flags[par])
+        if self.cpu_coll:
+            self.dC.copy_(self._all_gather_counts().reshape(-1))
+        else:
+            dist.all_gather_into_tensor(self.dC, self.send_counts, group=self.group)  # C[src][owner], device
+        c.query_keys_seg_dev(self.own_segs, self.dC, me, self.own_rows[par], self.own_flags[par])
         self._barrier()  # every owner's answers of this batch are in place
         # rows: each requester reads its answers in place from the owners' HBM
-        c.restore_p2p(self.peer_rows[par], self.peer_flags[par], off, out)
-        self.last_exchange = {"sent_keys": ns, "recv_keys": nr, "p2p_bytes_out": ns * 4,
-                              "p2p_bytes_in": ns * (4 * self.d + 1)}
+        c.restore_p2p_dev(self.peer_rows[par], self.peer_flags[par], self.dC, me, out)
+        self.last_exchange = None  # the per-batch byte counts stay on the device (no host read)
         return self.last_exchange
 
     def query(self, ids, out, lengths=None):

@@ -32,7 +32,15 @@ def _worker(rank, world, port, name, q):
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
         w = configs.get("cfg0").with_(batch_size=64)
-        buf, tabs, cleanup = shm.shared_tables(name, w.cards, w.dims, 0, rank, dist.barrier)
+        def ago(x):
+            out = [None] * world
+            dist.all_gather_object(out, x)
+            return out
+        node = 0  # CPU test: both ranks on node 0 -> one copy, created by the lowest rank
+        creator = shm.creator_ranks(rank, node, ago)
+        assert creator == (rank == 0)
+        buf, tabs, cleanup = shm.shared_tables(name, w.cards, w.dims, 0, rank, dist.barrier, node=node,
+                                               creator=creator)
         orc = O.Oracle(w.cards, w.dims, tabs, w.cache_bytes)
         outs = []
         for b in range(4):

@@ -89,6 +89,42 @@ def test_sharded_one_rank_nccl_bit_exact_and_exact_hits():
         dist.destroy_process_group()
 
 
+def test_sharded_p2p_one_rank_nccl_sync_free():
+    """The fused exchange on a real NCCL group (one rank): counts all-gathered into device
+    memory and read there by the owner query (grid-strided over the device-side total) and
+    the restore, no host read per batch (fleche_query_keys_seg_dev / fleche_restore_p2p_dev);
+    out bit-exact and per-lookup hits equal to the set oracle's every batch."""
+    import torch.distributed as dist
+
+    import paper_conf_eurosys_xiellwgrs22_b200 as fl
+    from paper_conf_eurosys_xiellwgrs22_b200.sharded import ShardedCache
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    dist.init_process_group("nccl", init_method=f"tcp://127.0.0.1:{port}", rank=0, world_size=1,
+                            device_id=torch.device("cuda", 0))
+    try:
+        w = configs.get("cfg0").with_(cache_frac=0.25, invalid_ppm=3000)
+        tabs = _tables(w)
+        gpu = fl.FlatCache(w.cards, w.dims, tabs, w.cache_bytes, w.batch_size * w.n, 0, 1.0, 0, H.HASH_SEED)
+        sc = ShardedCache(gpu, row_floats=w.dims[0], p2p=True)
+        orc = O.Oracle(w.cards, w.dims, tabs, w.cache_bytes, O.MODE_SETASSOC, hash_seed=H.HASH_SEED)
+        for b in range(20):
+            bt = w.batch(b)
+            ids = [torch.from_numpy(x).cuda() for x in bt.ids]
+            out = torch.full((gpu.out_floats([x.size for x in bt.ids]),), float("nan"), device="cuda")
+            h0 = gpu.shard_stats()["hits"]
+            o0 = orc.stats()["hits"]
+            sc.query(ids, out)
+            torch.cuda.synchronize()
+            assert H.bits_equal(out.cpu().numpy(), orc.query(bt.ids)), b
+            assert gpu.shard_stats()["hits"] - h0 == orc.stats()["hits"] - o0, b
+        sc.close()
+    finally:
+        dist.destroy_process_group()
+
+
 def test_p2p_two_processes_one_gpu(tmp_path):
     """The fused exchange (fleche_restore_p2p: every requester reads its rows in place from
     the owners' answer buffers through CUDA IPC mappings) with two ranks sharing cuda:0
