@@ -1436,6 +1436,8 @@ fleche_status launch_keys(fleche_ctx* c, const uint32_t* keys, int64_t count, fl
   ka.out = rows;
   ka.ncls = 1;
   ka.cls_dim[0] = c->max_dim;
+  qa.ncls = 1;
+  qa.ha_bell = c->dv.ha;  // host-assisted owner: KQ's last CTA rings the doorbell (as in launch_query)
   fleche_status st = prof_event(c, s, true, 4);
   if (st != FLECHE_OK) return st;
   if (dcnt) {  // count unknown on the host: a capacity-sized, grid-strided launch (TD = 0: no TMA variant)

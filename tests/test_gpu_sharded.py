@@ -89,7 +89,8 @@ def test_sharded_one_rank_nccl_bit_exact_and_exact_hits():
         dist.destroy_process_group()
 
 
-def test_sharded_p2p_one_rank_nccl_sync_free():
+@pytest.mark.parametrize("ha", [False, True])
+def test_sharded_p2p_one_rank_nccl_sync_free(monkeypatch, ha):
     """The fused exchange on a real NCCL group (one rank): counts all-gathered into device
     memory and read there by the owner query (grid-strided over the device-side total) and
     the restore, no host read per batch (fleche_query_keys_seg_dev / fleche_restore_p2p_dev);
@@ -107,7 +108,9 @@ def test_sharded_p2p_one_rank_nccl_sync_free():
     try:
         w = configs.get("cfg0").with_(cache_frac=0.25, invalid_ppm=3000)
         tabs = _tables(w)
-        gpu = fl.FlatCache(w.cards, w.dims, tabs, w.cache_bytes, w.batch_size * w.n, 0, 1.0, 0, H.HASH_SEED)
+        monkeypatch.setenv("FLECHE_HA_MIN_ROWS", "0")  # cfg0's few misses per batch: assist every batch
+        gpu = fl.FlatCache(w.cards, w.dims, tabs, w.cache_bytes, w.batch_size * w.n, 0, 1.0, 0, H.HASH_SEED,
+                           fl.binding.FLAG_HOST_ASSIST if ha else 0)
         sc = ShardedCache(gpu, row_floats=w.dims[0], p2p=True)
         orc = O.Oracle(w.cards, w.dims, tabs, w.cache_bytes, O.MODE_SETASSOC, hash_seed=H.HASH_SEED)
         for b in range(20):
@@ -120,6 +123,9 @@ def test_sharded_p2p_one_rank_nccl_sync_free():
             torch.cuda.synchronize()
             assert H.bits_equal(out.cpu().numpy(), orc.query(bt.ids)), b
             assert gpu.shard_stats()["hits"] - h0 == orc.stats()["hits"] - o0, b
+        st = gpu.stats()
+        if ha:  # the owner's misses went through the host threads, none timed out
+            assert st["assisted_rows"] > 0 and st["assist_timeouts"] == 0, st
         sc.close()
     finally:
         dist.destroy_process_group()
