@@ -110,19 +110,21 @@ typedef struct {
  * lies in the host tables.  On this platform scattered zero-copy reads are capped by
  * address translation (~80 M rows/s beyond a ~1 GiB span), while host cores
  * gather scattered rows at ~60 GB/s, so by DEFAULT a ctx whose host tier spans >= 1 GiB
- * (uniform row width, >= 8 host CPUs) runs host threads that gather a share of the batch's
+ * (>= 8 host CPUs; not the static per-table or per-table-launch ablations) runs host
+ * threads that gather a share of the batch's
  * unique missed rows into a contiguous pinned staging buffer, which the miss kernel reads
  * over the link at its full rate while it reads the rest zero-copy itself (two paths at
- * once).  HOST_ASSIST forces it on (also for mixed widths or small tiers),
+ * once).  HOST_ASSIST forces it on (also for small tiers),
  * NO_HOST_ASSIST off.  Requests travel GPU -> host through pinned memory, tagged with the
  * batch epoch; the query kernel's last CTA rings the doorbell; ONE miss-kernel warp polls
  * the threads' progress words and mirrors them into HBM for the others (no host sync, no
  * extra launch: the path stays asynchronous and graph-capturable).  Blocks not staged
  * within FLECHE_HA_TIMEOUT_US (default 2000) are read zero-copy from the tables, so
  * correctness never depends on the threads.  Env: FLECHE_HA_THREADS (default
- * min(12, CPUs - 4)), FLECHE_HA_STAGE_KB (staging per epoch parity, default 131072; rows
- * beyond it are read zero-copy), FLECHE_HA_FRAC (share of the batch's staging blocks the
- * host threads take, default 0.8, or 0.85 for host tiers over 32 GiB), FLECHE_HA_MIN_ROWS
+ * min(12, CPUs - 4)), FLECHE_HA_STAGE_KB (staging per epoch parity, default 131072, or
+ * 524288 with several row widths, shared equally by the widths; a width's misses beyond its
+ * rows are read zero-copy), FLECHE_HA_FRAC (fixes the share of the staging blocks the host
+ * threads take; default: tuned online, see fleche_stats.ui_share_ppm), FLECHE_HA_MIN_ROWS
  * (batches with fewer unique misses stay all zero-copy, default 1024).  Not with
  * PER_TABLE_LAUNCH (FLECHE_EINVAL).  `out`, hits and every cache decision are identical
  * with and without it; only where the missed rows are read from changes. */

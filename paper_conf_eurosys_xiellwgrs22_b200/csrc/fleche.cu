@@ -43,6 +43,7 @@ struct HostAssist {
   unsigned long long* bell = nullptr;  // doorbell (epoch)
   uint32_t* ready = nullptr;           // [2][blk_cap] ready word of each staging block (= epoch once staged)
   uint32_t blk_cap = 0;
+  uint32_t rbase[8] = {}, rcap[8] = {};  // staging rows of width class c: [rbase, rbase + rcap)
   float* stage = nullptr;              // [2][stage_floats]
   uint32_t req_cap = 0;
   bool nt_stores = true;  // FLECHE_HA_NT=0: plain memcpy into the staging buffer (A/B)
@@ -351,14 +352,6 @@ void ha_worker(HostAssist* h, int me) {
     uint32_t* ready = h->ready + (size_t)par * h->blk_cap;
     const HaReq* rq = h->req + (size_t)par * h->req_cap;
     float* st = h->stage + (size_t)par * h->stage_floats;
-    uint64_t lo_all = ~0ull, hi_all = 0;
-    for (int c = 0; c < 8; ++c)
-      if (d.cnt[c]) {
-        lo_all = std::min<uint64_t>(lo_all, d.off[c]);
-        hi_all = std::max<uint64_t>(hi_all, (uint64_t)d.off[c] + d.cnt[c]);
-      }
-    if (hi_all == 0 || hi_all > h->req_cap) continue;
-    const uint64_t kcut = d.kcut;  // blocks >= kcut: KM reads them from the tables itself
     // a request of this batch (KQ wrote it without a system fence: wait until both halves
     // carry this batch's tags, read twice so a torn read is never taken); false after ~1 ms
     auto fetch = [&](uint64_t i, HaReq* out) -> bool {
@@ -397,22 +390,22 @@ void ha_worker(HostAssist* h, int me) {
       if (const float* p = src_of(r, &dd, &so))
         for (int b = 0; b < dd * 4; b += 64) __builtin_prefetch((const char*)p + b, 0, 0);
     };
-    const uint64_t kb0 = lo_all / kHaBlock, kb1 = (hi_all - 1) / kHaBlock;
-    const uint64_t kend = std::min<uint64_t>(kb1 + 1, kcut);
-    // static ownership (block k belongs to thread k % nthreads in every batch, taken in
-    // increasing k): a thread that stalls past the GPU's give-up can only ever overwrite
-    // slots of its own blocks, which it republishes only after rewriting them
-    for (uint64_t kb = kb0; kb < kend && !lost; ++kb) {
-      if (kb % (uint64_t)h->nthreads != (uint64_t)me) continue;
-      if (h->delay_ns) {  // a stalled host thread (tests): its blocks time out on the GPU
-        struct timespec ts = {(time_t)(h->delay_ns / 1000000000ull), (long)(h->delay_ns % 1000000000ull)};
-        nanosleep(&ts, nullptr);
-      }
-      for (int c = 0; c < 8; ++c) {  // the rows of every class region that overlaps block kb
-        if (!d.cnt[c]) continue;
-        const uint64_t lo = std::max<uint64_t>(kb * kHaBlock, d.off[c]);
-        const uint64_t hi = std::min<uint64_t>(kb * kHaBlock + kHaBlock, (uint64_t)d.off[c] + d.cnt[c]);
-        if (lo >= hi) continue;
+    // static ownership (staging block b = rows [64b, 64b + 64) belongs to thread b % nthreads
+    // in every batch, taken in increasing b): a thread that stalls past the GPU's give-up can
+    // only ever overwrite its own blocks, which it republishes only after rewriting them
+    // (ADVICE r1); class c stages its first min(cnt, rcap) misses in rows [rbase_c, ...),
+    // the host threads take blocks below hcut_c of each class
+    for (int c = 0; c < 8 && !lost; ++c) {
+      if (!d.cnt[c] || !d.hcut[c]) continue;
+      const uint64_t rb = h->rbase[c], nrow = std::min<uint64_t>(d.cnt[c], h->rcap[c]);
+      const uint64_t kb0 = rb / kHaBlock, kend = kb0 + std::min<uint64_t>(d.hcut[c], (nrow + kHaBlock - 1) / kHaBlock);
+      for (uint64_t kb = kb0; kb < kend && !lost; ++kb) {
+        if (kb % (uint64_t)h->nthreads != (uint64_t)me) continue;
+        if (h->delay_ns) {  // a stalled host thread (tests): its blocks time out on the GPU
+          struct timespec ts = {(time_t)(h->delay_ns / 1000000000ull), (long)(h->delay_ns % 1000000000ull)};
+          nanosleep(&ts, nullptr);
+        }
+        const uint64_t lo = kb * kHaBlock, hi = std::min<uint64_t>(lo + kHaBlock, rb + nrow);
         constexpr uint64_t PF = 12;  // rows prefetched ahead (~4 lines each: keeps the line fill buffers busy)
         for (uint64_t i = lo; i < std::min(hi, lo + PF); ++i) prefetch(i);
         for (uint64_t i = lo; i < hi; ++i) {
@@ -432,17 +425,17 @@ void ha_worker(HostAssist* h, int me) {
             else memcpy(st + so, p, (size_t)dd * 4u);
           }
         }
-      }
-      if (h->nt_stores) _mm_sfence();  // streaming stores are weakly ordered: drain them before the ready word
-      if (lost) break;
-      __atomic_store_n(ready + kb, e, __ATOMIC_RELEASE);
+        if (h->nt_stores) _mm_sfence();  // streaming stores are weakly ordered: drain them before the ready word
+        if (lost) break;
+        __atomic_store_n(ready + kb, e, __ATOMIC_RELEASE);
 #ifdef FLECHE_EXPERIMENTS
-      if (h->exp_pub) {
-        struct timespec ts;
-        clock_gettime(CLOCK_REALTIME, &ts);
-        h->exp_pub[kb] = (uint64_t)ts.tv_sec * 1000000000ull + (uint64_t)ts.tv_nsec;
-      }
+        if (h->exp_pub) {
+          struct timespec ts;
+          clock_gettime(CLOCK_REALTIME, &ts);
+          h->exp_pub[kb] = (uint64_t)ts.tv_sec * 1000000000ull + (uint64_t)ts.tv_nsec;
+        }
 #endif
+      }
     }
 #ifdef FLECHE_EXPERIMENTS
     if (me < 64) {
@@ -912,12 +905,13 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   // KM: enough warps for the expected unique misses, km_bps CTAs of 4 warps per SM, and no
   // more CTAs than fit at once (cooperative launch: its grid barrier needs them all resident)
   // host-assisted miss fetch: forced by the flag, else by default on a large host tier
-  // (the translation-bound regime of scattered zero-copy reads) with uniform rows
+  // (the translation-bound regime of scattered zero-copy reads): cfg2 +25-33 %, cfg5 +45 %,
+  // cfg4 (mixed widths) +27 % over zero-copy (profiles/bench_r02_*)
   uint64_t tier_bytes = 0;
   for (int t = 0; t < n; ++t) tier_bytes += (uint64_t)c->card[t] * (uint64_t)c->dims[t] * 4u;
   const unsigned ncpu = std::thread::hardware_concurrency();
   const bool use_ha = (cfg->flags & FLECHE_FLAG_HOST_ASSIST) ||
-                      (!(cfg->flags & FLECHE_FLAG_NO_HOST_ASSIST) && !bytes && !part && !c->per_table_launch &&
+                      (!(cfg->flags & FLECHE_FLAG_NO_HOST_ASSIST) && !part && !c->per_table_launch &&
                        tier_bytes >= (1ull << 30) && ncpu >= 8 && !(getenv("FLECHE_HA") && !atoi(getenv("FLECHE_HA"))));
   c->km_smem = (size_t)kKmWarps * ((bytes ? kKmSmemF4 : 0) + (use_ha ? kHaSmemF4 : 0)) * sizeof(float4);
   {
@@ -959,9 +953,23 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
     };
     h->nthreads = (int)std::max<uint64_t>(
         1, std::min<uint64_t>(kHaMaxThreads, env_u("FLECHE_HA_THREADS", std::max(1u, std::min(12u, ncpu > 4 ? ncpu - 4 : 1)))));
-    h->req_cap = (uint32_t)cfg->max_lookups;  // requests are indexed like the miss list
+    // staging: rows of the widest width, shared equally by the width classes (whole blocks
+    // each); requests are indexed by staging row.  Default 128 MiB per epoch parity for one
+    // width, 512 MiB for several (cfg4 stages ~470K misses per batch)
+    const uint32_t ncls = (uint32_t)c->cls_dim.size();
+    h->stage_floats = std::max<uint64_t>(1024, env_u("FLECHE_HA_STAGE_KB", ncls > 1 ? 524288 : 131072) << 8);
+    {
+      const uint64_t rows = std::min<uint64_t>(h->stage_floats / (uint64_t)c->max_dim,
+                                               (uint64_t)cfg->max_lookups + kHaBlock * ncls);
+      const uint64_t per = (rows / ncls) / kHaBlock * kHaBlock;
+      for (uint32_t k = 0; k < 8; ++k) {
+        h->rbase[k] = k < ncls ? (uint32_t)(k * per) : 0u;
+        h->rcap[k] = k < ncls ? (uint32_t)per : 0u;
+      }
+      h->req_cap = (uint32_t)(per * ncls);
+      h->stage_floats = (uint64_t)h->req_cap * (uint64_t)c->max_dim;
+    }
     h->blk_cap = h->req_cap / kHaBlock + 2;
-    h->stage_floats = std::max<uint64_t>(1024, env_u("FLECHE_HA_STAGE_KB", 131072) << 8);
     const size_t o_req = 0, o_desc = o_req + 2 * sizeof(HaReq) * (size_t)h->req_cap, o_bell = o_desc + 2 * sizeof(HaDesc),
                  o_ready = (o_bell + 8 + 127) & ~size_t(127), o_stage = (o_ready + 8ull * h->blk_cap + 255) & ~size_t(255),
                  total = o_stage + 2 * 4 * h->stage_floats;
@@ -986,6 +994,11 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
     dv.ha_bell = (unsigned long long*)(db + o_bell);
     dv.ha_ready = (uint32_t*)(db + o_ready);
     dv.ha_blk_cap = h->blk_cap;
+    dv.ha_row_floats = (uint32_t)c->max_dim;
+    for (int k = 0; k < 8; ++k) {
+      dv.ha_rbase[k] = h->rbase[k];
+      dv.ha_rcap[k] = h->rcap[k];
+    }
     if (cudaMalloc((void**)&dv.ha_seen, 4ull * h->blk_cap) != cudaSuccess ||
         cudaMemset(dv.ha_seen, 0, 4ull * h->blk_cap) != cudaSuccess)
       return fail(FLECHE_ENOMEM);

@@ -176,9 +176,9 @@ __host__ __device__ __forceinline__ bool ha_req_current(const HaReq& r, uint32_t
 }
 struct HaDesc {            // written by the doorbell ringer, read by the host threads
   uint32_t epoch;
-  uint32_t cnt[8];         // unique misses of width class c (list indices off[c] .. off[c] + cnt[c])
-  uint32_t off[8];
-  uint32_t kcut;           // split: the host threads stage blocks < kcut, KM reads blocks >= kcut itself
+  uint32_t cnt[8];         // unique misses of width class c this batch
+  uint32_t hcut[8];        // split: the host threads stage class c's blocks < hcut[c], KM reads the rest itself
+  uint32_t pad;
   uint32_t epoch2;         // = epoch, written last: the host accepts the descriptor once both match
 };
 
@@ -220,7 +220,11 @@ struct Dev {
   uint32_t* ha_ready;          // [2][ha_blk_cap] (host memory) epoch of each staging block once staged
   uint32_t* ha_seen;           // [ha_blk_cap] (HBM) the poller warp's mirror of ha_ready[epoch & 1]
   float* ha_stage;             // [2][ha_stage_floats]
-  uint32_t ha_req_cap, ha_blk_cap;
+  uint32_t ha_req_cap, ha_blk_cap;  // staging rows (= request slots) and blocks per epoch parity
+  uint32_t ha_rbase[8];        // first staging row of width class c (a multiple of kHaBlock)
+  uint32_t ha_rcap[8];         // staging rows of class c (a multiple of kHaBlock): its misses beyond go zero-copy
+  uint32_t ha_row_floats;      // stride of a staging row (the widest row)
+  uint32_t ha_pad3;
   uint64_t ha_stage_floats;
   uint64_t ha_timeout_ns;
   uint32_t ha_frac_fixed;      // 1 = FLECHE_HA_FRAC fixed the host threads' share (no tuning loop)
@@ -412,19 +416,14 @@ __device__ __forceinline__ void st_release_gpu_u64(unsigned long long* p, unsign
   asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
-// Host-assisted geometry of a batch: staging blocks [kb0, kend) go to the host threads
-// (kend = the split point kcut, clipped to the batch's last block + 1).
-__device__ __forceinline__ void ha_range(const Dev& dv, const uint32_t (&cnt)[8], const int64_t* cls_off, int ncls,
-                                         uint32_t& kb0, uint32_t& kb1) {
-  uint32_t lo = 0xFFFFFFFFu, hi = 0;
-#pragma unroll
-  for (int c = 0; c < 8; ++c) {  // compile-time indices: cnt stays in registers
-    if (c >= ncls || !cnt[c]) continue;
-    lo = min(lo, (uint32_t)cls_off[c]);
-    hi = max(hi, (uint32_t)cls_off[c] + cnt[c]);
-  }
-  kb0 = hi ? lo / kHaBlock : 0u;
-  kb1 = hi ? (hi - 1) / kHaBlock : 0u;
+// Host-assisted geometry.  Staging row r = ha_rbase[c] + j holds the j-th unique miss of
+// width class c (its class-local miss-list index), for j < ha_rcap[c]; block b = r / 64 is
+// always the same 64 rows of staging memory, owned by host thread b % T in every batch
+// (a stalled thread can only ever rewrite its own blocks, whatever the batch geometry).
+// The host threads take class c's blocks below hcut (its share of the class's staged rows).
+__host__ __device__ __forceinline__ uint32_t ha_hcut(uint32_t cnt, uint32_t rcap, uint32_t frac_q16) {
+  const uint32_t nb = ((cnt < rcap ? cnt : rcap) + kHaBlock - 1) / kHaBlock;
+  return (uint32_t)(((unsigned long long)nb * frac_q16 + 65535ull) >> 16);
 }
 
 // The poller warp: mirror the ready words of staging blocks [kb0, kend) into HBM until all
@@ -439,40 +438,54 @@ __device__ __forceinline__ uint32_t ld_relaxed_sys_u32(const uint32_t* p) {
   asm volatile("ld.relaxed.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
   return v;
 }
-__device__ __forceinline__ void ha_poll(const Dev& dv, uint32_t epoch, uint32_t kb0, uint32_t kend, int lane) {
+// Ready words of the batch's host blocks: class c's blocks [rbase_c / 64, + hcut_c).
+struct HaBlocks {
+  uint32_t lo[8], n[8];
+  int ncls;
+};
+__device__ __forceinline__ void ha_poll(const Dev& dv, uint32_t epoch, const HaBlocks& hb, int lane) {
   const uint32_t* ready = dv.ha_ready + (size_t)(epoch & 1u) * dv.ha_blk_cap;
   const unsigned long long t0 = globaltimer_ns();
   unsigned long long t_progress = 0;  // last time a new block was seen ready (0: none yet)
-  uint32_t lo = kb0;                  // every block below lo has been mirrored
-  while (lo < kend) {
-    uint32_t first_missing = kend, fresh = 0;
-    for (uint32_t k0 = lo; k0 < kend; k0 += 32 * 4) {
-      uint32_t v[4];
+  uint32_t lo[8];
 #pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        const uint32_t k = k0 + 32 * q + lane;
-        v[q] = (k < kend && ld_acquire_gpu_u32(dv.ha_seen + k) != epoch) ? ld_relaxed_sys_u32(ready + k) : ~0u;
-      }
-      uint32_t newly = 0;
+  for (int c = 0; c < 8; ++c) lo[c] = c < hb.ncls ? hb.lo[c] : 0u;  // class c: blocks below lo[c] mirrored
+  while (true) {
+    uint32_t fresh = 0, missing = 0;
 #pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        const uint32_t k = k0 + 32 * q + lane;
-        if (v[q] == epoch) newly |= 1u << q;
-        const unsigned miss = __ballot_sync(kFull, k < kend && v[q] != ~0u && v[q] != epoch);
-        if (miss) first_missing = min(first_missing, k0 + 32 * q + (uint32_t)(__ffs(miss) - 1));
-      }
-      if (__any_sync(kFull, newly)) {
-        asm volatile("fence.acq_rel.sys;" ::: "memory");  // the rows staged before these ready words
+    for (int c = 0; c < 8; ++c) {
+      if (c >= hb.ncls) continue;
+      const uint32_t kend = hb.lo[c] + hb.n[c];
+      uint32_t first_missing = kend;
+      for (uint32_t k0 = lo[c]; k0 < kend; k0 += 32 * 4) {
+        uint32_t v[4];
 #pragma unroll
-        for (int q = 0; q < 4; ++q)
-          if (newly & (1u << q)) st_release_gpu_u32(dv.ha_seen + k0 + 32 * q + lane, epoch);
-        fresh += __popc(__ballot_sync(kFull, newly != 0));
+        for (int q = 0; q < 4; ++q) {
+          const uint32_t k = k0 + 32 * q + lane;
+          v[q] = (k < kend && ld_acquire_gpu_u32(dv.ha_seen + k) != epoch) ? ld_relaxed_sys_u32(ready + k) : ~0u;
+        }
+        uint32_t newly = 0;
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          const uint32_t k = k0 + 32 * q + lane;
+          if (v[q] == epoch) newly |= 1u << q;
+          const unsigned miss = __ballot_sync(kFull, k < kend && v[q] != ~0u && v[q] != epoch);
+          if (miss) first_missing = min(first_missing, k0 + 32 * q + (uint32_t)(__ffs(miss) - 1));
+        }
+        if (__any_sync(kFull, newly)) {
+          asm volatile("fence.acq_rel.sys;" ::: "memory");  // the rows staged before these ready words
+#pragma unroll
+          for (int q = 0; q < 4; ++q)
+            if (newly & (1u << q)) st_release_gpu_u32(dv.ha_seen + k0 + 32 * q + lane, epoch);
+          fresh += __popc(__ballot_sync(kFull, newly != 0));
+        }
       }
+      lo[c] = first_missing;
+      if (first_missing < kend) missing = 1;
     }
+    if (!missing) break;
     const unsigned long long now = globaltimer_ns();
     if (fresh) t_progress = now;
-    lo = first_missing;
-    if (lo >= kend) break;
     if (now - t0 > dv.ha_timeout_ns || (t_progress && now - t_progress > kHaStallNs)) {
       if (lane == 0) st_release_gpu_u32(&dv.ctl->ha_abort, epoch);
       break;
@@ -491,10 +504,10 @@ __device__ __forceinline__ bool ha_wait_block(const Dev& dv, uint32_t epoch, uin
   }
 }
 
-// Host-assisted split: the batch's miss list spans staging blocks [kb0, kb1]; the host
-// threads gather the first ceil(frac * nblocks) of them while KM's other warps read the
-// rest zero-copy from the tables at the same time (two independent paths to the rows:
-// host cores + contiguous link reads, and the GPU's own translated reads).
+// Host-assisted split: the host threads gather the first ceil(frac * nblocks) staging
+// blocks of every class while KM's other warps read the rest zero-copy from the tables at
+// the same time (two independent paths to the rows: host cores + contiguous link reads,
+// and the GPU's own translated reads).
 // Host-assisted fetch active for this batch: enough unique misses (FLECHE_HA_MIN_ROWS) and
 // a non-zero share.  Otherwise KM takes the plain (address-ordered) zero-copy path and the
 // host threads are not woken.
@@ -503,22 +516,6 @@ __device__ __forceinline__ bool ha_active(const Dev& dv, const KMArgs& ka, int p
   uint32_t total = 0;
   for (int c = 0; c < ka.ncls; ++c) total += *(volatile uint32_t*)&dv.ctl->counts[par][c];
   return total >= dv.ha_min_rows;
-}
-
-__device__ __forceinline__ uint32_t ha_kcut(const Dev& dv, const KMArgs& ka, int par) {
-  uint32_t lo = 0xFFFFFFFFu, hi = 0;
-  for (int c = 0; c < ka.ncls; ++c) {
-    const uint32_t n = *(volatile uint32_t*)&dv.ctl->counts[par][c];
-    if (!n) continue;
-    lo = min(lo, (uint32_t)ka.cls_off[c]);
-    hi = max(hi, (uint32_t)ka.cls_off[c] + n);
-  }
-  if (hi == 0) return 0;
-  const uint32_t kb0 = lo / kHaBlock, nb = (hi - 1) / kHaBlock - kb0 + 1;
-  uint32_t total = 0;
-  for (int c = 0; c < ka.ncls; ++c) total += *(volatile uint32_t*)&dv.ctl->counts[par][c];
-  if (total < dv.ha_min_rows) return kb0;  // small batch: the round trip to the host threads is not hidden
-  return kb0 + (uint32_t)(((unsigned long long)nb * *(volatile uint32_t*)&dv.ctl->ha_frac_q16 + 65535ull) >> 16);
 }
 
 // Programmatic dependent launch (sm_90+): the batch's kernels are launched with
@@ -895,22 +892,22 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
       b = __shfl_sync(kFull, b, leader);
       uint64_t hst = kNoStage;
       if (kind == 1) {
-        const uint32_t r = b + __popc(grp & lt);
-        const int64_t li = qa.cls_off[cls] + r;  // miss-list index = request index
-        // host-assisted staging slot = the list index times the widest row: every staging
-        // block (kHaBlock list indices) owns a fixed region, written only by the host
-        // thread that owns the block, batch after batch (no slot of a timed-out block can
-        // be handed to another thread's block); rows past the buffer are read zero-copy
-        if (dv.ha && (uint64_t)(li + 1) * (uint64_t)dv.dim <= dv.ha_stage_floats) hst = (uint64_t)li * dv.dim;
+        const uint32_t r = b + __popc(grp & lt);  // the miss's index within its width class
+        const int64_t li = qa.cls_off[cls] + r;    // miss-list index
+        // host-assisted: staging row ha_rbase[cls] + r (one request slot each); a class's
+        // misses past its ha_rcap rows are read zero-copy (see ha_hcut for the ownership)
+        const bool staged = dv.ha && r < dv.ha_rcap[cls];
+        const uint32_t srow = staged ? dv.ha_rbase[cls] + r : 0u;
+        if (staged) hst = (uint64_t)srow * dv.ha_row_floats;
         dv.miss[li] = MissRec{off, fk, scr, qa.t0 + t, 0, hst};
         dv.owner_off[scr] = off;
 #ifdef FLECHE_EXPERIMENTS
         if (dv.exp_mode != 4)
 #endif
-        if (dv.ha)  // published by KM's doorbell (after this grid completes)
+        if (staged)  // the host threads' request, tagged with the epoch (no fence needed)
         {
           const HaReq rq = ha_req_make(qa.t0 + t, id, hst, epoch);
-          asm volatile("st.global.v2.u64 [%0], {%1, %2};" ::"l"(dv.ha_req + (size_t)par * dv.ha_req_cap + li),
+          asm volatile("st.global.v2.u64 [%0], {%1, %2};" ::"l"(dv.ha_req + (size_t)par * dv.ha_req_cap + srow),
                        "l"(rq.tid), "l"(rq.stage)
                        : "memory");
         }
@@ -981,15 +978,13 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
         }
         const uint32_t frac = *(volatile uint32_t*)&dv.ctl->ha_frac_q16;  // KM reads the same value
         if (frac && total >= dv.ha_min_rows) {  // KM's ha_active() takes the same decision
-          uint32_t kb0, kb1;
-          ha_range(dv, cnt, qa.cls_off, qa.ncls, kb0, kb1);
           HaDesc hd;
           hd.epoch = epoch;
           for (int c = 0; c < 8; ++c) {
             hd.cnt[c] = cnt[c];
-            hd.off[c] = c < qa.ncls ? (uint32_t)qa.cls_off[c] : 0u;
+            hd.hcut[c] = c < qa.ncls ? ha_hcut(cnt[c], dv.ha_rcap[c], frac) : 0u;
           }
-          hd.kcut = kb0 + (uint32_t)(((unsigned long long)(kb1 - kb0 + 1u) * frac + 65535ull) >> 16);
+          hd.pad = 0;
           hd.epoch2 = epoch;
           dv.ha_desc[par] = hd;  // no system fence: the host re-reads until both epoch fields match
           asm volatile("st.relaxed.sys.global.u64 [%0], %1;" ::"l"(dv.ha_bell), "l"((unsigned long long)epoch) : "memory");
@@ -1217,38 +1212,35 @@ template <bool BYTES, int D>
 __device__ __forceinline__ void km_ha(const Dev& dv, float* __restrict__ out, const MissRec* __restrict__ mlist,
                                       uint32_t epoch, uint32_t nmiss, int lane, uint32_t gw, uint32_t nw, unsigned& ins,
                                       unsigned& ev, unsigned& byp, long long& docc, unsigned long long& hostb,
-                                      float4* hsm, float4* cbuf, unsigned& harows, unsigned& hato, uint32_t kcut,
-                                      uint32_t bkb0) {
+                                      float4* hsm, float4* cbuf, unsigned& harows, unsigned& hato, int cls,
+                                      uint32_t hcut) {
   constexpr int VEC = D / 4;
   constexpr int ROWS0 = (kHaSmemF4 / VEC) < kHaBlock ? (kHaSmemF4 / VEC) : kHaBlock;  // rows that fit the warp's smem
   constexpr int ROWS = ROWS0 < 16 ? ROWS0 : 16;  // rows per piece: one warp per piece, pieces of a block in parallel
   constexpr int PPB = kHaBlock / ROWS;           // pieces per staging block
   constexpr int PER_LANE = ROWS * VEC / 32;      // float4 per lane per piece
   constexpr int INFL = PER_LANE < 16 ? PER_LANE : 16;
-  const uint32_t off = (uint32_t)(mlist - dv.miss);
-  const uint32_t kb0 = off / kHaBlock, kb1 = (off + nmiss - 1) / kHaBlock;
   const float* stage = dv.ha_stage + (size_t)(epoch & 1u) * dv.ha_stage_floats;
-  // work unit = one piece of one block: every piece of the batch has a warp of its own
-  // (a staged piece starts as soon as its block is ready; the zero-copy blocks >= kcut
-  // get the whole grid's memory-level parallelism, not one warp per 64 rows)
-  // pieces per warp unit: as fine as the grid allows (one piece per warp while there are
-  // enough warps, cfg2 +8 %), coarser for big batches (consecutive pieces of a block in one
-  // warp, cfg5 +8 %); FLECHE_HA_UNIT_PIECES fixes it (A/B)
-  const uint32_t npieces = (kb1 - kb0 + 1) * PPB;
+  // work unit = pieces of this class's miss list (class-local index j; a piece never
+  // straddles a 64-row staging block): a staged piece starts as soon as its block is
+  // ready, and the zero-copy pieces (blocks >= hcut, or past the class's staging rows) get
+  // the whole grid's memory-level parallelism, not one warp per 64 rows.  Pieces per
+  // unit: as fine as the grid allows (one piece per warp while there are enough warps,
+  // cfg2 +8 %), coarser for big batches (cfg5 +8 %); FLECHE_HA_UNIT_PIECES fixes it (A/B)
+  const uint32_t npieces = (nmiss + ROWS - 1) / ROWS;
   const uint32_t ppu = dv.ha_unit_pieces ? min((uint32_t)PPB, dv.ha_unit_pieces)
                                          : min((uint32_t)PPB, max(1u, (npieces + nw - 1) / nw));
-  for (uint32_t u0 = gw * ppu; u0 < (kb1 - kb0 + 1) * PPB; u0 += nw * ppu)
-  for (uint32_t u = u0; u < min(u0 + ppu, (kb1 - kb0 + 1) * PPB); ++u) {
-    const uint32_t kb = kb0 + u / PPB, pc = u % PPB;
-    const uint32_t plo_abs = kb * kHaBlock + pc * ROWS;  // the piece's list indices [plo_abs, plo_abs + ROWS)
-    const uint32_t lo_abs = max(plo_abs, off), hi_abs = min(plo_abs + (uint32_t)ROWS, off + nmiss);
-    if (lo_abs >= hi_abs) continue;  // the piece lies outside this width's region
-    const uint32_t blo = lo_abs - off, bhi = hi_abs - off;
+  const uint32_t rcap = dv.ha_rcap[cls], blk0 = dv.ha_rbase[cls] / kHaBlock;
+  for (uint32_t u0 = gw * ppu; u0 < npieces; u0 += nw * ppu)
+  for (uint32_t u = u0; u < min(u0 + ppu, npieces); ++u) {
+    const uint32_t blo = u * ROWS, bhi = min(blo + (uint32_t)ROWS, nmiss);
+    const uint32_t hb = blo / kHaBlock, pc = (blo % kHaBlock) / ROWS;  // class-local staging block
+    const uint32_t kb = blk0 + hb;                                     // its absolute block id
     int ok = 0;
 #ifdef FLECHE_EXPERIMENTS
     if (dv.exp_blk && lane == 0 && pc == 0) dv.exp_blk[kb * 4 + 0] = globaltimer_ns();
 #endif
-    if (lane == 0 && kb < kcut) {  // the host threads' share; blocks >= kcut are read from the tables
+    if (lane == 0 && blo < rcap && hb < hcut) {  // the host threads' share; the rest from the tables
       ok = ha_wait_block(dv, epoch, kb);
       if (!ok && pc == 0) ++hato;
     }
@@ -1602,19 +1594,16 @@ __global__ void __launch_bounds__(128, 4) km_kernel(const __grid_constant__ Dev 
   const int lane = threadIdx.x & 31;
   if (dv.ha && blockIdx.x == 0 && threadIdx.x == 0) dv.ctl->km_t0 = globaltimer_ns();  // (ui_tune)
   const bool use_ha = ha_active(dv, ka, par);  // KQ's last CTA rang the doorbell (same test)
+  const uint32_t frac = use_ha ? *(volatile uint32_t*)&dv.ctl->ha_frac_q16 : 0u;  // as KQ's bell saw it
   if (use_ha && ka.bell && blockIdx.x == 0 && threadIdx.x == 0) {
     // doorbell from KM (ctx option): KQ's request writes completed with its grid
-    uint32_t cnt[8];
-    for (int c = 0; c < 8; ++c) cnt[c] = c < ka.ncls ? *(volatile uint32_t*)&dv.ctl->counts[par][c] : 0u;
-    uint32_t kb0, kb1;
-    ha_range(dv, cnt, ka.cls_off, ka.ncls, kb0, kb1);
     HaDesc hd;
     hd.epoch = epoch;
     for (int c = 0; c < 8; ++c) {
-      hd.cnt[c] = cnt[c];
-      hd.off[c] = c < ka.ncls ? (uint32_t)ka.cls_off[c] : 0u;
+      hd.cnt[c] = c < ka.ncls ? *(volatile uint32_t*)&dv.ctl->counts[par][c] : 0u;
+      hd.hcut[c] = c < ka.ncls ? ha_hcut(hd.cnt[c], dv.ha_rcap[c], frac) : 0u;
     }
-    hd.kcut = ha_kcut(dv, ka, par);
+    hd.pad = 0;
     hd.epoch2 = epoch;
     dv.ha_desc[par] = hd;
     __threadfence_system();
@@ -1631,16 +1620,21 @@ __global__ void __launch_bounds__(128, 4) km_kernel(const __grid_constant__ Dev 
   float4* wsm = hsm + (dv.ha ? kHaSmemF4 : 0);
   unsigned ins = 0, ev = 0, byp = 0, harows = 0, hato = 0;
   long long docc = 0;
-  const uint32_t kcut = use_ha ? ha_kcut(dv, ka, par) : 0u;
   unsigned long long hostb = 0;
-  uint32_t bkb0 = 0, bkb1 = 0;
   bool poller = false;
   if (use_ha) {  // warp 0 of CTA 0 polls the host threads' progress; the other warps read blocks
-    uint32_t cnt[8];
-    for (int c = 0; c < 8; ++c) cnt[c] = c < ka.ncls ? *(volatile uint32_t*)&dv.ctl->counts[par][c] : 0u;
-    ha_range(dv, cnt, ka.cls_off, ka.ncls, bkb0, bkb1);
     poller = gw == 0;
-    if (poller) ha_poll(dv, epoch, bkb0, min(kcut, bkb1 + 1u), lane);
+    if (poller) {
+      HaBlocks hb;
+      hb.ncls = ka.ncls;
+#pragma unroll
+      for (int c = 0; c < 8; ++c) {
+        const uint32_t cnt = c < ka.ncls ? *(volatile uint32_t*)&dv.ctl->counts[par][c] : 0u;
+        hb.lo[c] = dv.ha_rbase[c] / kHaBlock;
+        hb.n[c] = c < ka.ncls ? ha_hcut(cnt, dv.ha_rcap[c], frac) : 0u;
+      }
+      ha_poll(dv, epoch, hb, lane);
+    }
     gw -= 1;
     nw -= 1;
   }
@@ -1650,8 +1644,8 @@ __global__ void __launch_bounds__(128, 4) km_kernel(const __grid_constant__ Dev 
     const MissRec* ml = dv.miss + ka.cls_off[c];
 #define FL_KM(D)                                                                                              \
   if (use_ha)                                                                                                 \
-    km_ha<BYTES, D>(dv, ka.out, ml, epoch, nmiss, lane, gw, nw, ins, ev, byp, docc, hostb, hsm, wsm, harows, hato, kcut, \
-                    bkb0);                                                                                  \
+    km_ha<BYTES, D>(dv, ka.out, ml, epoch, nmiss, lane, gw, nw, ins, ev, byp, docc, hostb, hsm, wsm, harows, hato, c,  \
+                    ha_hcut(nmiss, dv.ha_rcap[c], frac));                                                   \
   else                                                                                                        \
     km_rows<BYTES, D, KmM<BYTES, D>::value>(dv, ka.out, ml, epoch, nmiss, lane, gw, nw, ins, ev, byp, docc, hostb, wsm)
     if constexpr (DU > 0) {
