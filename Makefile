@@ -39,3 +39,10 @@ $(PKG)/libfleche_exp.so: $(wildcard $(CSRC)/*.cu) $(HDRS)
 	@mkdir -p $(BUILD)/exp
 	for u in $(UNITS); do $(NVCC) $(NVFLAGS) -DFLECHE_EXPERIMENTS -c -o $(BUILD)/exp/$$u.o $(CSRC)/$$u.cu || exit 1; done
 	$(NVCC) $(ARCH) -shared -cudart static -o $@ $(UNITS:%=$(BUILD)/exp/%.o)
+
+# A/B variant build: make variant V=name EXTRA="-DFL_KQ_PROBE=16" -> $(PKG)/libfleche_name.so
+# (select at run time with FLECHE_LIB=libfleche_name.so)
+variant:
+	@mkdir -p $(BUILD)/v_$(V)
+	for u in $(UNITS); do $(NVCC) $(NVFLAGS) $(EXTRA) -c -o $(BUILD)/v_$(V)/$$u.o $(CSRC)/$$u.cu & done; wait
+	$(NVCC) $(ARCH) -shared -cudart static -o $(PKG)/libfleche_$(V).so $(UNITS:%=$(BUILD)/v_$(V)/%.o)

@@ -40,7 +40,8 @@ struct HostAssist {
   void* mem = nullptr;
   HaReq* req = nullptr;                // [2][req_cap] (indexed like the miss list)
   HaDesc* desc = nullptr;              // [2]
-  unsigned long long* bell = nullptr;  // doorbell (epoch)
+  unsigned long long* bell = nullptr;  // doorbell (epoch): the descriptor of that batch is written
+  unsigned long long* start = nullptr; // start word (epoch): KQ of that batch has begun
   uint32_t* ready = nullptr;           // [2][blk_cap] ready word of each staging block (= epoch once staged)
   uint32_t blk_cap = 0;
   uint32_t rbase[8] = {}, rcap[8] = {};  // staging rows of width class c: [rbase, rbase + rcap)
@@ -85,6 +86,7 @@ struct fleche_ctx {
   int km_bps = 4;  // KM CTAs per SM
   int kq_tma = 0;      // KQ's hit gather by bulk copies through shared memory (row width 32 or 64; 0 = registers)
   size_t kq_smem = 0;  // its dynamic shared memory (4 warps x 32 rows)
+  int kf_ctas = 0;     // host-assisted early fetch: KQ CTAs that copy staged blocks into HBM (0 = off)
   bool per_table_launch = false;
   // decoupled hit copy (uniform layout): KG on a side stream, forked after KQ, joined after KM
   bool decoupled = false;
@@ -298,31 +300,42 @@ __attribute__((target("avx2"))) void stage_row(float* dst, const float* src, siz
     _mm256_stream_si256((__m256i*)((char*)dst + b), _mm256_loadu_si256((const __m256i*)((const char*)src + b)));
 }
 
-// One host-assist thread: wait for a doorbell, gather this thread's blocks of the batch's
-// requests (block k = miss-list indices [64k, 64k + 64), rows of every width class in
-// it, k % nthreads == me, in increasing k) into the staging buffer with non-temporal
-// stores, and publish each block's ready word (= epoch) once its rows are in place.
-// Spins while batches keep coming; after ~20 ms without one it polls every 20 us (an idle
-// ctx burns no core).  No `pause` in the spin: on a KVM guest it can trigger pause-loop
-// exits that deschedule the vCPU.
+// One host-assist thread: the CPU-DRAM layer queried while the batch is still being
+// indexed (Fig 8b).  KQ's first CTA writes the batch's epoch to the start word
+// when it begins; from then on the thread streams its staging blocks (block k = staging
+// rows [64k, 64k + 64), k % nthreads == me, increasing k within each width class): KQ
+// hands out a class's staging rows in the order it discovers the misses, so block k's
+// requests arrive while later misses are still being found.  Each row is gathered as soon
+// as its request carries this batch's tags, with non-temporal stores, and a block's ready
+// word (= epoch) is published once its rows are in place -- a full block at once, the
+// class's last partial block once the doorbell descriptor (written by KQ's last CTA) gives
+// the class's count.  Blocks past the descriptor's host share (hcut) are not started; a
+// block gathered before the descriptor arrived and then left to KM's zero-copy share is
+// simply not read.  Spins while batches keep coming; after ~20 ms without progress it
+// polls every 20 us (an idle ctx burns no core).  No `pause` in the spin: on a KVM guest
+// it can trigger pause-loop exits that deschedule the vCPU.
 void ha_worker(HostAssist* h, int me) {
   prctl(PR_SET_TIMERSLACK, 1000UL, 0, 0, 0);  // idle polls wake within ~20 us, not the default 50 us slack
-  uint32_t last = 0;
-  uint64_t spins = 0;
   auto now_ns = []() {
     struct timespec ts;
     clock_gettime(CLOCK_MONOTONIC, &ts);
     return (uint64_t)ts.tv_sec * 1000000000ull + (uint64_t)ts.tv_nsec;
   };
-  uint64_t t_last = now_ns();
+  auto idle = [&](uint64_t since) {  // back off after 20 ms without anything to do
+    if (now_ns() - since > 20000000ull) {
+      struct timespec ts = {0, 20000};
+      nanosleep(&ts, nullptr);
+    }
+  };
   const int nt = (int)h->host.size();
+  const uint64_t T = (uint64_t)h->nthreads;
+  uint32_t last = 0;
+  uint64_t t_last = now_ns();
+  uint64_t spins = 0;
   while (!h->stop.load(std::memory_order_relaxed)) {
-    const uint32_t e = (uint32_t)__atomic_load_n(h->bell, __ATOMIC_ACQUIRE);
+    const uint32_t e = (uint32_t)__atomic_load_n(h->start, __ATOMIC_ACQUIRE);
     if (e == last) {
-      if ((++spins & 1023) == 0 && now_ns() - t_last > 20000000ull) {
-        struct timespec ts = {0, 20000};
-        nanosleep(&ts, nullptr);
-      }
+      if ((++spins & 1023) == 0) idle(t_last);
       continue;
     }
     last = e;
@@ -336,40 +349,36 @@ void ha_worker(HostAssist* h, int me) {
     if (me < 64) h->exp_t[(e % 64) * 128 + me] = rt();
 #endif
     const int par = e & 1u;
-    // the descriptor was written without a system fence before the doorbell: re-read until
-    // both epoch fields carry this batch (and a second read agrees), at most ~1 ms
-    HaDesc d;
-    bool got = false;
-    for (uint64_t n = 0; !got; ++n) {
-      memcpy(&d, (const void*)(h->desc + par), sizeof d);
-      __atomic_thread_fence(__ATOMIC_ACQUIRE);
-      HaDesc d2;
-      memcpy(&d2, (const void*)(h->desc + par), sizeof d2);
-      got = d.epoch == e && d.epoch2 == e && !memcmp(&d, &d2, sizeof d);
-      if (!got && (n & 255) == 255 && now_ns() - t_last > 1000000ull) break;
-    }
-    if (!got) continue;  // the GPU moved on (a later batch's doorbell, or a parity cycle ahead)
     uint32_t* ready = h->ready + (size_t)par * h->blk_cap;
-    const HaReq* rq = h->req + (size_t)par * h->req_cap;
+    const volatile HaReq* rq = h->req + (size_t)par * h->req_cap;
     float* st = h->stage + (size_t)par * h->stage_floats;
-    // a request of this batch (KQ wrote it without a system fence: wait until both halves
-    // carry this batch's tags, read twice so a torn read is never taken); false after ~1 ms
-    auto fetch = [&](uint64_t i, HaReq* out) -> bool {
-      const volatile HaReq* p = rq + i;
-      for (uint64_t n = 0;; ++n) {
-        HaReq a{p->tid, p->stage};
-        if (ha_req_current(a, e)) {
-          HaReq b{p->tid, p->stage};
-          if (b.tid == a.tid && b.stage == a.stage) {
-            *out = a;
-            return true;
-          }
-        }
-        if ((n & 255) == 255 && (h->stop.load(std::memory_order_relaxed) || now_ns() - t_last > 1000000ull))
-          return false;
+    // the doorbell descriptor of this batch (written without a system fence: accepted once
+    // both epoch fields carry this batch and a second read agrees)
+    HaDesc d;
+    bool have_d = false;
+    uint64_t t_d = 0;
+    auto poll_desc = [&]() {
+      if (have_d) return;
+      HaDesc a, b2;
+      memcpy(&a, (const void*)(h->desc + par), sizeof a);
+      __atomic_thread_fence(__ATOMIC_ACQUIRE);
+      memcpy(&b2, (const void*)(h->desc + par), sizeof b2);
+      if (a.epoch == e && a.epoch2 == e && !memcmp(&a, &b2, sizeof a)) {
+        d = a;
+        have_d = true;
+        t_d = now_ns();
       }
     };
-    bool lost = false;  // a request never arrived: stop publishing (KM times out and reads zero-copy)
+    // request i of this batch, if it has arrived (KQ wrote it without a system fence: both
+    // halves must carry this batch's tags, and a second read must agree -- never torn)
+    auto fetch = [&](uint64_t i, HaReq* out) -> bool {
+      HaReq a{rq[i].tid, rq[i].stage};
+      if (!ha_req_current(a, e)) return false;
+      HaReq b2{rq[i].tid, rq[i].stage};
+      if (b2.tid != a.tid || b2.stage != a.stage) return false;
+      *out = a;
+      return true;
+    };
     auto src_of = [&](const HaReq& r, int32_t* dim, uint64_t* so) -> const float* {
       const int t = (int)(r.tid >> 55);
       const int64_t id = (int64_t)(r.tid & kReqLow40);
@@ -379,70 +388,102 @@ void ha_worker(HostAssist* h, int me) {
       if (*so + (uint64_t)*dim > h->stage_floats) return nullptr;
       return h->host[t] + (size_t)id * (size_t)*dim;
     };
-    auto prefetch = [&](uint64_t i) {
-      HaReq r;
-      int32_t dd = 0;
-      uint64_t so = 0;
-      if (lost || !fetch(i, &r)) {
-        lost = true;
-        return;
-      }
-      if (const float* p = src_of(r, &dd, &so))
-        for (int b = 0; b < dd * 4; b += 64) __builtin_prefetch((const char*)p + b, 0, 0);
-    };
-    // static ownership (staging block b = rows [64b, 64b + 64) belongs to thread b % nthreads
-    // in every batch, taken in increasing b): a thread that stalls past the GPU's give-up can
-    // only ever overwrite its own blocks, which it republishes only after rewriting them
-    // (ADVICE r1); class c stages its first min(cnt, rcap) misses in rows [rbase_c, ...),
-    // the host threads take blocks below hcut_c of each class
-    for (int c = 0; c < 8 && !lost; ++c) {
-      if (!d.cnt[c] || !d.hcut[c]) continue;
-      const uint64_t rb = h->rbase[c], nrow = std::min<uint64_t>(d.cnt[c], h->rcap[c]);
-      const uint64_t kb0 = rb / kHaBlock, kend = kb0 + std::min<uint64_t>(d.hcut[c], (nrow + kHaBlock - 1) / kHaBlock);
-      for (uint64_t kb = kb0; kb < kend && !lost; ++kb) {
-        if (kb % (uint64_t)h->nthreads != (uint64_t)me) continue;
-        if (h->delay_ns) {  // a stalled host thread (tests): its blocks time out on the GPU
+    // static ownership (staging block b belongs to thread b % nthreads in every batch, taken
+    // in increasing b): a thread that stalls past the GPU's give-up can only ever overwrite
+    // its own blocks, which it republishes only after rewriting them
+    struct Cursor {
+      uint64_t kb = 0, i = 0;  // current block, next row
+      bool done = true;
+    } cur[8];
+    for (int c = 0; c < 8; ++c) {
+      if (!h->rcap[c]) continue;
+      const uint64_t kb0 = h->rbase[c] / kHaBlock;
+      cur[c].kb = kb0 + (T - kb0 % T + (uint64_t)me) % T;
+      cur[c].i = cur[c].kb * kHaBlock;
+      cur[c].done = cur[c].i >= (uint64_t)h->rbase[c] + h->rcap[c];
+    }
+    uint64_t t_prog = now_ns();
+    bool delayed = false;  // fault injection: once per block
+    while (true) {
+      poll_desc();
+      bool all_done = true, progressed = false;
+      for (int c = 0; c < 8; ++c) {
+        Cursor& q = cur[c];
+        if (q.done) continue;
+        const uint64_t rb = h->rbase[c], lo = q.kb * kHaBlock;
+        uint64_t hi = std::min<uint64_t>(lo + kHaBlock, rb + h->rcap[c]);
+        if (have_d) {  // the batch's count and the host share are known
+          const uint64_t nrow = std::min<uint64_t>(d.cnt[c], h->rcap[c]);
+          if (q.kb - rb / kHaBlock >= d.hcut[c] || lo >= rb + nrow) {
+            q.done = true;
+            continue;
+          }
+          hi = std::min<uint64_t>(hi, rb + nrow);
+        }
+        all_done = false;
+        if (h->delay_ns && !delayed) {  // a stalled host thread (tests): its blocks time out on the GPU
           struct timespec ts = {(time_t)(h->delay_ns / 1000000000ull), (long)(h->delay_ns % 1000000000ull)};
           nanosleep(&ts, nullptr);
+          delayed = true;
         }
-        const uint64_t lo = kb * kHaBlock, hi = std::min<uint64_t>(lo + kHaBlock, rb + nrow);
         constexpr uint64_t PF = 12;  // rows prefetched ahead (~4 lines each: keeps the line fill buffers busy)
-        for (uint64_t i = lo; i < std::min(hi, lo + PF); ++i) prefetch(i);
-        for (uint64_t i = lo; i < hi; ++i) {
-          if (i + PF < hi) prefetch(i + PF);
+        for (; q.i < hi; ++q.i) {
           HaReq r;
-          if (lost || !fetch(i, &r)) {  // never arrived: abandon the batch (KM's poller times out)
-            lost = true;
-            break;
+          if (!fetch(q.i, &r)) break;  // not arrived yet
+          if (q.i + PF < hi) {
+            HaReq r2;
+            int32_t d2 = 0;
+            uint64_t so2 = 0;
+            const float* p2 = fetch(q.i + PF, &r2) ? src_of(r2, &d2, &so2) : nullptr;
+            if (p2)
+              for (int b = 0; b < d2 * 4; b += 64) __builtin_prefetch((const char*)p2 + b, 0, 0);
           }
           int32_t dd = 0;
           uint64_t so = 0;
           if (const float* p = src_of(r, &dd, &so)) {
 #ifdef FLECHE_EXPERIMENTS
-            if (h->exp_nogather) continue;  // timing experiment: publish without gathering (wrong rows)
+            if (!h->exp_nogather)  // timing experiment: publish without gathering (wrong rows)
 #endif
-            if (h->nt_stores) stage_row(st + so, p, (size_t)dd * 4u);
-            else memcpy(st + so, p, (size_t)dd * 4u);
+            {
+              if (h->nt_stores) stage_row(st + so, p, (size_t)dd * 4u);
+              else memcpy(st + so, p, (size_t)dd * 4u);
+            }
           }
+          progressed = true;
         }
-        if (h->nt_stores) _mm_sfence();  // streaming stores are weakly ordered: drain them before the ready word
-        if (lost) break;
-        __atomic_store_n(ready + kb, e, __ATOMIC_RELEASE);
+        if (q.i == hi && (hi == lo + kHaBlock || have_d)) {  // the block is complete
+          if (h->nt_stores) _mm_sfence();  // streaming stores are weakly ordered: drain them before the ready word
+          __atomic_store_n(ready + q.kb, e, __ATOMIC_RELEASE);
 #ifdef FLECHE_EXPERIMENTS
-        if (h->exp_pub) {
-          struct timespec ts;
-          clock_gettime(CLOCK_REALTIME, &ts);
-          h->exp_pub[kb] = (uint64_t)ts.tv_sec * 1000000000ull + (uint64_t)ts.tv_nsec;
-        }
+          if (h->exp_pub) {
+            struct timespec ts;
+            clock_gettime(CLOCK_REALTIME, &ts);
+            h->exp_pub[q.kb] = (uint64_t)ts.tv_sec * 1000000000ull + (uint64_t)ts.tv_nsec;
+          }
 #endif
+          q.kb += T;
+          q.i = q.kb * kHaBlock;
+          q.done = q.i >= rb + h->rcap[c];
+          delayed = false;
+          progressed = true;
+        }
       }
+      if (all_done || h->stop.load(std::memory_order_relaxed)) break;
+      const uint64_t now = now_ns();
+      if (progressed) {
+        t_prog = now;
+        continue;
+      }
+      // waiting for requests: give up on this batch when a newer one has started, or when a
+      // request never arrived ~1 ms after the descriptor (KM's poller times out and reads
+      // those blocks zero-copy)
+      if ((uint32_t)__atomic_load_n(h->start, __ATOMIC_ACQUIRE) != e) break;
+      if (have_d && now - std::max(t_d, t_prog) > 1000000ull) break;
+      if ((++spins & 1023) == 0) idle(t_prog);
     }
+    t_last = now_ns();
 #ifdef FLECHE_EXPERIMENTS
-    if (me < 64) {
-      struct timespec ts;
-      clock_gettime(CLOCK_REALTIME, &ts);
-      h->exp_t[(e % 64) * 128 + 64 + me] = (uint64_t)ts.tv_sec * 1000000000ull + (uint64_t)ts.tv_nsec;
-    }
+    if (me < 64) h->exp_t[(e % 64) * 128 + 64 + me] = rt();
 #endif
   }
 }
@@ -463,7 +504,7 @@ void free_all(fleche_ctx* c) {
                   c->dv.miss, c->dv.dup, c->dv.ctl, c->dv.stats, c->d_tables, c->d_ids_stage, c->d_out_stage,
                   c->d_pool_stage, c->d_kdec, c->rd.scratch, c->rd.slotval, c->rd.inv, c->rd.region, c->rd.cnt,
                   c->rd.prefix, c->rd.done, c->rd.stats, c->d_slots, c->d_age_hist, c->d_prefill_out,
-                  c->d_out_stage2, c->dv.ha_seen};
+                  c->d_out_stage2, c->dv.ha_seen, c->dv.ha_hstage, c->dv.ha_hseen};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   for (auto& r : c->registered) cudaHostUnregister(r.first);
@@ -607,8 +648,10 @@ fleche_status launch_query(fleche_ctx* c, const int64_t* const* ids, const int64
   qa.ha_bell = c->dv.ha && !bell_km;
   ka.bell = c->dv.ha && bell_km;
   qa.ncls = ka.ncls;
+  for (int k = 0; k < ka.ncls; ++k) qa.cls_dim[k] = c->cls_dim[k];
   if (total > 0 && !c->per_table_launch) {
-    const int64_t blocks = (total + 127) / 128;
+    qa.nfetch = (qa.ha_bell && !decouple) ? c->kf_ctas : 0;
+    const int64_t blocks = (total + 127) / 128 + qa.nfetch;
     launch_k(kPdlKQ, kq_fn<MAXT>(c->kq_tma), (unsigned)blocks, 128, c->kq_smem, s, qa, c->dv);
     c->kernels++;
     if (decouple) {  // fork: the hit copy runs on the side stream, concurrently with KM
@@ -971,7 +1014,7 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
     }
     h->blk_cap = h->req_cap / kHaBlock + 2;
     const size_t o_req = 0, o_desc = o_req + 2 * sizeof(HaReq) * (size_t)h->req_cap, o_bell = o_desc + 2 * sizeof(HaDesc),
-                 o_ready = (o_bell + 8 + 127) & ~size_t(127), o_stage = (o_ready + 8ull * h->blk_cap + 255) & ~size_t(255),
+                 o_start = (o_bell + 8 + 63) & ~size_t(63), o_ready = (o_start + 8 + 127) & ~size_t(127), o_stage = (o_ready + 8ull * h->blk_cap + 255) & ~size_t(255),
                  total = o_stage + 2 * 4 * h->stage_floats;
     if (cudaHostAlloc(&h->mem, total, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess) {
       cudaGetLastError();
@@ -983,6 +1026,7 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
     h->req = (HaReq*)(b + o_req);
     h->desc = (HaDesc*)(b + o_desc);
     h->bell = (unsigned long long*)(b + o_bell);
+    h->start = (unsigned long long*)(b + o_start);
     h->ready = (uint32_t*)(b + o_ready);
     h->stage = (float*)(b + o_stage);
     void* dmem = nullptr;
@@ -992,6 +1036,7 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
     dv.ha_req = (HaReq*)(db + o_req);
     dv.ha_desc = (HaDesc*)(db + o_desc);
     dv.ha_bell = (unsigned long long*)(db + o_bell);
+    dv.ha_start = (unsigned long long*)(db + o_start);
     dv.ha_ready = (uint32_t*)(db + o_ready);
     dv.ha_blk_cap = h->blk_cap;
     dv.ha_row_floats = (uint32_t)c->max_dim;
@@ -1002,6 +1047,16 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
     if (cudaMalloc((void**)&dv.ha_seen, 4ull * h->blk_cap) != cudaSuccess ||
         cudaMemset(dv.ha_seen, 0, 4ull * h->blk_cap) != cudaSuccess)
       return fail(FLECHE_ENOMEM);
+    // early fetch (FLECHE_HA_EARLY=0 turns it off): KQ's first kf_ctas CTAs move staged
+    // blocks into an HBM copy while the lookups run
+    c->kf_ctas = (int)env_u("FLECHE_HA_EARLY", 1) ? (int)std::min<uint64_t>(64, std::max<uint64_t>(1, env_u("FLECHE_KF_CTAS", 16))) : 0;
+    dv.ha_kf_tail = (uint32_t)env_u("FLECHE_KF_TAIL", 0);
+    if (c->kf_ctas) {
+      if (cudaMalloc((void**)&dv.ha_hstage, 2ull * 4ull * h->stage_floats) != cudaSuccess ||
+          cudaMalloc((void**)&dv.ha_hseen, 4ull * h->blk_cap) != cudaSuccess ||
+          cudaMemset(dv.ha_hseen, 0, 4ull * h->blk_cap) != cudaSuccess)
+        return fail(FLECHE_ENOMEM);
+    }
     dv.ha_stage = (float*)(db + o_stage);
     dv.ha_req_cap = h->req_cap;
     dv.ha_stage_floats = h->stage_floats;
@@ -1032,8 +1087,8 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
   cudaMemset(dv.exp_buf, 0, ((size_t)c->km_blocks * 4 * 4 + 8) * 8);
   dv.exp_slots = (uint32_t)c->km_blocks * 16;
   if (c->ha) {
-    if (cudaMalloc((void**)&dv.exp_blk, ((size_t)c->ha->blk_cap * 4) * 8) != cudaSuccess) return fail(FLECHE_ENOMEM);
-    cudaMemset(dv.exp_blk, 0, ((size_t)c->ha->blk_cap * 4) * 8);
+    if (cudaMalloc((void**)&dv.exp_blk, ((size_t)c->ha->blk_cap * 8) * 8) != cudaSuccess) return fail(FLECHE_ENOMEM);
+    cudaMemset(dv.exp_blk, 0, ((size_t)c->ha->blk_cap * 8) * 8);
     c->ha->exp_pub = new uint64_t[c->ha->blk_cap]();
   }
 #endif
@@ -1828,17 +1883,18 @@ extern "C" __attribute__((visibility("default"))) fleche_status fleche_exp_ha_ti
   memcpy(host, c->ha->exp_t, std::min(n, (size_t)64 * 2 * 64) * 8);
   return FLECHE_OK;
 }
-// per staging block: [GPU wait start, GPU flag seen, GPU rows landed, GPU done, CPU published (REALTIME)]
+// per staging block: [KM wait start, KM flag seen, KM rows landed, KM done, early-fetch mirror,
+// early-fetch copy done (GPU globaltimer), CPU published (REALTIME)]
 extern "C" __attribute__((visibility("default"))) fleche_status fleche_exp_ha_blocks(fleche_ctx* c, uint64_t* host,
                                                                                      size_t nblk) {
   if (!c || !host || !c->ha) return FLECHE_EINVAL;
   if (c->have_last) cudaStreamSynchronize(c->last_stream);
   const size_t m = std::min(nblk, (size_t)c->ha->blk_cap);
-  std::vector<uint64_t> g(m * 4);
-  if (cudaMemcpy(g.data(), c->dv.exp_blk, m * 4 * 8, cudaMemcpyDeviceToHost) != cudaSuccess) return FLECHE_ECUDA;
+  std::vector<uint64_t> g(m * 8);
+  if (cudaMemcpy(g.data(), c->dv.exp_blk, m * 8 * 8, cudaMemcpyDeviceToHost) != cudaSuccess) return FLECHE_ECUDA;
   for (size_t k = 0; k < m; ++k) {
-    for (int j = 0; j < 4; ++j) host[k * 5 + j] = g[k * 4 + j];
-    host[k * 5 + 4] = c->ha->exp_pub[k];
+    for (int j = 0; j < 6; ++j) host[k * 7 + j] = g[k * 8 + j];
+    host[k * 7 + 6] = c->ha->exp_pub[k];
   }
   return FLECHE_OK;
 }

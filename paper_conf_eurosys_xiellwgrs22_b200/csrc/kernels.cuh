@@ -37,7 +37,7 @@
 #define FL_GATHER_F4 8  // float4 loads per lane in flight in a row gather (A/B builds vary it)
 #endif
 #ifndef FL_KQ_PROBE
-#define FL_KQ_PROBE 32  // index lines per lane in flight in KQ's probe (a divisor of 32; A/B builds vary it)
+#define FL_KQ_PROBE 16  // index lines per lane in flight in KQ's probe (a divisor of 32): 16 = no spill with 64 registers; cfg2 KQ 36.9 vs 39.2 us at 32 (same box)
 #endif
 #ifndef FL_KQ_TS_DEFER
 #define FL_KQ_TS_DEFER 1  // KQ consumes its timestamp-exchange result late (0 = right after it; A/B builds)
@@ -130,6 +130,8 @@ struct Ctl {
   uint32_t km_bar;        // KM grid barrier: epoch whose owner rows are all in `out`
   long long ke_occ;
   uint32_t kq_done;       // host-assisted: KQ CTA arrivals (the last one rings the doorbell)
+  uint32_t kq_end;        // early fetch: epoch whose KQ lookup CTAs have all finished (counts final)
+  uint32_t kq_end_pad;
   uint32_t ha_abort;      // host-assisted: epoch whose staging the poller gave up on (timeout)
   // unified-index share tuning (see ui_tune): the host threads' share of a
   // batch's staging blocks (x 2^-16; the GPU's zero-copy reads -- the unified index -- take
@@ -217,9 +219,12 @@ struct Dev {
   HaReq* ha_req;               // [2][ha_req_cap]: indexed like the miss list
   HaDesc* ha_desc;             // [2]
   unsigned long long* ha_bell; // doorbell: epoch of the latest published descriptor
+  unsigned long long* ha_start;  // start word: epoch of the batch whose KQ has begun (host threads stream its requests)
   uint32_t* ha_ready;          // [2][ha_blk_cap] (host memory) epoch of each staging block once staged
   uint32_t* ha_seen;           // [ha_blk_cap] (HBM) the poller warp's mirror of ha_ready[epoch & 1]
   float* ha_stage;             // [2][ha_stage_floats]
+  float* ha_hstage;            // early fetch: [2][ha_stage_floats] (HBM) copy of the staged blocks
+  uint32_t* ha_hseen;          // early fetch: [ha_blk_cap] (HBM) epoch once a block's rows are in ha_hstage
   uint32_t ha_req_cap, ha_blk_cap;  // staging rows (= request slots) and blocks per epoch parity
   uint32_t ha_rbase[8];        // first staging row of width class c (a multiple of kHaBlock)
   uint32_t ha_rcap[8];         // staging rows of class c (a multiple of kHaBlock): its misses beyond go zero-copy
@@ -230,7 +235,7 @@ struct Dev {
   uint32_t ha_frac_fixed;      // 1 = FLECHE_HA_FRAC fixed the host threads' share (no tuning loop)
   uint32_t ha_min_rows;        // batches with fewer unique misses stay all zero-copy (the split loses there)
   uint32_t ha_unit_pieces;     // KM work unit = this many 16-row pieces (0: adaptive to the batch)
-  uint32_t ha_pad2;
+  uint32_t ha_kf_tail;         // early fetch: 1 = the fetch CTAs copy every host block (KQ ends after them), 0 = stop with the lookups
 #ifdef FLECHE_EXPERIMENTS
   int32_t exp_mode;  // timing experiments only (libfleche_exp.so); breaks semantics
   int32_t exp_pad;
@@ -259,7 +264,8 @@ struct QArgs {
   int32_t ncls;              //   (number of width classes of the miss list)
   const int64_t* dcnt;       // key-sharded sync-free: [n][n] routed-count matrix in device memory
   int32_t dme;               //   this rank (segment i's count = dcnt[i * n + dme])
-  int32_t pad3;
+  int32_t nfetch;            // early fetch: CTAs 0..nfetch-1 copy staged blocks into HBM (kq_fetch)
+  int32_t cls_dim[8];        //   (row width of each class)
 };
 
 struct KMArgs {
@@ -451,6 +457,7 @@ __device__ __forceinline__ void ha_poll(const Dev& dv, uint32_t epoch, const HaB
 #pragma unroll
   for (int c = 0; c < 8; ++c) lo[c] = c < hb.ncls ? hb.lo[c] : 0u;  // class c: blocks below lo[c] mirrored
   while (true) {
+    if (*(volatile uint32_t*)&dv.ctl->ha_abort == epoch) break;  // given up already (early fetch's poller)
     uint32_t fresh = 0, missing = 0;
 #pragma unroll
     for (int c = 0; c < 8; ++c) {
@@ -694,6 +701,144 @@ __device__ __forceinline__ void bulk_s2g(void* gmem, const void* smem, unsigned 
   asm volatile("cp.async.bulk.commit_group;" ::: "memory");
 }
 
+// Early fetch (host-assisted): the first qa.nfetch CTAs of KQ do no lookups; they move the
+// batch's staged blocks over the link into HBM WHILE the other CTAs are still indexing, so
+// the link is busy during KQ instead of only during KM (the host threads stream the
+// requests as KQ writes them).  Warp 0 of CTA 0 mirrors the host threads' ready words into
+// ha_seen (as KM's poller does); every other warp copies its static share of each width
+// class's blocks (class-local block b = w, w + W, ...) as they become ready, and publishes
+// ha_hseen[kb] = epoch; KM then reads those rows from HBM.  The batch's block counts are
+// known once the last lookup CTA has rung the doorbell (ctl->kq_end = epoch); the fetch
+// CTAs stop at the host share (hcut) or give up (ha_abort) when the host threads stall, and
+// KM fetches whatever is not in HBM exactly as without early fetch.
+constexpr unsigned long long kKfStallNs = 150000;
+template <int MAXT>
+__device__ __noinline__ void kq_fetch(const QArgs<MAXT>& qa, const Dev& dv) {
+  const int lane = threadIdx.x & 31;
+  const uint32_t w = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+  const uint32_t nwk = (uint32_t)qa.nfetch * (blockDim.x >> 5) - 1u;  // copy warps
+  const uint32_t epoch = *(volatile uint32_t*)&dv.ctl->epoch;
+  const int par = epoch & 1u;
+  const int ncls = qa.ncls;
+  const uint32_t* ready = dv.ha_ready + (size_t)par * dv.ha_blk_cap;
+  const float* stage = dv.ha_stage + (size_t)par * dv.ha_stage_floats;
+  float* hstage = dv.ha_hstage + (size_t)par * dv.ha_stage_floats;
+  // the batch's host share per class, once every lookup CTA has finished (0xFFFFFFFF before)
+  auto share = [&](int c, bool& known, bool& active) -> uint32_t {
+    if (ld_acquire_gpu_u32(&dv.ctl->kq_end) != epoch) {
+      known = false;
+      return 0xFFFFFFFFu;
+    }
+    known = true;
+    active = *(volatile uint32_t*)&dv.ctl->ha_rung == epoch;
+    if (!active || !dv.ha_kf_tail) return 0u;  // default: stop with the lookups (KM takes the rest)
+    const uint32_t cnt = *(volatile uint32_t*)&dv.ctl->counts[par][c];
+    return ha_hcut(cnt, dv.ha_rcap[c], *(volatile uint32_t*)&dv.ctl->ha_frac_q16);
+  };
+  if (w == 0) {  // the poller: ready words -> ha_seen (a window of 128 blocks per class ahead)
+    uint32_t lo[8];
+#pragma unroll
+    for (int c = 0; c < 8; ++c) lo[c] = 0;  // class-local: blocks below lo[c] mirrored
+    unsigned long long t_prog = globaltimer_ns();
+    while (true) {
+      if (*(volatile uint32_t*)&dv.ctl->ha_abort == epoch) return;
+      bool known = false, active = true, left = false, fresh = false;
+#pragma unroll 1
+      for (int c = 0; c < ncls; ++c) {
+        const uint32_t b0 = dv.ha_rbase[c] / kHaBlock, nb = min(share(c, known, active), dv.ha_rcap[c] / kHaBlock);
+        if (lo[c] >= nb) continue;
+        left = true;
+        const uint32_t b = lo[c] + 4u * lane;
+        uint32_t v[4];
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+          v[q] = (b + q < nb && b + q < lo[c] + 128u && ld_acquire_gpu_u32(dv.ha_seen + b0 + b + q) != epoch)
+                     ? ld_relaxed_sys_u32(ready + b0 + b + q)
+                     : epoch;
+        unsigned newly = 0;
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+          if (b + q < nb && b + q < lo[c] + 128u && v[q] == epoch) newly |= 1u << q;
+        if (__any_sync(kFull, newly)) {
+          asm volatile("fence.acq_rel.sys;" ::: "memory");  // the rows staged before these ready words
+#pragma unroll
+          for (int q = 0; q < 4; ++q)
+            if (newly & (1u << q)) {
+              st_release_gpu_u32(dv.ha_seen + b0 + b + q, epoch);
+#ifdef FLECHE_EXPERIMENTS
+              if (dv.exp_blk) dv.exp_blk[(b0 + b + q) * 8 + 4] = globaltimer_ns();
+#endif
+            }
+        }
+        // advance past the mirrored prefix
+        const unsigned all4 = __ballot_sync(kFull, b >= nb || b >= lo[c] + 128u ||
+                                                       (v[0] == epoch && v[1] == epoch && v[2] == epoch && v[3] == epoch));
+        const uint32_t adv = all4 == kFull ? 128u : 4u * (uint32_t)(__ffs(~all4) - 1);
+        if (adv) fresh = true;
+        lo[c] = min(nb, lo[c] + adv);
+        if (lo[c] < nb) left = true;
+      }
+      if (!left && known) return;
+      if (known && !active) return;
+      const unsigned long long now = globaltimer_ns();
+      if (fresh) t_prog = now;
+      if (known && now - t_prog > kKfStallNs) {  // a host thread stalled: KM takes over (zero-copy)
+        if (lane == 0) st_release_gpu_u32(&dv.ctl->ha_abort, epoch);
+        return;
+      }
+      __nanosleep(200);
+    }
+  }
+  // copy warps: class-local blocks b = w - 1 + k * nwk of every class, as they become ready
+  uint32_t cur[8];
+#pragma unroll
+  for (int c = 0; c < 8; ++c) cur[c] = w - 1u;
+  while (true) {
+    if (*(volatile uint32_t*)&dv.ctl->ha_abort == epoch) return;
+    bool left = false, progressed = false;
+#pragma unroll 1
+    for (int c = 0; c < ncls; ++c) {
+      bool known = false, active = true;
+      const uint32_t nb = min(share(c, known, active), dv.ha_rcap[c] / kHaBlock);
+      if (cur[c] >= nb) continue;
+      left = true;
+      const uint32_t kb = dv.ha_rbase[c] / kHaBlock + cur[c];
+      if (ld_acquire_gpu_u32(dv.ha_seen + kb) != epoch) continue;
+      // the block's rows: host staging -> HBM (row stride ha_row_floats, class width D)
+      const int D = qa.cls_dim[c];
+      const uint32_t vec = (uint32_t)D / 4u, n4 = (uint32_t)kHaBlock * vec;
+      const size_t base = (size_t)kb * kHaBlock * dv.ha_row_floats;
+#pragma unroll 1
+      for (uint32_t q0 = 0; q0 < n4; q0 += 32u * 8u) {
+        float4 v[8];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          const uint32_t q = q0 + 32u * i + lane;
+          v[i] = q < n4 ? ld_cv_v4(stage + base + (size_t)(q / vec) * dv.ha_row_floats + 4u * (q % vec))
+                        : make_float4(0.f, 0.f, 0.f, 0.f);
+        }
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          const uint32_t q = q0 + 32u * i + lane;
+          if (q < n4) st_v4(hstage + base + (size_t)(q / vec) * dv.ha_row_floats + 4u * (q % vec), v[i]);
+        }
+      }
+      __syncwarp();
+      if (lane == 0) {
+        __threadfence();
+        st_release_gpu_u32(dv.ha_hseen + kb, epoch);
+#ifdef FLECHE_EXPERIMENTS
+        if (dv.exp_blk) dv.exp_blk[kb * 8 + 5] = globaltimer_ns();
+#endif
+      }
+      cur[c] += nwk;
+      progressed = true;
+    }
+    if (!left) return;
+    if (!progressed) __nanosleep(200);
+  }
+}
+
 // TD > 0: hit rows gathered with bulk copies through TD-float shared-memory rows (one row
 // width for every table; dynamic shared memory = 4 warps x 32 rows x TD floats).
 template <int MAXT, int TD>
@@ -709,6 +854,11 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   pdl_wait();  // the previous batch (or the caller's producer of ids) has completed
+  if ((int)blockIdx.x < qa.nfetch) {  // early-fetch CTA (no lookups)
+    kq_fetch<MAXT>(qa, dv);
+    return;
+  }
+  const uint32_t bid = blockIdx.x - (uint32_t)qa.nfetch, nbid = gridDim.x - (uint32_t)qa.nfetch;  // lookup CTAs
   if (qa.dcnt && threadIdx.x == 0) {
     // key-sharded, sync-free: segment i's count is C[i][me] of the routed-count matrix in
     // device memory (written by the collective the stream ran before this launch)
@@ -719,12 +869,19 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
     }
     s_scan[qa.n] = acc;
   }
+#ifdef FLECHE_EXPERIMENTS
+  if (dv.exp_buf && bid == 0 && threadIdx.x == 0) dv.exp_buf[dv.exp_slots + 1] = globaltimer_ns();
+#endif
+  if (dv.ha && bid == 0 && threadIdx.x == 0)  // the host threads start streaming this batch's requests
+    asm volatile("st.relaxed.sys.global.u64 [%0], %1;" ::"l"(dv.ha_start),
+                 "l"((unsigned long long)*(volatile uint32_t*)&dv.ctl->epoch)
+                 : "memory");
   __syncthreads();
 
   const int lane = threadIdx.x & 31;
   const int64_t N = s_scan[qa.n];
   uint32_t it = 0;  // grid-stride iterations (one unless the grid was sized for a capacity, not N)
-  for (int64_t g0 = (int64_t)blockIdx.x * blockDim.x; g0 < N; g0 += (int64_t)gridDim.x * blockDim.x, ++it) {
+  for (int64_t g0 = (int64_t)bid * blockDim.x; g0 < N; g0 += (int64_t)nbid * blockDim.x, ++it) {
   const int64_t g = g0 + threadIdx.x;
   if (g - lane < N) {  // warp-uniform
     const uint32_t epoch = *(volatile uint32_t*)&dv.ctl->epoch;
@@ -777,7 +934,15 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
     const uint32_t fk = valid ? ti->base + (uint32_t)id : kEmpty;
     const uint32_t s = valid ? set_of_t(dv, ti, fk) : 0u;
 
-    // A3 probe: lane k holds way k of each of the warp's 32 sets (one 128 B line each)
+    // in-warp key groups (Zipf batches repeat hot keys within a warp): the lowest lane of
+    // each group (its first occurrence) probes, refreshes the timestamp and claims the
+    // miss for the whole group; the others take its result
+    const unsigned peers = __match_any_sync(kFull, fk);
+    const int klead = __ffs(peers) - 1;
+    const bool lead = lane == klead;
+    const unsigned pm = __ballot_sync(kFull, valid && lead);  // lanes whose set line is read
+
+    // A3 probe: lane k holds way k of each probed set (one 128 B line each)
     // (FL_KQ_PROBE lines in flight per lane: fewer registers, more CTAs per SM)
     int way = -1;
 #pragma unroll
@@ -786,7 +951,7 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
 #pragma unroll
       for (int i = 0; i < FL_KQ_PROBE; ++i) {
         const uint32_t si = __shfl_sync(kFull, s, i0 + i);
-        kw[i] = ld_nc_u32(dv.keys + (size_t)si * 32u + lane);
+        kw[i] = ((pm >> (i0 + i)) & 1u) ? ld_nc_u32(dv.keys + (size_t)si * 32u + lane) : kEmpty;
       }
 #pragma unroll
       for (int i = 0; i < FL_KQ_PROBE; ++i) {
@@ -795,6 +960,7 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
         if (lane == i0 + i && m) way = __ffs(m) - 1;
       }
     }
+    way = __shfl_sync(kFull, way, klead);
     const bool hit = valid && way >= 0;
     const bool miss = valid && way < 0;
     const uint32_t slot = s * 32u + (uint32_t)way;
@@ -815,8 +981,8 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
     // L2 round trips overlap the row gather; they are consumed after it
     uint32_t old_ts = 0, h = 0;
     unsigned long long cur = 0;
-    if (hit) old_ts = ld_cg_u32(dv.ts + slot);
-    if (miss) {
+    if (hit && lead) old_ts = ld_cg_u32(dv.ts + slot);
+    if (miss && lead) {
       h = dv.ordered ? (uint32_t)__umul64hi((uint64_t)(ti->host + (size_t)id * (size_t)d) - dv.host_lo, dv.host_mul) &
                            dv.scr_mask
                      : scr_hash(fk) & dv.scr_mask;
@@ -849,19 +1015,19 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
 #if FL_KQ_TS_DEFER
     // issued predicated (no branch) and consumed only at the stats ballot, so its L2 round
     // trip overlaps the miss lanes' dedup CAS instead of preceding it
-    const uint32_t need = (hit && old_ts != epoch) ? 1u : 0u;
+    const uint32_t need = (hit && lead && old_ts != epoch) ? 1u : 0u;
     uint32_t prev_ts = epoch;
     asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p atom.global.exch.b32 %0, [%1], %3;\n\t}"
                  : "+r"(prev_ts) : "l"(dv.ts + slot), "r"(need), "r"(epoch) : "memory");
 #else
     bool uhit = false;
-    if (hit && old_ts != epoch) uhit = atomicExch(dv.ts + slot, epoch) != epoch;
+    if (hit && lead && old_ts != epoch) uhit = atomicExch(dv.ts + slot, epoch) != epoch;
 #endif
 
     // A5 miss dedup: the lane whose CAS installs (epoch, fk) owns the miss
     int kind = 0;  // 1 = owner, 2 = duplicate
     uint32_t scr = 0;
-    if (miss) {
+    if (miss && lead) {
       const unsigned long long tag = ((unsigned long long)epoch << 32) | fk;
       while (true) {
         if (cur == tag) { kind = 2; break; }
@@ -877,6 +1043,13 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
       scr = h;
       // first occurrence of the key in canonical (table-major) order: the insert priority
       atomicMin(dv.firstpos + h, ((unsigned long long)(~epoch) << 32) | (uint32_t)(qa.g0 + g));
+    }
+    {  // the group's later lanes are duplicates of its leader's key
+      const uint32_t scr_l = __shfl_sync(kFull, scr, klead);
+      if (miss && !lead) {
+        kind = 2;
+        scr = scr_l;
+      }
     }
 
     const int par = epoch & 1u;
@@ -966,7 +1139,7 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
     __syncthreads();
     if (threadIdx.x == 0) {
       const uint32_t prev = atomicAdd(&dv.ctl->kq_done, 1u);
-      if (prev == gridDim.x - 1) {
+      if (prev == nbid - 1) {
         __threadfence();
         dv.ctl->kq_done = 0;
         const uint32_t epoch = *(volatile uint32_t*)&dv.ctl->epoch;
@@ -990,6 +1163,10 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
           asm volatile("st.relaxed.sys.global.u64 [%0], %1;" ::"l"(dv.ha_bell), "l"((unsigned long long)epoch) : "memory");
           *(volatile uint32_t*)&dv.ctl->ha_rung = epoch;
         }
+        if (qa.nfetch) st_release_gpu_u32(&dv.ctl->kq_end, epoch);  // the fetch CTAs: counts are final
+#ifdef FLECHE_EXPERIMENTS
+        if (dv.exp_buf) dv.exp_buf[dv.exp_slots + 2] = globaltimer_ns();
+#endif
       }
     }
   }
@@ -1221,6 +1398,7 @@ __device__ __forceinline__ void km_ha(const Dev& dv, float* __restrict__ out, co
   constexpr int PER_LANE = ROWS * VEC / 32;      // float4 per lane per piece
   constexpr int INFL = PER_LANE < 16 ? PER_LANE : 16;
   const float* stage = dv.ha_stage + (size_t)(epoch & 1u) * dv.ha_stage_floats;
+  const float* hstage = dv.ha_hstage ? dv.ha_hstage + (size_t)(epoch & 1u) * dv.ha_stage_floats : nullptr;
   // work unit = pieces of this class's miss list (class-local index j; a piece never
   // straddles a 64-row staging block): a staged piece starts as soon as its block is
   // ready, and the zero-copy pieces (blocks >= hcut, or past the class's staging rows) get
@@ -1238,14 +1416,18 @@ __device__ __forceinline__ void km_ha(const Dev& dv, float* __restrict__ out, co
     const uint32_t kb = blk0 + hb;                                     // its absolute block id
     int ok = 0;
 #ifdef FLECHE_EXPERIMENTS
-    if (dv.exp_blk && lane == 0 && pc == 0) dv.exp_blk[kb * 4 + 0] = globaltimer_ns();
+    if (dv.exp_blk && lane == 0 && pc == 0) dv.exp_blk[kb * 8 + 0] = globaltimer_ns();
 #endif
     if (lane == 0 && blo < rcap && hb < hcut) {  // the host threads' share; the rest from the tables
-      ok = ha_wait_block(dv, epoch, kb);
-      if (!ok && pc == 0) ++hato;
+      if (dv.ha_hstage && ld_acquire_gpu_u32(dv.ha_hseen + kb) == epoch) {
+        ok = 2;  // early fetch already moved the block into HBM
+      } else {
+        ok = ha_wait_block(dv, epoch, kb);
+        if (!ok && pc == 0) ++hato;
+      }
     }
 #ifdef FLECHE_EXPERIMENTS
-    if (dv.exp_blk && lane == 0 && pc == 0) dv.exp_blk[kb * 4 + 1] = globaltimer_ns();
+    if (dv.exp_blk && lane == 0 && pc == 0) dv.exp_blk[kb * 8 + 1] = globaltimer_ns();
 #endif
     ok = __shfl_sync(kFull, ok, 0);
     for (uint32_t plo = blo; plo < bhi; plo += ROWS) {  // one iteration: the piece
@@ -1261,7 +1443,7 @@ __device__ __forceinline__ void km_ha(const Dev& dv, float* __restrict__ out, co
           m[h] = mlist[plo + r];
           const TableInfo* ti = dv.tables + m[h].t;
           const bool st = ok && m[h].hst != kNoStage;
-          src[h] = st ? stage + m[h].hst : ti->host + (size_t)(m[h].fk - ti->base) * D;
+          src[h] = st ? (ok == 2 ? hstage : stage) + m[h].hst : ti->host + (size_t)(m[h].fk - ti->base) * D;
           if (st) ++harows;
           hostb += 4ull * D;
         }
@@ -1284,7 +1466,7 @@ __device__ __forceinline__ void km_ha(const Dev& dv, float* __restrict__ out, co
       }
       __syncwarp();
 #ifdef FLECHE_EXPERIMENTS
-      if (dv.exp_blk && lane == 0 && plo == blo) dv.exp_blk[kb * 4 + 2] = globaltimer_ns();
+      if (dv.exp_blk && lane == 0 && plo == blo) dv.exp_blk[kb * 8 + 2] = globaltimer_ns();
 #endif
       // place the rows, 32 at a time (lane = row)
 #pragma unroll
@@ -1349,7 +1531,7 @@ __device__ __forceinline__ void km_ha(const Dev& dv, float* __restrict__ out, co
       __syncwarp();
     }
 #ifdef FLECHE_EXPERIMENTS
-    if (dv.exp_blk && lane == 0) dv.exp_blk[kb * 4 + 3] = globaltimer_ns();
+    if (dv.exp_blk && lane == 0) dv.exp_blk[kb * 8 + 3] = globaltimer_ns();
 #endif
   }
 }

@@ -1,12 +1,12 @@
 #!/bin/bash
 # One parameterised GPU batch (run under gpurun from the repo root):
-#   tools/gpu_r02.sh TAG "pytest args|-" "bench-variant ..." 
+#   tools/gpu_r02.sh TAG "pytest args (e.g. tests -m gpu)|-" "bench-variant ..." 
 # Each bench variant is "name:ENV=V,ENV2=V2:bench args" and writes gpurun_out/<TAG>_<name>.json.
 TAG=$1; shift
 PYT=$1; shift
 mkdir -p gpurun_out
 if [ "$PYT" != "-" ]; then
-  timeout 1500 python -m pytest tests -x -q $PYT > gpurun_out/${TAG}_pytest.txt 2>&1
+  timeout 1500 python -m pytest -x -q $PYT > gpurun_out/${TAG}_pytest.txt 2>&1
   tail -3 gpurun_out/${TAG}_pytest.txt
 fi
 for v in "$@"; do

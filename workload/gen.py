@@ -91,6 +91,26 @@ def fill_table(dst: np.ndarray, t: int, mode: int = 0, row0: int = 0, nthreads: 
     lib().flg_fill_table(seeds()["val"], t, row0, rows, d, d, mode, dst.ctypes.data, nthreads)
 
 
+def alloc_host_f32(n: int) -> np.ndarray:
+    """A float32 host buffer of n elements backed by transparent huge pages where the kernel
+    allows it (anonymous mmap + MADV_HUGEPAGE; THP "madvise" mode).  A host tier of several
+    GiB in 4 KiB pages makes every scattered row read of the host-assist threads a TLB miss
+    and page walk; 2 MiB pages keep their gather near the memory system's rate."""
+    import mmap
+
+    nbytes = max(4, 4 * int(n))
+    if nbytes < (64 << 20) or os.environ.get("FLECHE_TIER_NO_THP"):  # (A/B: 4 KiB pages)
+        return np.empty(int(n), dtype=np.float32)
+    mm = mmap.mmap(-1, nbytes, flags=mmap.MAP_PRIVATE | mmap.MAP_ANONYMOUS,
+                   prot=mmap.PROT_READ | mmap.PROT_WRITE)
+    if hasattr(mm, "madvise") and hasattr(mmap, "MADV_HUGEPAGE"):
+        try:
+            mm.madvise(mmap.MADV_HUGEPAGE)
+        except OSError:
+            pass
+    return np.frombuffer(mm, dtype=np.float32, count=int(n))
+
+
 def make_tables(cards, dims, mode: int = 0, nthreads: int = 0, buf: np.ndarray | None = None):
     """One contiguous float32 buffer holding every table row-major; returns (buf, [views]).
     `buf` (optional): a caller-provided float32 buffer of at least sum(c_t * d_t) elements
@@ -98,7 +118,7 @@ def make_tables(cards, dims, mode: int = 0, nthreads: int = 0, buf: np.ndarray |
     sizes = [int(c) * int(d) for c, d in zip(cards, dims)]
     total = sum(sizes)
     if buf is None:
-        buf = np.empty(total, dtype=np.float32)
+        buf = alloc_host_f32(total)
     assert buf.dtype == np.float32 and buf.flags["C_CONTIGUOUS"] and buf.size >= total
     buf = buf[:total]
     views = []
