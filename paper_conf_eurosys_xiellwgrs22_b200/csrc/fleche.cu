@@ -87,6 +87,10 @@ struct fleche_ctx {
   int kq_tma = 0;      // KQ's hit gather by bulk copies through shared memory (row width 32 or 64; 0 = registers)
   size_t kq_smem = 0;  // its dynamic shared memory (4 warps x 32 rows)
   int kf_ctas = 0;     // host-assisted early fetch: KQ CTAs that copy staged blocks into HBM (0 = off)
+  // ... from this many lookups per batch (FLECHE_HA_EARLY_MIN): a short KQ ends before the
+  // host threads have staged much (cfg2, 213K lookups: 111 vs 106 us per batch without;
+  // cfg5, 1.7M: 495 vs 570 us, profiles/)
+  int64_t kf_min = 524288;
   bool per_table_launch = false;
   // decoupled hit copy (uniform layout): KG on a side stream, forked after KQ, joined after KM
   bool decoupled = false;
@@ -650,7 +654,7 @@ fleche_status launch_query(fleche_ctx* c, const int64_t* const* ids, const int64
   qa.ncls = ka.ncls;
   for (int k = 0; k < ka.ncls; ++k) qa.cls_dim[k] = c->cls_dim[k];
   if (total > 0 && !c->per_table_launch) {
-    qa.nfetch = (qa.ha_bell && !decouple) ? c->kf_ctas : 0;
+    qa.nfetch = (qa.ha_bell && !decouple && total >= c->kf_min) ? c->kf_ctas : 0;
     const int64_t blocks = (total + 127) / 128 + qa.nfetch;
     launch_k(kPdlKQ, kq_fn<MAXT>(c->kq_tma), (unsigned)blocks, 128, c->kq_smem, s, qa, c->dv);
     c->kernels++;
@@ -1051,6 +1055,7 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
     // blocks into an HBM copy while the lookups run
     c->kf_ctas = (int)env_u("FLECHE_HA_EARLY", 1) ? (int)std::min<uint64_t>(64, std::max<uint64_t>(1, env_u("FLECHE_KF_CTAS", 16))) : 0;
     dv.ha_kf_tail = (uint32_t)env_u("FLECHE_KF_TAIL", 0);
+    c->kf_min = (int64_t)env_u("FLECHE_HA_EARLY_MIN", 524288);
     if (c->kf_ctas) {
       if (cudaMalloc((void**)&dv.ha_hstage, 2ull * 4ull * h->stage_floats) != cudaSuccess ||
           cudaMalloc((void**)&dv.ha_hseen, 4ull * h->blk_cap) != cudaSuccess ||
@@ -1083,8 +1088,10 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
     for (int i = 0; i < h->nthreads; ++i) h->th.emplace_back(ha_worker, h, i);
   }
 #ifdef FLECHE_EXPERIMENTS
-  if (cudaMalloc((void**)&dv.exp_buf, ((size_t)c->km_blocks * 4 * 4 + 8) * 8) != cudaSuccess) return fail(FLECHE_ENOMEM);
-  cudaMemset(dv.exp_buf, 0, ((size_t)c->km_blocks * 4 * 4 + 8) * 8);
+  // KM warps x 4, then [exp_slots + 0..7] KQ stamps, [exp_slots + 8 + w] early-fetch warp w's exit,
+  // [exp_slots + 264 + (epoch % 64) * 4 + {0,1,2}] per-batch ring: KQ start, lookups end, last fetch exit
+  if (cudaMalloc((void**)&dv.exp_buf, ((size_t)c->km_blocks * 4 * 4 + 8 + 512) * 8) != cudaSuccess) return fail(FLECHE_ENOMEM);
+  cudaMemset(dv.exp_buf, 0, ((size_t)c->km_blocks * 4 * 4 + 8 + 512) * 8);
   dv.exp_slots = (uint32_t)c->km_blocks * 16;
   if (c->ha) {
     if (cudaMalloc((void**)&dv.exp_blk, ((size_t)c->ha->blk_cap * 8) * 8) != cudaSuccess) return fail(FLECHE_ENOMEM);
@@ -1871,7 +1878,7 @@ extern "C" __attribute__((visibility("default"))) fleche_status fleche_exp_timel
                                                                                     size_t n) {
   if (!c || !host) return FLECHE_EINVAL;
   if (c->have_last) cudaStreamSynchronize(c->last_stream);
-  const size_t m = std::min(n, (size_t)c->km_blocks * 16 + 8);
+  const size_t m = std::min(n, (size_t)c->km_blocks * 16 + 8 + 512);
   return cudaMemcpy(host, c->dv.exp_buf, m * 8, cudaMemcpyDeviceToHost) == cudaSuccess ? FLECHE_OK : FLECHE_ECUDA;
 }
 // host-assist threads: CLOCK_REALTIME (ns) when each thread saw the doorbell of epoch e

@@ -808,8 +808,13 @@ __device__ __noinline__ void kq_fetch(const QArgs<MAXT>& qa, const Dev& dv) {
       const int D = qa.cls_dim[c];
       const uint32_t vec = (uint32_t)D / 4u, n4 = (uint32_t)kHaBlock * vec;
       const size_t base = (size_t)kb * kHaBlock * dv.ha_row_floats;
+      bool quit = false;
 #pragma unroll 1
       for (uint32_t q0 = 0; q0 < n4; q0 += 32u * 8u) {
+        if (!dv.ha_kf_tail && ld_acquire_gpu_u32(&dv.ctl->kq_end) == epoch) {  // lookups done: KM takes over
+          quit = true;
+          break;
+        }
         float4 v[8];
 #pragma unroll
         for (int i = 0; i < 8; ++i) {
@@ -824,6 +829,7 @@ __device__ __noinline__ void kq_fetch(const QArgs<MAXT>& qa, const Dev& dv) {
         }
       }
       __syncwarp();
+      if (quit) return;
       if (lane == 0) {
         __threadfence();
         st_release_gpu_u32(dv.ha_hseen + kb, epoch);
@@ -856,6 +862,13 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
   pdl_wait();  // the previous batch (or the caller's producer of ids) has completed
   if ((int)blockIdx.x < qa.nfetch) {  // early-fetch CTA (no lookups)
     kq_fetch<MAXT>(qa, dv);
+#ifdef FLECHE_EXPERIMENTS
+    if (dv.exp_buf && (threadIdx.x & 31) == 0 && blockIdx.x * 4 + threadIdx.x / 32 < 256) {
+      const unsigned long long tx = globaltimer_ns();
+      dv.exp_buf[dv.exp_slots + 8 + blockIdx.x * 4 + threadIdx.x / 32] = tx;
+      atomicMax(dv.exp_buf + dv.exp_slots + 264 + (*(volatile uint32_t*)&dv.ctl->epoch % 64) * 4 + 2, tx);
+    }
+#endif
     return;
   }
   const uint32_t bid = blockIdx.x - (uint32_t)qa.nfetch, nbid = gridDim.x - (uint32_t)qa.nfetch;  // lookup CTAs
@@ -870,7 +883,12 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
     s_scan[qa.n] = acc;
   }
 #ifdef FLECHE_EXPERIMENTS
-  if (dv.exp_buf && bid == 0 && threadIdx.x == 0) dv.exp_buf[dv.exp_slots + 1] = globaltimer_ns();
+  if (dv.exp_buf && bid == 0 && threadIdx.x == 0) {
+    const unsigned long long tx = globaltimer_ns();
+    dv.exp_buf[dv.exp_slots + 1] = tx;
+    dv.exp_buf[dv.exp_slots + 264 + (*(volatile uint32_t*)&dv.ctl->epoch % 64) * 4 + 0] = tx;
+    dv.exp_buf[dv.exp_slots + 264 + (*(volatile uint32_t*)&dv.ctl->epoch % 64) * 4 + 2] = 0;
+  }
 #endif
   if (dv.ha && bid == 0 && threadIdx.x == 0)  // the host threads start streaming this batch's requests
     asm volatile("st.relaxed.sys.global.u64 [%0], %1;" ::"l"(dv.ha_start),
@@ -1165,7 +1183,10 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
         }
         if (qa.nfetch) st_release_gpu_u32(&dv.ctl->kq_end, epoch);  // the fetch CTAs: counts are final
 #ifdef FLECHE_EXPERIMENTS
-        if (dv.exp_buf) dv.exp_buf[dv.exp_slots + 2] = globaltimer_ns();
+        if (dv.exp_buf) {
+          dv.exp_buf[dv.exp_slots + 2] = globaltimer_ns();
+          dv.exp_buf[dv.exp_slots + 264 + (epoch % 64) * 4 + 1] = dv.exp_buf[dv.exp_slots + 2];
+        }
 #endif
       }
     }

@@ -25,10 +25,10 @@ lib = fl.binding._lib
 for f in (lib.fleche_exp_timeline, lib.fleche_exp_ha_times, lib.fleche_exp_ha_blocks):
     f.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_size_t]
 nth = int(os.environ.get("FLECHE_HA_THREADS", "12"))
-out = torch.empty(sum(w.batch_size * d for d in w.dims), device="cuda")
-pre = [[torch.from_numpy(x).cuda() for x in w.batch(b).ids] for b in range(nbatch)]
-for b in range(nbatch):
-    c.query(pre[b], out)
+outs = [torch.empty(sum(w.batch_size * d for d in w.dims), device="cuda") for _ in range(4)]
+pre = [[torch.from_numpy(x).cuda() for x in w.batch(b).ids] for b in range(min(nbatch, 64))]
+for b in range(nbatch):  # like bench.py: back to back, rotating output buffers
+    c.query(pre[b % len(pre)], outs[b % 4])
 torch.cuda.synchronize()
 buf = np.zeros(c.max_lookups * 16 // 256 * 16 + 200000, np.uint64)
 lib.fleche_exp_timeline(c.h, buf.ctypes.data, buf.size)
@@ -40,8 +40,14 @@ lib.fleche_exp_ha_blocks(c.h, blk.ctypes.data, nb)
 blk = blk.reshape(-1, 7).astype(np.int64)
 e = nbatch
 nz = np.nonzero(buf)[0]
-# KQ's stamps are the last two non-zero words (exp_slots + 1: start, + 2: lookups end)
-kq0, kqend = int(buf[nz[-2]]), int(buf[nz[-1]])
+# KQ's stamps: exp_slots + 1: start, + 2: lookups end; exp_slots + 8 + w: fetch warp w's exit
+exp_slots = int(os.environ.get("KM_BLOCKS", "592")) * 16
+kq0, kqend = int(buf[exp_slots + 1]), int(buf[exp_slots + 2])
+kf_exit = buf[exp_slots + 8: exp_slots + 8 + 256].astype(np.int64)
+kf_exit = kf_exit[kf_exit > 0]
+if len(kf_exit):
+    print("early-fetch warps exit: p0 %.1f p50 %.1f p100 %.1f us after KQ start (lookups end %.1f)" % (
+        (kf_exit.min() - kq0) / 1e3, (np.median(kf_exit) - kq0) / 1e3, (kf_exit.max() - kq0) / 1e3, (kqend - kq0) / 1e3))
 seen = hbuf[(e % 64) * 128: (e % 64) * 128 + nth].astype(np.int64)
 done = hbuf[(e % 64) * 128 + 64: (e % 64) * 128 + 64 + nth].astype(np.int64)
 tail = buf[-200000:]
