@@ -412,7 +412,7 @@ def run_config(args, w, P, W, K, world, rank, local, dist, primary: bool, extra_
     for i in range(W):
         step(i, outs[i % 4])
     torch.cuda.synchronize()
-    reps, stats = [], []
+    reps, stats, submit_us = [], [], []
     r0 = cache.shard_stats() if sharded else None
     s0 = cache.stats()
     tw0 = time.perf_counter()
@@ -422,8 +422,10 @@ def run_config(args, w, P, W, K, world, rank, local, dist, primary: bool, extra_
         torch.cuda.synchronize()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
+        ts0 = time.perf_counter()
         for k in range(K):
             step(W + rep * K + k, outs[k % 4])
+        submit_us.append((time.perf_counter() - ts0) * 1e6 / K)
         e1.record(stream)
         torch.cuda.synchronize()
         if dist:
@@ -525,6 +527,8 @@ def run_config(args, w, P, W, K, world, rank, local, dist, primary: bool, extra_
             "step_frac_note": "T_roof = max(HBM bytes / HBM BW, host bytes / link BW) over the measured step; "
                               "measured: MEASURED_PEAKS hbm_gbs + in-run copy-engine H2D; datasheet: 8 TB/s + 63 GB/s"}
     res = {"value": value, "ms_per_step": ms_step, "repetitions_ms_per_step": [r / K for r in reps],
+           # host time to submit one step (a step is host-bound when this reaches the device time)
+           "submit_us_per_step": sorted(submit_us)[len(submit_us) // 2],
            "hit_ratio": hit, "hit_ratio_unique": uhit, "unique_misses_per_step": dst["unique_misses"] / steps_timed,
            "roofline": roof, "gpu_launches_per_step": dst["kernels_launched"] / steps_timed,
            "gpu_launches": int(dst["kernels_launched"] / nrep), "clocks": clk,
@@ -719,7 +723,7 @@ def main():
             "metric": "embedding lookups/s", "value": r["value"], "unit": "Mkeys/s", "n_gpus": world, "steps": K,
             "warmup": W, "ms_per_step": r["ms_per_step"], "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "f32", "data": "synthetic", "config": cf,
-            "repetitions_ms_per_step": r["repetitions_ms_per_step"],
+            "repetitions_ms_per_step": r["repetitions_ms_per_step"], "submit_us_per_step": r["submit_us_per_step"],
             "hit_ratio": r["hit_ratio"], "hit_ratio_unique": r["hit_ratio_unique"],
             "unique_misses_per_step": r["unique_misses_per_step"],
             "p50_batch_latency_us": r["p50_batch_latency_us"], "p99_batch_latency_us": r["p99_batch_latency_us"],

@@ -48,6 +48,7 @@ struct HostAssist {
   float* stage = nullptr;              // [2][stage_floats]
   uint32_t req_cap = 0;
   bool nt_stores = true;  // FLECHE_HA_NT=0: plain memcpy into the staging buffer (A/B)
+  bool stream = true;     // FLECHE_HA_STREAM=0: start on the doorbell, not on KQ's start word (A/B)
   uint64_t delay_ns = 0;  // FLECHE_HA_DELAY_US: fault injection (tests): each block is gathered this late
   uint64_t stage_floats = 0;
   // the tables as the host threads see them
@@ -336,8 +337,10 @@ void ha_worker(HostAssist* h, int me) {
   uint32_t last = 0;
   uint64_t t_last = now_ns();
   uint64_t spins = 0;
+  // FLECHE_HA_STREAM=0: wait for the doorbell (every request written) instead of the start word
+  const unsigned long long* wake = h->stream ? h->start : h->bell;
   while (!h->stop.load(std::memory_order_relaxed)) {
-    const uint32_t e = (uint32_t)__atomic_load_n(h->start, __ATOMIC_ACQUIRE);
+    const uint32_t e = (uint32_t)__atomic_load_n(wake, __ATOMIC_ACQUIRE);
     if (e == last) {
       if ((++spins & 1023) == 0) idle(t_last);
       continue;
@@ -481,7 +484,7 @@ void ha_worker(HostAssist* h, int me) {
       // waiting for requests: give up on this batch when a newer one has started, or when a
       // request never arrived ~1 ms after the descriptor (KM's poller times out and reads
       // those blocks zero-copy)
-      if ((uint32_t)__atomic_load_n(h->start, __ATOMIC_ACQUIRE) != e) break;
+      if ((uint32_t)__atomic_load_n(wake, __ATOMIC_ACQUIRE) != e) break;
       if (have_d && now - std::max(t_d, t_prog) > 1000000ull) break;
       if ((++spins & 1023) == 0) idle(t_prog);
     }
@@ -598,7 +601,7 @@ cudaError_t launch_k(int which, void (*kern)(KArgs...), unsigned grid, unsigned 
 // barrier before the restore needs every CTA resident; km_blocks never exceeds that).
 void launch_miss(fleche_ctx* c, cudaStream_t s, const KMArgs& ka) {
   static const bool coop = !(getenv("FLECHE_KM_COOP") && !atoi(getenv("FLECHE_KM_COOP")));  // A/B of the launch cost only
-  launch_k(coop ? kPdlCoop : kPdlNone, km_fn(c->dv.bytes != 0, c->cls_dim.size() == 1 ? c->max_dim : 0), c->km_blocks, 128, c->km_smem, s,
+  launch_k(coop ? kPdlCoop : kPdlKM, km_fn(c->dv.bytes != 0, c->cls_dim.size() == 1 ? c->max_dim : 0), c->km_blocks, 128, c->km_smem, s,
            c->dv, ka);
   c->kernels += 1;
 }
@@ -1082,6 +1085,7 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
     }
     h->nt_stores = env_u("FLECHE_HA_NT", 1) != 0 && __builtin_cpu_supports("avx2");
     h->delay_ns = env_u("FLECHE_HA_DELAY_US", 0) * 1000ull;
+    h->stream = env_u("FLECHE_HA_STREAM", 1) != 0;
     h->host.assign(cfg->host_tables, cfg->host_tables + n);
     h->card = c->card;
     h->dims = c->dims;

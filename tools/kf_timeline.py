@@ -20,15 +20,15 @@ w = configs.get(sys.argv[1] if len(sys.argv) > 1 else "cfg2")
 nbatch = int(sys.argv[2]) if len(sys.argv) > 2 else 200
 _, tabs = w.make_tables()
 N = w.batch_size * w.n
-c = fl.FlatCache(w.cards, w.dims, tabs, w.cache_bytes, N, 0, 1.0, 0, 0x9E3779B9, fl.binding.FLAG_HOST_ASSIST)
+c = fl.FlatCache(w.cards, w.dims, tabs, w.cache_bytes, N, 0, 1.0, 0, 0x9E3779B9)
 lib = fl.binding._lib
 for f in (lib.fleche_exp_timeline, lib.fleche_exp_ha_times, lib.fleche_exp_ha_blocks):
     f.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_size_t]
 nth = int(os.environ.get("FLECHE_HA_THREADS", "12"))
 outs = [torch.empty(sum(w.batch_size * d for d in w.dims), device="cuda") for _ in range(4)]
-pre = [[torch.from_numpy(x).cuda() for x in w.batch(b).ids] for b in range(min(nbatch, 64))]
-for b in range(nbatch):  # like bench.py: back to back, rotating output buffers
-    c.query(pre[b % len(pre)], outs[b % 4])
+pre = [[torch.from_numpy(x).cuda() for x in w.batch(b).ids] for b in range(nbatch)]
+for b in range(nbatch):  # like bench.py: fresh batches back to back, rotating output buffers
+    c.query(pre[b], outs[b % 4])
 torch.cuda.synchronize()
 buf = np.zeros(c.max_lookups * 16 // 256 * 16 + 200000, np.uint64)
 lib.fleche_exp_timeline(c.h, buf.ctypes.data, buf.size)
@@ -68,7 +68,14 @@ print(f"{len(cur)} blocks of the last batch; GPU times rel. to KQ start, CPU rel
 for q in (0, 10, 50, 90, 100):
     f = lambda col, fn=rg: np.percentile(fn(cur[cur[:, col] > 0, col]), q) if (cur[:, col] > 0).any() else float("nan")  # noqa: E731
     print(f"  p{q:3d}: CPU published {f(6, rc):7.1f}  KF mirrored {f(4):7.1f}  KF copied {f(5):7.1f}  "
-          f"KM wait {f(0):7.1f}  KM done {f(3):7.1f}")
+          f"KM wait {f(0):7.1f}  KM ready {f(1):7.1f}  KM landed {f(2):7.1f}  KM done {f(3):7.1f}")
+ok = cur[(cur[:, 1] > 0) & (cur[:, 6] > 0) & (cur[:, 2] > 0) & (cur[:, 3] > 0)]
+if len(ok):
+    lag_seen = (ok[:, 1] - g0) / 1e3 - (ok[:, 6] - c0) / 1e3
+    print("  per block: published->KM saw ready p50 %.1f p90 %.1f | ready->landed p50 %.1f p90 %.1f | landed->done p50 %.1f p90 %.1f us" % (
+        np.median(lag_seen), np.percentile(lag_seen, 90), np.median((ok[:, 2] - ok[:, 1]) / 1e3),
+        np.percentile((ok[:, 2] - ok[:, 1]) / 1e3, 90), np.median((ok[:, 3] - ok[:, 2]) / 1e3),
+        np.percentile((ok[:, 3] - ok[:, 2]) / 1e3, 90)))
 m = cur[(cur[:, 4] > 0) & (cur[:, 5] > 0)]
 if len(m):
     print(f"  copy after mirror: p50 {np.median((m[:, 5] - m[:, 4]) / 1e3):.1f} us, p90 {np.percentile((m[:, 5] - m[:, 4]) / 1e3, 90):.1f}")
