@@ -314,8 +314,9 @@ __attribute__((target("avx2"))) void stage_row(float* dst, const float* src, siz
 // as its request carries this batch's tags, with non-temporal stores, and a block's ready
 // word (= epoch) is published once its rows are in place -- a full block at once, the
 // class's last partial block once the doorbell descriptor (written by KQ's last CTA) gives
-// the class's count.  The host threads take only their share of the blocks (ha_host_blk
-// with the split the start word carries); the others are the GPU's (the unified index).  Spins while batches keep coming; after ~20 ms without progress it
+// the class's count.  Blocks past the descriptor's host share (hcut) are not started; a
+// block gathered before the descriptor arrived and then left to KM's zero-copy share is
+// simply not read.  Spins while batches keep coming; after ~20 ms without progress it
 // polls every 20 us (an idle ctx burns no core).  No `pause` in the spin: on a KVM guest
 // it can trigger pause-loop exits that deschedule the vCPU.
 void ha_worker(HostAssist* h, int me) {
@@ -339,8 +340,7 @@ void ha_worker(HostAssist* h, int me) {
   // FLECHE_HA_STREAM=0: wait for the doorbell (every request written) instead of the start word
   const unsigned long long* wake = h->stream ? h->start : h->bell;
   while (!h->stop.load(std::memory_order_relaxed)) {
-    const unsigned long long wv = __atomic_load_n(wake, __ATOMIC_ACQUIRE);
-    const uint32_t e = (uint32_t)wv;
+    const uint32_t e = (uint32_t)__atomic_load_n(wake, __ATOMIC_ACQUIRE);
     if (e == last) {
       if ((++spins & 1023) == 0) idle(t_last);
       continue;
@@ -411,32 +411,17 @@ void ha_worker(HostAssist* h, int me) {
     }
     uint64_t t_prog = now_ns();
     bool delayed = false;  // fault injection: once per block
-    // the batch's split (ha_host_blk): the start word carries it; the doorbell mode reads it
-    // from the descriptor
-    uint32_t frac = h->stream ? (uint32_t)(wv >> 32) : 0u;
-    bool have_frac = h->stream;
     while (true) {
       poll_desc();
-      if (have_d && !have_frac) {
-        frac = d.frac;
-        have_frac = true;
-      }
-      bool all_done = !have_frac ? false : true, progressed = false;
-      for (int c = 0; c < 8 && have_frac; ++c) {
+      bool all_done = true, progressed = false;
+      for (int c = 0; c < 8; ++c) {
         Cursor& q = cur[c];
         if (q.done) continue;
-        const uint64_t rb = h->rbase[c];
-        while (!q.done && !ha_host_blk((uint32_t)(q.kb - rb / kHaBlock), frac)) {  // the GPU's block: skip
-          q.kb += T;
-          q.i = q.kb * kHaBlock;
-          q.done = q.i >= rb + h->rcap[c];
-        }
-        if (q.done) continue;
-        const uint64_t lo = q.kb * kHaBlock;
+        const uint64_t rb = h->rbase[c], lo = q.kb * kHaBlock;
         uint64_t hi = std::min<uint64_t>(lo + kHaBlock, rb + h->rcap[c]);
-        if (have_d) {  // the batch's count is known
+        if (have_d) {  // the batch's count and the host share are known
           const uint64_t nrow = std::min<uint64_t>(d.cnt[c], h->rcap[c]);
-          if (q.kb - rb / kHaBlock >= d.nblk[c] || lo >= rb + nrow) {
+          if (q.kb - rb / kHaBlock >= d.hcut[c] || lo >= rb + nrow) {
             q.done = true;
             continue;
           }
@@ -526,7 +511,7 @@ void free_all(fleche_ctx* c) {
                   c->dv.miss, c->dv.dup, c->dv.ctl, c->dv.stats, c->d_tables, c->d_ids_stage, c->d_out_stage,
                   c->d_pool_stage, c->d_kdec, c->rd.scratch, c->rd.slotval, c->rd.inv, c->rd.region, c->rd.cnt,
                   c->rd.prefix, c->rd.done, c->rd.stats, c->d_slots, c->d_age_hist, c->d_prefill_out,
-                  c->d_out_stage2, c->dv.ha_seen, c->dv.ha_hstage, c->dv.ha_hseen, c->dv.ha_frec};
+                  c->d_out_stage2, c->dv.ha_seen, c->dv.ha_hstage, c->dv.ha_hseen};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   for (auto& r : c->registered) cudaHostUnregister(r.first);
@@ -1072,12 +1057,10 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
     // early fetch (FLECHE_HA_EARLY=0 turns it off): KQ's first kf_ctas CTAs move staged
     // blocks into an HBM copy while the lookups run
     c->kf_ctas = (int)env_u("FLECHE_HA_EARLY", 1) ? (int)std::min<uint64_t>(64, std::max<uint64_t>(1, env_u("FLECHE_KF_CTAS", 16))) : 0;
+    dv.ha_kf_tail = (uint32_t)env_u("FLECHE_KF_TAIL", 0);
     c->kf_min = (int64_t)env_u("FLECHE_HA_EARLY_MIN", 524288);
-    dv.ha_kf_gpu = (uint32_t)env_u("FLECHE_KF_GPU", 0);
     if (c->kf_ctas) {
       if (cudaMalloc((void**)&dv.ha_hstage, 2ull * 4ull * h->stage_floats) != cudaSuccess ||
-          cudaMalloc((void**)&dv.ha_frec, sizeof(FetchRec) * (size_t)h->req_cap) != cudaSuccess ||
-          cudaMemset(dv.ha_frec, 0, sizeof(FetchRec) * (size_t)h->req_cap) != cudaSuccess ||
           cudaMalloc((void**)&dv.ha_hseen, 4ull * h->blk_cap) != cudaSuccess ||
           cudaMemset(dv.ha_hseen, 0, 4ull * h->blk_cap) != cudaSuccess)
         return fail(FLECHE_ENOMEM);

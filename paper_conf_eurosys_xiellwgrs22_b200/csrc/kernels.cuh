@@ -107,7 +107,7 @@ struct MissRec {  // one unique missed key (its owner lookup)
   uint32_t fk;    // flat key
   uint32_t scr;   // scratch slot of the key (head of its duplicate chain)
   int32_t t;      // table
-  int32_t pad;    // the batch epoch that wrote the record
+  int32_t pad;
   uint64_t hst;   // host-assisted: float offset of the row's staging slot (kNoStage: read the table)
 };
 constexpr unsigned long long kNoStage = ~0ull;
@@ -179,18 +179,9 @@ __host__ __device__ __forceinline__ bool ha_req_current(const HaReq& r, uint32_t
 struct HaDesc {            // written by the doorbell ringer, read by the host threads
   uint32_t epoch;
   uint32_t cnt[8];         // unique misses of width class c this batch
-  uint32_t nblk[8];        // staged blocks of class c (ha_nblk); the host threads take those with ha_host_blk
-  uint32_t frac;           // the host share (x 2^-16) of this batch's split
-  uint32_t epoch2;         // = epoch, written last: the host accepts the descriptor once both match
-};
-// Early zero-copy fetch: KQ's owner lane of a staged miss also writes this 16-byte record
-// (one vector store: never torn) at its staging row, so KQ's fetch warps can read the
-// unified index's share of the rows while the lookups are still running.
-struct FetchRec {
-  uint32_t fk;     // flat key
-  int32_t t;       // table
-  uint32_t epoch;  // the batch that wrote it
+  uint32_t hcut[8];        // split: the host threads stage class c's blocks < hcut[c], KM reads the rest itself
   uint32_t pad;
+  uint32_t epoch2;         // = epoch, written last: the host accepts the descriptor once both match
 };
 
 struct Dev {
@@ -234,7 +225,6 @@ struct Dev {
   float* ha_stage;             // [2][ha_stage_floats]
   float* ha_hstage;            // early fetch: [2][ha_stage_floats] (HBM) copy of the staged blocks
   uint32_t* ha_hseen;          // early fetch: [ha_blk_cap] (HBM) epoch once a block's rows are in ha_hstage
-  FetchRec* ha_frec;           // early fetch: [ha_req_cap] (HBM) the miss of each staging row (FetchRec)
   uint32_t ha_req_cap, ha_blk_cap;  // staging rows (= request slots) and blocks per epoch parity
   uint32_t ha_rbase[8];        // first staging row of width class c (a multiple of kHaBlock)
   uint32_t ha_rcap[8];         // staging rows of class c (a multiple of kHaBlock): its misses beyond go zero-copy
@@ -245,8 +235,7 @@ struct Dev {
   uint32_t ha_frac_fixed;      // 1 = FLECHE_HA_FRAC fixed the host threads' share (no tuning loop)
   uint32_t ha_min_rows;        // batches with fewer unique misses stay all zero-copy (the split loses there)
   uint32_t ha_unit_pieces;     // KM work unit = this many 16-row pieces (0: adaptive to the batch)
-  uint32_t ha_kf_gpu;          // early fetch: 1 = the fetch warps also read the GPU's blocks zero-copy during KQ
-                               // (FLECHE_KF_GPU; off: its translation-bound reads stall KQ's lookups, 29 -> 87-165 us at cfg2)
+  uint32_t ha_kf_tail;         // early fetch: 1 = the fetch CTAs copy every host block (KQ ends after them), 0 = stop with the lookups
 #ifdef FLECHE_EXPERIMENTS
   int32_t exp_mode;  // timing experiments only (libfleche_exp.so); breaks semantics
   int32_t exp_pad;
@@ -437,16 +426,10 @@ __device__ __forceinline__ void st_release_gpu_u64(unsigned long long* p, unsign
 // width class c (its class-local miss-list index), for j < ha_rcap[c]; block b = r / 64 is
 // always the same 64 rows of staging memory, owned by host thread b % T in every batch
 // (a stalled thread can only ever rewrite its own blocks, whatever the batch geometry).
-// The host threads take the class's staged blocks that ha_host_blk assigns them.
-__host__ __device__ __forceinline__ uint32_t ha_nblk(uint32_t cnt, uint32_t rcap) {  // staged blocks of a class
-  return ((cnt < rcap ? cnt : rcap) + kHaBlock - 1) / kHaBlock;
-}
-// The split of a class's staged blocks between the host threads (share f = frac_q16 / 2^16)
-// and the GPU's own zero-copy reads (the unified index, 1 - f): block b is the host's iff
-// floor((b + 1) f) > floor(b f) -- interleaved evenly and known from the block index alone,
-// so both sides can start on their blocks before the batch's miss count is known.
-__host__ __device__ __forceinline__ bool ha_host_blk(uint32_t b, uint32_t frac_q16) {
-  return (((unsigned long long)(b + 1u) * frac_q16) >> 16) > (((unsigned long long)b * frac_q16) >> 16);
+// The host threads take class c's blocks below hcut (its share of the class's staged rows).
+__host__ __device__ __forceinline__ uint32_t ha_hcut(uint32_t cnt, uint32_t rcap, uint32_t frac_q16) {
+  const uint32_t nb = ((cnt < rcap ? cnt : rcap) + kHaBlock - 1) / kHaBlock;
+  return (uint32_t)(((unsigned long long)nb * frac_q16 + 65535ull) >> 16);
 }
 
 // The poller warp: mirror the ready words of staging blocks [kb0, kend) into HBM until all
@@ -461,12 +444,10 @@ __device__ __forceinline__ uint32_t ld_relaxed_sys_u32(const uint32_t* p) {
   asm volatile("ld.relaxed.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
   return v;
 }
-// Ready words of the batch's host blocks: the ha_host_blk(frac) blocks among class c's
-// [rbase_c / 64, + n_c) (the GPU's own blocks count as mirrored).
+// Ready words of the batch's host blocks: class c's blocks [rbase_c / 64, + hcut_c).
 struct HaBlocks {
   uint32_t lo[8], n[8];
   int ncls;
-  uint32_t frac;
 };
 __device__ __forceinline__ void ha_poll(const Dev& dv, uint32_t epoch, const HaBlocks& hb, int lane) {
   const uint32_t* ready = dv.ha_ready + (size_t)(epoch & 1u) * dv.ha_blk_cap;
@@ -488,9 +469,7 @@ __device__ __forceinline__ void ha_poll(const Dev& dv, uint32_t epoch, const HaB
 #pragma unroll
         for (int q = 0; q < 4; ++q) {
           const uint32_t k = k0 + 32 * q + lane;
-          v[q] = (k < kend && ha_host_blk(k - hb.lo[c], hb.frac) && ld_acquire_gpu_u32(dv.ha_seen + k) != epoch)
-                     ? ld_relaxed_sys_u32(ready + k)
-                     : ~0u;
+          v[q] = (k < kend && ld_acquire_gpu_u32(dv.ha_seen + k) != epoch) ? ld_relaxed_sys_u32(ready + k) : ~0u;
         }
         uint32_t newly = 0;
 #pragma unroll
@@ -722,58 +701,64 @@ __device__ __forceinline__ void bulk_s2g(void* gmem, const void* smem, unsigned 
   asm volatile("cp.async.bulk.commit_group;" ::: "memory");
 }
 
-// Early fetch (host-assisted): the first qa.nfetch CTAs of KQ do no lookups; they start
-// the batch's host-link traffic WHILE the other CTAs are still indexing, so the link is
-// busy during KQ instead of only during KM.  The staged blocks are split between the host
-// threads and the GPU by ha_host_blk (interleaved, known from the block index alone):
-//  * the GPU's blocks (FLECHE_KF_GPU=1 only): as soon as a block's misses are known (KQ's
-//    owner lanes write a FetchRec per staging row), a fetch warp reads its rows zero-copy
-//    from the tables -- the unified index's share of the batch -- into the HBM copy.  Off
-//    by default: those translation-bound reads stall the lookups' own memory accesses
-//    (cfg2 KQ lookups 29 -> 87-165 us, profiles/);
-//  * the host threads' blocks: warp 0 of CTA 0 mirrors the threads' ready words into
-//    ha_seen (as KM's poller does) and a fetch warp copies each published block into HBM.
-// Each fetch warp takes class-local blocks b = w - 1 + k * W of every class; a block
-// finished in HBM gets ha_hseen[kb] = epoch and KM reads it from there.  Everything stops
-// when the last lookup CTA has finished (ctl->kq_end = epoch) -- a block in flight is
-// abandoned -- and KM fetches whatever is not in HBM exactly as without early fetch.
+// Early fetch (host-assisted): the first qa.nfetch CTAs of KQ do no lookups; they move the
+// batch's staged blocks over the link into HBM WHILE the other CTAs are still indexing, so
+// the link is busy during KQ instead of only during KM (the host threads stream the
+// requests as KQ writes them).  Warp 0 of CTA 0 mirrors the host threads' ready words into
+// ha_seen (as KM's poller does); every other warp copies its static share of each width
+// class's blocks (class-local block b = w, w + W, ...) as they become ready, and publishes
+// ha_hseen[kb] = epoch; KM then reads those rows from HBM.  The batch's block counts are
+// known once the last lookup CTA has rung the doorbell (ctl->kq_end = epoch); the fetch
+// CTAs stop at the host share (hcut) or give up (ha_abort) when the host threads stall, and
+// KM fetches whatever is not in HBM exactly as without early fetch.
+constexpr unsigned long long kKfStallNs = 150000;
 template <int MAXT>
 __device__ __noinline__ void kq_fetch(const QArgs<MAXT>& qa, const Dev& dv) {
   const int lane = threadIdx.x & 31;
   const uint32_t w = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
-  const uint32_t nwk = (uint32_t)qa.nfetch * (blockDim.x >> 5) - 1u;  // fetch warps
+  const uint32_t nwk = (uint32_t)qa.nfetch * (blockDim.x >> 5) - 1u;  // copy warps
   const uint32_t epoch = *(volatile uint32_t*)&dv.ctl->epoch;
-  const uint32_t frac = *(volatile uint32_t*)&dv.ctl->ha_frac_q16;  // this batch's split (changes only in KM)
   const int par = epoch & 1u;
   const int ncls = qa.ncls;
   const uint32_t* ready = dv.ha_ready + (size_t)par * dv.ha_blk_cap;
   const float* stage = dv.ha_stage + (size_t)par * dv.ha_stage_floats;
   float* hstage = dv.ha_hstage + (size_t)par * dv.ha_stage_floats;
-  auto done = [&]() {
-    return ld_acquire_gpu_u32(&dv.ctl->kq_end) == epoch || *(volatile uint32_t*)&dv.ctl->ha_abort == epoch;
+  // the batch's host share per class, once every lookup CTA has finished (0xFFFFFFFF before)
+  auto share = [&](int c, bool& known, bool& active) -> uint32_t {
+    if (ld_acquire_gpu_u32(&dv.ctl->kq_end) != epoch) {
+      known = false;
+      return 0xFFFFFFFFu;
+    }
+    known = true;
+    active = *(volatile uint32_t*)&dv.ctl->ha_rung == epoch;
+    if (!active || !dv.ha_kf_tail) return 0u;  // default: stop with the lookups (KM takes the rest)
+    const uint32_t cnt = *(volatile uint32_t*)&dv.ctl->counts[par][c];
+    return ha_hcut(cnt, dv.ha_rcap[c], *(volatile uint32_t*)&dv.ctl->ha_frac_q16);
   };
-  if (w == 0) {  // the poller: host blocks' ready words -> ha_seen (a window of 128 blocks per class ahead)
-    if (!frac) return;
+  if (w == 0) {  // the poller: ready words -> ha_seen (a window of 128 blocks per class ahead)
     uint32_t lo[8];
 #pragma unroll
-    for (int c = 0; c < 8; ++c) lo[c] = 0;  // class-local: blocks below lo[c] mirrored (or the GPU's)
-    while (!done()) {
+    for (int c = 0; c < 8; ++c) lo[c] = 0;  // class-local: blocks below lo[c] mirrored
+    unsigned long long t_prog = globaltimer_ns();
+    while (true) {
+      if (*(volatile uint32_t*)&dv.ctl->ha_abort == epoch) return;
+      bool known = false, active = true, left = false, fresh = false;
 #pragma unroll 1
       for (int c = 0; c < ncls; ++c) {
-        const uint32_t b0 = dv.ha_rbase[c] / kHaBlock, nb = dv.ha_rcap[c] / kHaBlock;
+        const uint32_t b0 = dv.ha_rbase[c] / kHaBlock, nb = min(share(c, known, active), dv.ha_rcap[c] / kHaBlock);
         if (lo[c] >= nb) continue;
+        left = true;
         const uint32_t b = lo[c] + 4u * lane;
         uint32_t v[4];
 #pragma unroll
         for (int q = 0; q < 4; ++q)
-          v[q] = (b + q < nb && b + q < lo[c] + 128u && ha_host_blk(b + q, frac) &&
-                  ld_acquire_gpu_u32(dv.ha_seen + b0 + b + q) != epoch)
+          v[q] = (b + q < nb && b + q < lo[c] + 128u && ld_acquire_gpu_u32(dv.ha_seen + b0 + b + q) != epoch)
                      ? ld_relaxed_sys_u32(ready + b0 + b + q)
-                     : ~0u;
+                     : epoch;
         unsigned newly = 0;
 #pragma unroll
         for (int q = 0; q < 4; ++q)
-          if (v[q] == epoch) newly |= 1u << q;
+          if (b + q < nb && b + q < lo[c] + 128u && v[q] == epoch) newly |= 1u << q;
         if (__any_sync(kFull, newly)) {
           asm volatile("fence.acq_rel.sys;" ::: "memory");  // the rows staged before these ready words
 #pragma unroll
@@ -785,99 +770,77 @@ __device__ __noinline__ void kq_fetch(const QArgs<MAXT>& qa, const Dev& dv) {
 #endif
             }
         }
-        // advance past the prefix that is mirrored (or the GPU's)
-        bool all = true;
-#pragma unroll
-        for (int q = 0; q < 4; ++q) all = all && (v[q] == ~0u || v[q] == epoch);
-        const unsigned a4 = __ballot_sync(kFull, all);
-        lo[c] = min(nb, lo[c] + (a4 == kFull ? 128u : 4u * (uint32_t)(__ffs(~a4) - 1)));
+        // advance past the mirrored prefix
+        const unsigned all4 = __ballot_sync(kFull, b >= nb || b >= lo[c] + 128u ||
+                                                       (v[0] == epoch && v[1] == epoch && v[2] == epoch && v[3] == epoch));
+        const uint32_t adv = all4 == kFull ? 128u : 4u * (uint32_t)(__ffs(~all4) - 1);
+        if (adv) fresh = true;
+        lo[c] = min(nb, lo[c] + adv);
+        if (lo[c] < nb) left = true;
+      }
+      if (!left && known) return;
+      if (known && !active) return;
+      const unsigned long long now = globaltimer_ns();
+      if (fresh) t_prog = now;
+      if (known && now - t_prog > kKfStallNs) {  // a host thread stalled: KM takes over (zero-copy)
+        if (lane == 0) st_release_gpu_u32(&dv.ctl->ha_abort, epoch);
+        return;
       }
       __nanosleep(200);
     }
-    return;
   }
-  // fetch warps: per class, a cursor over this warp's host blocks and one over its GPU blocks
-  uint32_t curh[8], curg[8];
+  // copy warps: class-local blocks b = w - 1 + k * nwk of every class, as they become ready
+  uint32_t cur[8];
 #pragma unroll
-  for (int c = 0; c < 8; ++c) curh[c] = curg[c] = w - 1u;
+  for (int c = 0; c < 8; ++c) cur[c] = w - 1u;
   while (true) {
+    if (*(volatile uint32_t*)&dv.ctl->ha_abort == epoch) return;
     bool left = false, progressed = false;
 #pragma unroll 1
     for (int c = 0; c < ncls; ++c) {
-      const uint32_t nb = dv.ha_rcap[c] / kHaBlock, b0 = dv.ha_rbase[c] / kHaBlock;
+      bool known = false, active = true;
+      const uint32_t nb = min(share(c, known, active), dv.ha_rcap[c] / kHaBlock);
+      if (cur[c] >= nb) continue;
+      left = true;
+      const uint32_t kb = dv.ha_rbase[c] / kHaBlock + cur[c];
+      if (ld_acquire_gpu_u32(dv.ha_seen + kb) != epoch) continue;
+      // the block's rows: host staging -> HBM (row stride ha_row_floats, class width D)
       const int D = qa.cls_dim[c];
-      const uint32_t vec = (uint32_t)D / 4u;
-      // next block of each kind
-      while (curh[c] < nb && !ha_host_blk(curh[c], frac)) curh[c] += nwk;
-      while (curg[c] < nb && ha_host_blk(curg[c], frac)) curg[c] += nwk;
-      if (curh[c] < nb) {
-        left = true;
-        const uint32_t kb = b0 + curh[c];
-        if (ld_acquire_gpu_u32(dv.ha_seen + kb) == epoch) {  // published: host staging -> HBM
-          const uint32_t n4 = (uint32_t)kHaBlock * vec;
-          const size_t base = (size_t)kb * kHaBlock * dv.ha_row_floats;
-          bool quit = false;
+      const uint32_t vec = (uint32_t)D / 4u, n4 = (uint32_t)kHaBlock * vec;
+      const size_t base = (size_t)kb * kHaBlock * dv.ha_row_floats;
+      bool quit = false;
 #pragma unroll 1
-          for (uint32_t q0 = 0; q0 < n4; q0 += 32u * 8u) {
-            if (done()) {
-              quit = true;
-              break;
-            }
-            float4 v[8];
+      for (uint32_t q0 = 0; q0 < n4; q0 += 32u * 8u) {
+        if (!dv.ha_kf_tail && ld_acquire_gpu_u32(&dv.ctl->kq_end) == epoch) {  // lookups done: KM takes over
+          quit = true;
+          break;
+        }
+        float4 v[8];
 #pragma unroll
-            for (int i = 0; i < 8; ++i) {
-              const uint32_t q = q0 + 32u * i + lane;
-              v[i] = q < n4 ? ld_cv_v4(stage + base + (size_t)(q / vec) * dv.ha_row_floats + 4u * (q % vec))
-                            : make_float4(0.f, 0.f, 0.f, 0.f);
-            }
+        for (int i = 0; i < 8; ++i) {
+          const uint32_t q = q0 + 32u * i + lane;
+          v[i] = q < n4 ? ld_cv_v4(stage + base + (size_t)(q / vec) * dv.ha_row_floats + 4u * (q % vec))
+                        : make_float4(0.f, 0.f, 0.f, 0.f);
+        }
 #pragma unroll
-            for (int i = 0; i < 8; ++i) {
-              const uint32_t q = q0 + 32u * i + lane;
-              if (q < n4) st_v4(hstage + base + (size_t)(q / vec) * dv.ha_row_floats + 4u * (q % vec), v[i]);
-            }
-          }
-          __syncwarp();
-          if (quit) return;
-          if (lane == 0) {
-            __threadfence();
-            st_release_gpu_u32(dv.ha_hseen + kb, epoch);
-#ifdef FLECHE_EXPERIMENTS
-            if (dv.exp_blk) dv.exp_blk[kb * 8 + 5] = globaltimer_ns();
-#endif
-          }
-          curh[c] += nwk;
-          progressed = true;
+        for (int i = 0; i < 8; ++i) {
+          const uint32_t q = q0 + 32u * i + lane;
+          if (q < n4) st_v4(hstage + base + (size_t)(q / vec) * dv.ha_row_floats + 4u * (q % vec), v[i]);
         }
       }
-      if (dv.ha_kf_gpu && curg[c] < nb) {
-        left = true;
-        const uint32_t kb = b0 + curg[c];
-        // the block's 64 misses, 32 at a time (lane = row), once KQ has found them all
-        const FetchRec* fr = dv.ha_frec + (size_t)kb * kHaBlock;
-        uint4 r0 = ld_cg_v4u((const uint32_t*)(fr + lane)), r1 = ld_cg_v4u((const uint32_t*)(fr + 32 + lane));
-        if (__all_sync(kFull, r0.z == epoch && r1.z == epoch)) {
-#pragma unroll 1
-          for (int h = 0; h < 2; ++h) {
-            const uint4 r = h ? r1 : r0;
-            const TableInfo* ti = dv.tables + (int32_t)r.y;
-            const float* src = ti->host + (size_t)(r.x - ti->base) * (size_t)D;  // the unified index: computed host address
-            float* dst = hstage + ((size_t)kb * kHaBlock + h * 32 + lane) * dv.ha_row_floats;
-            gather_dispatch(src, dst, D, true, lane);
-          }
-          __syncwarp();
-          if (lane == 0) {
-            __threadfence();
-            st_release_gpu_u32(dv.ha_hseen + kb, epoch);
+      __syncwarp();
+      if (quit) return;
+      if (lane == 0) {
+        __threadfence();
+        st_release_gpu_u32(dv.ha_hseen + kb, epoch);
 #ifdef FLECHE_EXPERIMENTS
-            if (dv.exp_blk) dv.exp_blk[kb * 8 + 5] = globaltimer_ns();
+        if (dv.exp_blk) dv.exp_blk[kb * 8 + 5] = globaltimer_ns();
 #endif
-          }
-          curg[c] += nwk;
-          progressed = true;
-        }
       }
+      cur[c] += nwk;
+      progressed = true;
     }
-    if (!left || done()) return;
+    if (!left) return;
     if (!progressed) __nanosleep(200);
   }
 }
@@ -929,8 +892,7 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
 #endif
   if (dv.ha && bid == 0 && threadIdx.x == 0)  // the host threads start streaming this batch's requests
     asm volatile("st.relaxed.sys.global.u64 [%0], %1;" ::"l"(dv.ha_start),
-                 "l"(((unsigned long long)*(volatile uint32_t*)&dv.ctl->ha_frac_q16 << 32) |
-                     (unsigned long long)*(volatile uint32_t*)&dv.ctl->epoch)
+                 "l"((unsigned long long)*(volatile uint32_t*)&dv.ctl->epoch)
                  : "memory");
   __syncthreads();
 
@@ -1124,19 +1086,15 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
         const uint32_t r = b + __popc(grp & lt);  // the miss's index within its width class
         const int64_t li = qa.cls_off[cls] + r;    // miss-list index
         // host-assisted: staging row ha_rbase[cls] + r (one request slot each); a class's
-        // misses past its ha_rcap rows are read zero-copy (see ha_host_blk for the split)
+        // misses past its ha_rcap rows are read zero-copy (see ha_hcut for the ownership)
         const bool staged = dv.ha && r < dv.ha_rcap[cls];
         const uint32_t srow = staged ? dv.ha_rbase[cls] + r : 0u;
         if (staged) hst = (uint64_t)srow * dv.ha_row_floats;
-        dv.miss[li] = MissRec{off, fk, scr, qa.t0 + t, (int32_t)epoch, hst};  // pad: epoch tag (early readers)
+        dv.miss[li] = MissRec{off, fk, scr, qa.t0 + t, 0, hst};
         dv.owner_off[scr] = off;
 #ifdef FLECHE_EXPERIMENTS
         if (dv.exp_mode != 4)
 #endif
-        if (staged && qa.nfetch && dv.ha_kf_gpu)  // the early fetch warps' copy of the miss (HBM, one 16-byte store)
-          asm volatile("st.global.cg.v4.u32 [%0], {%1, %2, %3, %4};" ::"l"(dv.ha_frec + srow), "r"(fk),
-                       "r"(qa.t0 + t), "r"(epoch), "r"(0u)
-                       : "memory");
         if (staged)  // the host threads' request, tagged with the epoch (no fence needed)
         {
           const HaReq rq = ha_req_make(qa.t0 + t, id, hst, epoch);
@@ -1215,9 +1173,9 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
           hd.epoch = epoch;
           for (int c = 0; c < 8; ++c) {
             hd.cnt[c] = cnt[c];
-            hd.nblk[c] = c < qa.ncls ? ha_nblk(cnt[c], dv.ha_rcap[c]) : 0u;
+            hd.hcut[c] = c < qa.ncls ? ha_hcut(cnt[c], dv.ha_rcap[c], frac) : 0u;
           }
-          hd.frac = frac;
+          hd.pad = 0;
           hd.epoch2 = epoch;
           dv.ha_desc[par] = hd;  // no system fence: the host re-reads until both epoch fields match
           asm volatile("st.relaxed.sys.global.u64 [%0], %1;" ::"l"(dv.ha_bell), "l"((unsigned long long)epoch) : "memory");
@@ -1453,7 +1411,7 @@ __device__ __forceinline__ void km_ha(const Dev& dv, float* __restrict__ out, co
                                       uint32_t epoch, uint32_t nmiss, int lane, uint32_t gw, uint32_t nw, unsigned& ins,
                                       unsigned& ev, unsigned& byp, long long& docc, unsigned long long& hostb,
                                       float4* hsm, float4* cbuf, unsigned& harows, unsigned& hato, int cls,
-                                      uint32_t nblk, uint32_t frac) {
+                                      uint32_t hcut) {
   constexpr int VEC = D / 4;
   constexpr int ROWS0 = (kHaSmemF4 / VEC) < kHaBlock ? (kHaSmemF4 / VEC) : kHaBlock;  // rows that fit the warp's smem
   constexpr int ROWS = ROWS0 < 16 ? ROWS0 : 16;  // rows per piece: one warp per piece, pieces of a block in parallel
@@ -1464,7 +1422,7 @@ __device__ __forceinline__ void km_ha(const Dev& dv, float* __restrict__ out, co
   const float* hstage = dv.ha_hstage ? dv.ha_hstage + (size_t)(epoch & 1u) * dv.ha_stage_floats : nullptr;
   // work unit = pieces of this class's miss list (class-local index j; a piece never
   // straddles a 64-row staging block): a staged piece starts as soon as its block is
-  // ready, and the zero-copy pieces (the GPU's blocks, or past the class's staging rows) get
+  // ready, and the zero-copy pieces (blocks >= hcut, or past the class's staging rows) get
   // the whole grid's memory-level parallelism, not one warp per 64 rows.  Pieces per
   // unit: as fine as the grid allows (one piece per warp while there are enough warps,
   // cfg2 +8 %), coarser for big batches (cfg5 +8 %); FLECHE_HA_UNIT_PIECES fixes it (A/B)
@@ -1481,10 +1439,10 @@ __device__ __forceinline__ void km_ha(const Dev& dv, float* __restrict__ out, co
 #ifdef FLECHE_EXPERIMENTS
     if (dv.exp_blk && lane == 0 && pc == 0) dv.exp_blk[kb * 8 + 0] = globaltimer_ns();
 #endif
-    if (lane == 0 && blo < rcap && hb < nblk) {  // a staged block
+    if (lane == 0 && blo < rcap && hb < hcut) {  // the host threads' share; the rest from the tables
       if (dv.ha_hstage && ld_acquire_gpu_u32(dv.ha_hseen + kb) == epoch) {
-        ok = 2;  // early fetch already moved the block's rows into HBM
-      } else if (ha_host_blk(hb, frac)) {  // the host threads' block; the GPU's own blocks: from the tables
+        ok = 2;  // early fetch already moved the block into HBM
+      } else {
         ok = ha_wait_block(dv, epoch, kb);
         if (!ok && pc == 0) ++hato;
       }
@@ -1846,9 +1804,9 @@ __global__ void __launch_bounds__(128, 4) km_kernel(const __grid_constant__ Dev 
     hd.epoch = epoch;
     for (int c = 0; c < 8; ++c) {
       hd.cnt[c] = c < ka.ncls ? *(volatile uint32_t*)&dv.ctl->counts[par][c] : 0u;
-      hd.nblk[c] = c < ka.ncls ? ha_nblk(hd.cnt[c], dv.ha_rcap[c]) : 0u;
+      hd.hcut[c] = c < ka.ncls ? ha_hcut(hd.cnt[c], dv.ha_rcap[c], frac) : 0u;
     }
-    hd.frac = frac;
+    hd.pad = 0;
     hd.epoch2 = epoch;
     dv.ha_desc[par] = hd;
     __threadfence_system();
@@ -1872,12 +1830,11 @@ __global__ void __launch_bounds__(128, 4) km_kernel(const __grid_constant__ Dev 
     if (poller) {
       HaBlocks hb;
       hb.ncls = ka.ncls;
-      hb.frac = frac;
 #pragma unroll
       for (int c = 0; c < 8; ++c) {
         const uint32_t cnt = c < ka.ncls ? *(volatile uint32_t*)&dv.ctl->counts[par][c] : 0u;
         hb.lo[c] = dv.ha_rbase[c] / kHaBlock;
-        hb.n[c] = c < ka.ncls ? ha_nblk(cnt, dv.ha_rcap[c]) : 0u;
+        hb.n[c] = c < ka.ncls ? ha_hcut(cnt, dv.ha_rcap[c], frac) : 0u;
       }
       ha_poll(dv, epoch, hb, lane);
     }
@@ -1891,7 +1848,7 @@ __global__ void __launch_bounds__(128, 4) km_kernel(const __grid_constant__ Dev 
 #define FL_KM(D)                                                                                              \
   if (use_ha)                                                                                                 \
     km_ha<BYTES, D>(dv, ka.out, ml, epoch, nmiss, lane, gw, nw, ins, ev, byp, docc, hostb, hsm, wsm, harows, hato, c,  \
-                    ha_nblk(nmiss, dv.ha_rcap[c]), frac);                                                   \
+                    ha_hcut(nmiss, dv.ha_rcap[c], frac));                                                   \
   else                                                                                                        \
     km_rows<BYTES, D, KmM<BYTES, D>::value>(dv, ka.out, ml, epoch, nmiss, lane, gw, nw, ins, ev, byp, docc, hostb, wsm)
     if constexpr (DU > 0) {
