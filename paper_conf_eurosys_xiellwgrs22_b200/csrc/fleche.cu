@@ -88,6 +88,7 @@ struct fleche_ctx {
   int kq_tma = 0;      // KQ's hit gather by bulk copies through shared memory (row width 32 or 64; 0 = registers)
   size_t kq_smem = 0;  // its dynamic shared memory (4 warps x 32 rows)
   int kf_ctas = 0;     // host-assisted early fetch: KQ CTAs that copy staged blocks into HBM (0 = off)
+  int fwd_ctas = 0;    // host-assisted request forwarding: KQ CTAs that move requests to the host (0 = off)
   // ... from this many lookups per batch (FLECHE_HA_EARLY_MIN): a short KQ ends before the
   // host threads have staged much (cfg2, 213K lookups: 111 vs 106 us per batch without;
   // cfg5, 1.7M: 495 vs 570 us, profiles/)
@@ -376,13 +377,12 @@ void ha_worker(HostAssist* h, int me) {
         t_d = now_ns();
       }
     };
-    // request i of this batch, if it has arrived (KQ wrote it without a system fence: both
-    // halves must carry this batch's tags, and a second read must agree -- never torn)
+    // request i of this batch, if it has arrived (KQ wrote it without a system fence: each
+    // 8-byte half is written and read whole, and both carry this batch's tags, so a request
+    // still in flight -- or a read that caught only one half -- is never taken)
     auto fetch = [&](uint64_t i, HaReq* out) -> bool {
       HaReq a{rq[i].tid, rq[i].stage};
       if (!ha_req_current(a, e)) return false;
-      HaReq b2{rq[i].tid, rq[i].stage};
-      if (b2.tid != a.tid || b2.stage != a.stage) return false;
       *out = a;
       return true;
     };
@@ -511,7 +511,7 @@ void free_all(fleche_ctx* c) {
                   c->dv.miss, c->dv.dup, c->dv.ctl, c->dv.stats, c->d_tables, c->d_ids_stage, c->d_out_stage,
                   c->d_pool_stage, c->d_kdec, c->rd.scratch, c->rd.slotval, c->rd.inv, c->rd.region, c->rd.cnt,
                   c->rd.prefix, c->rd.done, c->rd.stats, c->d_slots, c->d_age_hist, c->d_prefill_out,
-                  c->d_out_stage2, c->dv.ha_seen, c->dv.ha_hstage, c->dv.ha_hseen};
+                  c->d_out_stage2, c->dv.ha_seen, c->dv.ha_hstage, c->dv.ha_hseen, c->dv.ha_reqd};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   for (auto& r : c->registered) cudaHostUnregister(r.first);
@@ -658,7 +658,8 @@ fleche_status launch_query(fleche_ctx* c, const int64_t* const* ids, const int64
   for (int k = 0; k < ka.ncls; ++k) qa.cls_dim[k] = c->cls_dim[k];
   if (total > 0 && !c->per_table_launch) {
     qa.nfetch = (qa.ha_bell && !decouple && total >= c->kf_min) ? c->kf_ctas : 0;
-    const int64_t blocks = (total + 127) / 128 + qa.nfetch;
+    qa.nfwd = (qa.ha_bell && c->dv.ha_reqd) ? c->fwd_ctas : 0;
+    const int64_t blocks = (total + 127) / 128 + qa.nfetch + qa.nfwd;
     launch_k(kPdlKQ, kq_fn<MAXT>(c->kq_tma), (unsigned)blocks, 128, c->kq_smem, s, qa, c->dv);
     c->kernels++;
     if (decouple) {  // fork: the hit copy runs on the side stream, concurrently with KM
@@ -1056,6 +1057,11 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out) {
       return fail(FLECHE_ENOMEM);
     // early fetch (FLECHE_HA_EARLY=0 turns it off): KQ's first kf_ctas CTAs move staged
     // blocks into an HBM copy while the lookups run
+    // request forwarding (FLECHE_HA_FWD = CTAs, 0 = KQ's lanes write the host list directly)
+    c->fwd_ctas = (int)std::min<uint64_t>(64, env_u("FLECHE_HA_FWD", 8));
+    if (c->fwd_ctas && (cudaMalloc((void**)&dv.ha_reqd, sizeof(HaReq) * (size_t)h->req_cap) != cudaSuccess ||
+                        cudaMemset(dv.ha_reqd, 0, sizeof(HaReq) * (size_t)h->req_cap) != cudaSuccess))
+      return fail(FLECHE_ENOMEM);
     c->kf_ctas = (int)env_u("FLECHE_HA_EARLY", 1) ? (int)std::min<uint64_t>(64, std::max<uint64_t>(1, env_u("FLECHE_KF_CTAS", 16))) : 0;
     dv.ha_kf_tail = (uint32_t)env_u("FLECHE_KF_TAIL", 0);
     c->kf_min = (int64_t)env_u("FLECHE_HA_EARLY_MIN", 524288);

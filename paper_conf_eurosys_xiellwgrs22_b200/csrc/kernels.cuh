@@ -58,7 +58,10 @@ constexpr uint32_t kSlotMiss = 0xFFFFFFFFu, kSlotZero = 0xFFFFFFFEu;  // KQ -> K
 constexpr int kKmWarps = 4;     // KM CTA = 4 warps
 constexpr int kKmStageF4 = 256; // bytes layout, per warp: staged rows of a chunk (<= 4 KB) ...
 constexpr int kKmSmemF4 = 512;  // ... + the compaction buffer of one set region (<= 4 KB)
-constexpr int kHaBlock = 64;    // host-assisted miss fetch: rows per staging block
+#ifndef FL_HA_BLOCK
+#define FL_HA_BLOCK 64
+#endif
+constexpr int kHaBlock = FL_HA_BLOCK;  // host-assisted miss fetch: rows per staging block
 constexpr int kHaMaxThreads = 16;  // host-assisted: at most this many host threads
 constexpr int kHaSmemF4 = 512;  // host-assisted KM, per warp: 8 KB of rows landed from the host (4 KM CTAs per SM)
 
@@ -142,8 +145,10 @@ struct Ctl {
   unsigned long long win_ns;   // current window: KM time summed
   unsigned long long win_miss; //   unique misses summed
   uint32_t win_n;              //   batches
-  uint32_t tune_pad;
-  double prev_cost;            // ns per unique miss of the previous window (growing) / at the peak (paused)       // watermark eviction: occ_bytes as KE1 saw it (KE2's one snapshot per scan)
+  uint32_t tune_since;         // paused: windows since the last probe
+  double prev_cost;            // ns per unique miss of the previous window (growing) / at the peak (paused)
+  uint32_t tune_best;          // probing: the share to return to
+  int32_t tune_dir;            // probing: direction of the next probe (+1 / -1 share step)       // watermark eviction: occ_bytes as KE1 saw it (KE2's one snapshot per scan)
 };
 
 // Host-assisted miss fetch (FLECHE_FLAG_HOST_ASSIST): the CPU-DRAM layer's threads
@@ -224,6 +229,7 @@ struct Dev {
   uint32_t* ha_seen;           // [ha_blk_cap] (HBM) the poller warp's mirror of ha_ready[epoch & 1]
   float* ha_stage;             // [2][ha_stage_floats]
   float* ha_hstage;            // early fetch: [2][ha_stage_floats] (HBM) copy of the staged blocks
+  HaReq* ha_reqd;              // request forwarding: [ha_req_cap] (HBM) KQ's requests before they go to the host
   uint32_t* ha_hseen;          // early fetch: [ha_blk_cap] (HBM) epoch once a block's rows are in ha_hstage
   uint32_t ha_req_cap, ha_blk_cap;  // staging rows (= request slots) and blocks per epoch parity
   uint32_t ha_rbase[8];        // first staging row of width class c (a multiple of kHaBlock)
@@ -265,6 +271,8 @@ struct QArgs {
   const int64_t* dcnt;       // key-sharded sync-free: [n][n] routed-count matrix in device memory
   int32_t dme;               //   this rank (segment i's count = dcnt[i * n + dme])
   int32_t nfetch;            // early fetch: CTAs 0..nfetch-1 copy staged blocks into HBM (kq_fetch)
+  int32_t nfwd;              // request forwarding: the next nfwd CTAs move requests to the host (kq_forward)
+  int32_t pad4;
   int32_t cls_dim[8];        //   (row width of each class)
 };
 
@@ -701,6 +709,73 @@ __device__ __forceinline__ void bulk_s2g(void* gmem, const void* smem, unsigned 
   asm volatile("cp.async.bulk.commit_group;" ::: "memory");
 }
 
+// Request forwarding (host-assisted): KQ's owner lanes write their 16-byte requests into HBM
+// and qa.nfwd CTAs of KQ move them to the host threads' pinned request list a staging block
+// (64 requests, 1 KiB) at a time, coalesced.  The lookups themselves then never store to
+// system memory: scattered 16-byte posted writes over the link cost KQ +6 us at cfg2 and
+// +100 us at cfg4, and on some boxes of the pool they stalled whole KQ launches for 0.2-0.4
+// ms (ncu launch list, profiles/r02b).  A forwarder warp takes class-local blocks w, w + W,
+// ...: a block goes once all its requests carry this batch's tags (the last partial block
+// once the last lookup CTA has published the counts, ctl->kq_end); the host threads wait on
+// the same tags, so nothing else changes for them.  Bounded: after the counts are known, a
+// block that makes no progress for kFwdStallNs is left to the host threads' own timeout.
+constexpr unsigned long long kFwdStallNs = 200000;
+template <int MAXT>
+__device__ __forceinline__ void kq_forward(const QArgs<MAXT>& qa, const Dev& dv) {
+  const int lane = threadIdx.x & 31;
+  const uint32_t W = (uint32_t)qa.nfwd * (blockDim.x >> 5);
+  const uint32_t w = (blockIdx.x - (uint32_t)qa.nfetch) * (blockDim.x >> 5) + (threadIdx.x >> 5);
+  const uint32_t epoch = *(volatile uint32_t*)&dv.ctl->epoch;
+  const int par = epoch & 1u;
+  HaReq* hreq = dv.ha_req + (size_t)par * dv.ha_req_cap;
+  uint32_t cur[8];
+#pragma unroll
+  for (int c = 0; c < 8; ++c) cur[c] = w;
+  unsigned long long t_prog = 0;
+  while (true) {
+    const bool known = ld_acquire_gpu_u32(&dv.ctl->kq_end) == epoch;
+    if (known && *(volatile uint32_t*)&dv.ctl->ha_rung != epoch) return;  // not a host-assisted batch
+    bool left = false, prog = false;
+#pragma unroll 1
+    for (int c = 0; c < qa.ncls; ++c) {
+      const uint32_t rcap = dv.ha_rcap[c];
+      const uint32_t nrow = known ? min(*(volatile uint32_t*)&dv.ctl->counts[par][c], rcap) : rcap;
+      const uint32_t nb = known ? (nrow + kHaBlock - 1) / kHaBlock : rcap / kHaBlock;
+      if (cur[c] >= nb) continue;
+      left = true;
+      const uint32_t lim = known ? min((uint32_t)kHaBlock, nrow - cur[c] * kHaBlock) : (uint32_t)kHaBlock;
+      const size_t r0 = (size_t)dv.ha_rbase[c] + (size_t)cur[c] * kHaBlock;
+      bool ok = true;
+      HaReq q[kHaBlock / 32 > 0 ? kHaBlock / 32 : 1];
+#pragma unroll
+      for (int h = 0; h < (kHaBlock + 31) / 32; ++h) {
+        const uint32_t i = h * 32 + lane;
+        if (i < lim) {
+          asm volatile("ld.global.cg.v2.u64 {%0, %1}, [%2];" : "=l"(q[h].tid), "=l"(q[h].stage) : "l"(dv.ha_reqd + r0 + i));
+          ok = ok && ha_req_current(q[h], epoch);
+        }
+      }
+      if (__all_sync(kFull, ok)) {
+#pragma unroll
+        for (int h = 0; h < (kHaBlock + 31) / 32; ++h) {
+          const uint32_t i = h * 32 + lane;
+          if (i < lim)
+            asm volatile("st.global.v2.u64 [%0], {%1, %2};" ::"l"(hreq + r0 + i), "l"(q[h].tid), "l"(q[h].stage) : "memory");
+        }
+        cur[c] += W;
+        prog = true;
+      }
+    }
+    if (!left) return;
+    if (known) {
+      const unsigned long long now = globaltimer_ns();
+      if (prog || !t_prog) t_prog = now;
+      else if (now - t_prog > kFwdStallNs) return;
+    }
+    if (!prog) __nanosleep(100);
+  }
+}
+
 // Early fetch (host-assisted): the first qa.nfetch CTAs of KQ do no lookups; they move the
 // batch's staged blocks over the link into HBM WHILE the other CTAs are still indexing, so
 // the link is busy during KQ instead of only during KM (the host threads stream the
@@ -713,7 +788,7 @@ __device__ __forceinline__ void bulk_s2g(void* gmem, const void* smem, unsigned 
 // KM fetches whatever is not in HBM exactly as without early fetch.
 constexpr unsigned long long kKfStallNs = 150000;
 template <int MAXT>
-__device__ __noinline__ void kq_fetch(const QArgs<MAXT>& qa, const Dev& dv) {
+__device__ __forceinline__ void kq_fetch(const QArgs<MAXT>& qa, const Dev& dv) {
   const int lane = threadIdx.x & 31;
   const uint32_t w = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
   const uint32_t nwk = (uint32_t)qa.nfetch * (blockDim.x >> 5) - 1u;  // copy warps
@@ -845,6 +920,14 @@ __device__ __noinline__ void kq_fetch(const QArgs<MAXT>& qa, const Dev& dv) {
   }
 }
 
+// KQ's side CTAs: [0, nfetch) early fetch, [nfetch, nfetch + nfwd) request forwarding (one
+// call site, so the lookup path keeps its registers)
+template <int MAXT>
+__device__ __forceinline__ void kq_side(const QArgs<MAXT>& qa, const Dev& dv) {
+  if ((int)blockIdx.x < qa.nfetch) kq_fetch<MAXT>(qa, dv);
+  else kq_forward<MAXT>(qa, dv);
+}
+
 // TD > 0: hit rows gathered with bulk copies through TD-float shared-memory rows (one row
 // width for every table; dynamic shared memory = 4 warps x 32 rows x TD floats).
 template <int MAXT, int TD>
@@ -860,8 +943,8 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   pdl_wait();  // the previous batch (or the caller's producer of ids) has completed
-  if ((int)blockIdx.x < qa.nfetch) {  // early-fetch CTA (no lookups)
-    kq_fetch<MAXT>(qa, dv);
+  if ((int)blockIdx.x < qa.nfetch + qa.nfwd) {  // early-fetch / request-forwarding CTA (no lookups)
+    kq_side<MAXT>(qa, dv);
 #ifdef FLECHE_EXPERIMENTS
     if (dv.exp_buf && (threadIdx.x & 31) == 0 && blockIdx.x * 4 + threadIdx.x / 32 < 256) {
       const unsigned long long tx = globaltimer_ns();
@@ -871,7 +954,8 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
 #endif
     return;
   }
-  const uint32_t bid = blockIdx.x - (uint32_t)qa.nfetch, nbid = gridDim.x - (uint32_t)qa.nfetch;  // lookup CTAs
+  const uint32_t nside = (uint32_t)(qa.nfetch + qa.nfwd);
+  const uint32_t bid = blockIdx.x - nside, nbid = gridDim.x - nside;  // lookup CTAs
   if (qa.dcnt && threadIdx.x == 0) {
     // key-sharded, sync-free: segment i's count is C[i][me] of the routed-count matrix in
     // device memory (written by the collective the stream ran before this launch)
@@ -1098,9 +1182,13 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
         if (staged)  // the host threads' request, tagged with the epoch (no fence needed)
         {
           const HaReq rq = ha_req_make(qa.t0 + t, id, hst, epoch);
-          asm volatile("st.global.v2.u64 [%0], {%1, %2};" ::"l"(dv.ha_req + (size_t)par * dv.ha_req_cap + srow),
-                       "l"(rq.tid), "l"(rq.stage)
-                       : "memory");
+          if (qa.nfwd)  // to HBM; KQ's forwarder CTAs move it to the host in 1 KiB blocks
+            asm volatile("st.global.cg.v2.u64 [%0], {%1, %2};" ::"l"(dv.ha_reqd + srow), "l"(rq.tid), "l"(rq.stage)
+                         : "memory");
+          else
+            asm volatile("st.global.v2.u64 [%0], {%1, %2};" ::"l"(dv.ha_req + (size_t)par * dv.ha_req_cap + srow),
+                         "l"(rq.tid), "l"(rq.stage)
+                         : "memory");
         }
       }
     }
@@ -1181,7 +1269,7 @@ __global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_
           asm volatile("st.relaxed.sys.global.u64 [%0], %1;" ::"l"(dv.ha_bell), "l"((unsigned long long)epoch) : "memory");
           *(volatile uint32_t*)&dv.ctl->ha_rung = epoch;
         }
-        if (qa.nfetch) st_release_gpu_u32(&dv.ctl->kq_end, epoch);  // the fetch CTAs: counts are final
+        if (nside) st_release_gpu_u32(&dv.ctl->kq_end, epoch);  // the fetch / forward CTAs: counts are final
 #ifdef FLECHE_EXPERIMENTS
         if (dv.exp_buf) {
           dv.exp_buf[dv.exp_slots + 2] = globaltimer_ns();
@@ -1748,18 +1836,26 @@ struct KmM {
 // blocks, 1 - ha_frac: it starts at 0 (the host threads take every block), grows by
 // kTuneStep per window of kTuneWin batches while the miss kernel's time per unique miss
 // improves, pauses one step back at the peak, and restarts from 0 when a paused window is
-// kTuneDecline slower than the peak.  Run by KM's last CTA; it changes where rows are read
-// from only, never a result.
+// kTuneDecline slower than the peak.  While paused it re-probes one step to either side every
+// kTuneProbe windows and keeps a probe that is kTuneGain faster (a single greedy climb from 0
+// stopped on one noisy window: cfg4 settled at 0.0 or 0.4 from run to run).  A window is 16
+// batches, or fewer when they are slow (at least 2 batches and 2 ms of KM time), so slow
+// configurations are tuned within a few hundred milliseconds too.  Run by KM's last CTA; it
+// changes where rows are read from only, never a result.
 constexpr uint32_t kTuneWin = 16;
+constexpr unsigned long long kTuneWinNs = 2000000;
 constexpr uint32_t kTuneStep = 6554;  // 0.1 of the blocks (x 2^-16)
 constexpr double kTuneDecline = 1.15;
+constexpr uint32_t kTuneProbe = 4;
+constexpr double kTuneGain = 0.97;
 __device__ __forceinline__ void ui_tune(const Dev& dv, uint32_t nmiss) {
   Ctl* c = dv.ctl;
   const unsigned long long t = globaltimer_ns() - c->km_t0;
   if (dv.ha_frac_fixed || nmiss < dv.ha_min_rows || t > 1000000000ull) return;
   c->win_ns += t;
   c->win_miss += nmiss;
-  if (++c->win_n < kTuneWin) return;
+  ++c->win_n;
+  if (c->win_n < kTuneWin && (c->win_n < 2 || c->win_ns < kTuneWinNs)) return;
   const double cost = (double)c->win_ns / (double)max(1ull, c->win_miss);
   c->win_ns = c->win_miss = 0;
   c->win_n = 0;
@@ -1776,10 +1872,29 @@ __device__ __forceinline__ void ui_tune(const Dev& dv, uint32_t nmiss) {
       f = min(65536u, f + kTuneStep);  // one step back: the previous share was the peak
       c->tune_phase = 1;
     }
-  } else if (cost > c->prev_cost * kTuneDecline) {  // the workload changed: clear and repeat
-    f = 65536u;
-    c->tune_phase = 0;
-    c->prev_cost = 0.0;
+    c->tune_since = 0;
+  } else if (c->tune_phase == 1) {  // paused at the peak
+    if (cost > c->prev_cost * kTuneDecline) {  // the workload changed: clear and repeat
+      f = 65536u;
+      c->tune_phase = 0;
+      c->prev_cost = 0.0;
+    } else {
+      c->prev_cost = cost;  // the peak's current cost
+      if (++c->tune_since >= kTuneProbe) {  // probe one step to one side
+        c->tune_since = 0;
+        c->tune_dir = c->tune_dir > 0 ? -1 : 1;
+        const int64_t g = (int64_t)f + (int64_t)c->tune_dir * kTuneStep;
+        if (g >= (int64_t)kTuneStep && g <= 65536) {
+          c->tune_best = f;
+          f = (uint32_t)g;
+          c->tune_phase = 2;
+        }
+      }
+    }
+  } else {  // one probe window
+    if (cost < c->prev_cost * kTuneGain) c->prev_cost = cost;  // better: the probe is the new peak
+    else f = c->tune_best;
+    c->tune_phase = 1;
   }
   c->ha_frac_q16 = f;
 }
