@@ -116,9 +116,15 @@ typedef struct {
  * over the link at its full rate while it reads the rest zero-copy itself (two paths at
  * once).  HOST_ASSIST forces it on (also for small tiers),
  * NO_HOST_ASSIST off.  Requests travel GPU -> host through pinned memory, tagged with the
- * batch epoch; the query kernel's last CTA rings the doorbell; ONE miss-kernel warp polls
- * the threads' progress words and mirrors them into HBM for the others (no host sync, no
- * extra launch: the path stays asynchronous and graph-capturable).  Blocks not staged
+ * batch epoch: the query kernel's owner lanes write them to HBM and a few side CTAs of the
+ * same launch forward them to the host list 1 KiB per staging block (FLECHE_HA_FWD = CTAs,
+ * default 8; 0 = the lanes write the host list directly); the query kernel's first CTA
+ * writes a start word (the threads stream the requests as they come) and its last CTA
+ * rings the doorbell with the counts; ONE miss-kernel warp polls the threads' progress
+ * words and mirrors them into HBM for the others (no host sync, no extra launch: the path
+ * stays asynchronous and graph-capturable).  From FLECHE_HA_EARLY_MIN lookups per batch
+ * (default 524288) 16 more side CTAs copy already staged blocks into HBM while the
+ * lookups run (FLECHE_HA_EARLY=0 turns that off).  Blocks not staged
  * within FLECHE_HA_TIMEOUT_US (default 2000) are read zero-copy from the tables, so
  * correctness never depends on the threads.  Env: FLECHE_HA_THREADS (default
  * min(12, CPUs - 4)), FLECHE_HA_STAGE_KB (staging per epoch parity, default 131072, or

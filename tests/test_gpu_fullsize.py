@@ -56,7 +56,10 @@ def test_cfg5_full_size(monkeypatch, cfg5_tables, ha):
         # the host threads idle (50 us polls) while the oracle runs between batches here, so
         # some staging blocks time out and are fetched zero-copy: allowed (values are checked
         # above), as long as the host threads still stage most of their share
-        assert 0 < dg["assisted_rows"] < dg["unique_misses"], dg
+        assert 0 < dg["assisted_rows"] <= dg["unique_misses"], dg
+        if ha == "split":  # a fixed share of 0.5 leaves half the blocks to the GPU's zero-copy reads;
+            # the tuned default may settle at any share, all-host (ui 0) included (DESIGN R25)
+            assert dg["assisted_rows"] < dg["unique_misses"], dg
         blocks = dg["unique_misses"] / 64
         assert dg["assist_timeouts"] < 0.25 * blocks, dg
 
