@@ -189,7 +189,7 @@ fleche_status fleche_create(const fleche_config* cfg, fleche_ctx** out);
  * cached, and make the next fleche_stats return FLECHE_ERANGE.  Caller owns ids and
  * out; they must stay valid until the stream has passed this call.  Enqueues 2
  * kernels on `stream` -- the query kernel (KQ: probe, hit gather, miss dedup) and the
- * miss kernel (KM: miss fetch, insert, and each owner's row to its duplicates) -- plus,
+ * miss kernel (KM, a cooperative launch: miss fetch, insert, restore of duplicate misses) -- plus,
  * only when decoupling is enabled (FLECHE_DECOUPLE_MIN lookups per batch; off by default),
  * the decoupled hit copy (KG) on a ctx-owned side stream that `stream` joins; with watermarks set (fleche_set_watermarks)
  * 2 scan kernels follow.  Never blocks the host. */
