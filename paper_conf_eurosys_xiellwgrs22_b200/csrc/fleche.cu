@@ -659,8 +659,8 @@ fleche_status launch_query(fleche_ctx* c, const int64_t* const* ids, const int64
   if (total > 0 && !c->per_table_launch) {
     qa.nfetch = (qa.ha_bell && !decouple && total >= c->kf_min) ? c->kf_ctas : 0;
     qa.nfwd = (qa.ha_bell && c->dv.ha_reqd) ? c->fwd_ctas : 0;
-    const int64_t blocks = (total + 127) / 128 + qa.nfetch + qa.nfwd;
-    launch_k(kPdlKQ, kq_fn<MAXT>(c->kq_tma), (unsigned)blocks, 128, c->kq_smem, s, qa, c->dv);
+    const int64_t blocks = (total + FL_KQ_THREADS - 1) / FL_KQ_THREADS + qa.nfetch + qa.nfwd;
+    launch_k(kPdlKQ, kq_fn<MAXT>(c->kq_tma), (unsigned)blocks, FL_KQ_THREADS, c->kq_smem, s, qa, c->dv);
     c->kernels++;
     if (decouple) {  // fork: the hit copy runs on the side stream, concurrently with KM
       FL_CUDA(c, cudaEventRecord(c->fork_ev, s));
@@ -683,7 +683,8 @@ fleche_status launch_query(fleche_ctx* c, const int64_t* const* ids, const int64
       q1.scan[0] = 0;
       q1.scan[1] = lengths[t];
       q1.out_off[0] = qa.out_off[t];
-      launch_k(kPdlKQ, kq_fn<32>(c->kq_tma), (unsigned)((lengths[t] + 127) / 128), 128, c->kq_smem, s, q1, c->dv);
+      launch_k(kPdlKQ, kq_fn<32>(c->kq_tma), (unsigned)((lengths[t] + FL_KQ_THREADS - 1) / FL_KQ_THREADS), FL_KQ_THREADS,
+               c->kq_smem, s, q1, c->dv);
       c->kernels++;
     }
   }
@@ -1526,11 +1527,13 @@ fleche_status launch_keys(fleche_ctx* c, const uint32_t* keys, int64_t count, fl
   fleche_status st = prof_event(c, s, true, 4);
   if (st != FLECHE_OK) return st;
   if (dcnt) {  // count unknown on the host: a capacity-sized, grid-strided launch (TD = 0: no TMA variant)
-    const int64_t blocks = std::min<int64_t>((c->max_lookups + 127) / 128, (int64_t)FL_KQ_MIN_BLOCKS * c->sm_count);
-    launch_k(kPdlKQ, kq_fn<MAXT>(0), (unsigned)std::max<int64_t>(1, blocks), 128, 0, s, qa, c->dv);
+    const int64_t blocks = std::min<int64_t>((c->max_lookups + FL_KQ_THREADS - 1) / FL_KQ_THREADS,
+                                             (int64_t)FL_KQ_MIN_BLOCKS * c->sm_count);
+    launch_k(kPdlKQ, kq_fn<MAXT>(0), (unsigned)std::max<int64_t>(1, blocks), FL_KQ_THREADS, 0, s, qa, c->dv);
     c->kernels++;
   } else if (count > 0) {
-    launch_k(kPdlKQ, kq_fn<MAXT>(c->kq_tma), (unsigned)((count + 127) / 128), 128, c->kq_smem, s, qa, c->dv);
+    launch_k(kPdlKQ, kq_fn<MAXT>(c->kq_tma), (unsigned)((count + FL_KQ_THREADS - 1) / FL_KQ_THREADS), FL_KQ_THREADS,
+             c->kq_smem, s, qa, c->dv);
     c->kernels++;
   }
   if ((st = prof_event(c, s, false, 0)) != FLECHE_OK) return st;

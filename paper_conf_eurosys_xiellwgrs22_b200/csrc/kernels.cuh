@@ -42,6 +42,9 @@
 #ifndef FL_KQ_TS_DEFER
 #define FL_KQ_TS_DEFER 1  // KQ consumes its timestamp-exchange result late (0 = right after it; A/B builds)
 #endif
+#ifndef FL_KQ_THREADS
+#define FL_KQ_THREADS 128  // KQ CTA size (A/B builds: 64 with FL_KQ_MIN_BLOCKS 16 = the same warps per SM, finer CTAs)
+#endif
 #ifndef FL_KQ_MIN_BLOCKS
 #define FL_KQ_MIN_BLOCKS 8  // KQ CTAs per SM the register budget must allow: 8 (64 regs, no spill) measured
                             // KQ 33.4 vs 35.5 us at 5 CTAs (profiles/bench_r01_kq_occupancy_*.json)
@@ -931,7 +934,7 @@ __device__ __forceinline__ void kq_side(const QArgs<MAXT>& qa, const Dev& dv) {
 // TD > 0: hit rows gathered with bulk copies through TD-float shared-memory rows (one row
 // width for every table; dynamic shared memory = 4 warps x 32 rows x TD floats).
 template <int MAXT, int TD>
-__global__ void __launch_bounds__(128, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_constant__ QArgs<MAXT> qa,
+__global__ void __launch_bounds__(FL_KQ_THREADS, FL_KQ_MIN_BLOCKS) kq_kernel(const __grid_constant__ QArgs<MAXT> qa,
                                                                    const __grid_constant__ Dev dv) {
   __shared__ int64_t s_scan[MAXT + 1];
   __shared__ __align__(8) unsigned long long s_mbar[4];
