@@ -16,7 +16,11 @@ from workload import configs  # noqa: E402
 nb = int(os.environ.get("NB", "3"))
 for name, kw, flags in [("uniform", dict(cache_frac=0.02, invalid_ppm=3000), 0),
                         ("mixed", dict(cache_frac=0.05, dims=[8, 16, 32, 64, 128, 8, 256]), 0),
-                        ("static", dict(cache_frac=0.05), 2)]:
+                        ("static", dict(cache_frac=0.05), 2),
+                        # host-assisted (forced, every batch): request forwarding and early-fetch side CTAs of KQ
+                        ("assisted", dict(cache_frac=0.02, invalid_ppm=3000), 8)]:
+    if name == "assisted":
+        os.environ.update(FLECHE_HA_MIN_ROWS="0", FLECHE_HA_EARLY_MIN="0", FLECHE_HA_FRAC="0.5")
     w = configs.get("cfg0").with_(batch_size=100, **kw)
     tabs = [np.ascontiguousarray(t) for t in w.make_tables()[1]]
     g = fl.FlatCache(w.cards, w.dims, tabs, w.cache_bytes, w.batch_size * w.n, 0, 1.0, 0, H.HASH_SEED, flags)
